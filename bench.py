@@ -1,0 +1,420 @@
+#!/usr/bin/env python
+"""Benchmark of the symbolic LU hot path (fill2 count -> scan -> allocate -> fill2 emit ->
+levelize) on synthetic BASELINE.json workloads.
+
+  python bench.py [--gpus N] [--steps K] [--warmup W] [--config C] [--impl ours|reference]
+
+One step = one pass of the whole hot path (SURVEY §8(a) S1-S9 minus the create-time S1/S2,
+which are timed in the e2e number) over the workload, inputs resident in HBM.  For N > 1 the
+script runs under torchrun, one rank per GPU, rows sharded (strong scaling of one matrix):
+count own rows, all-reduce counts, scan, emit own rows, allgatherv the pattern, levelize.
+Timed with CUDA events on the launching stream, K steps bracketed by barrier + synchronize,
+max over ranks.  L2 is flushed (256 MiB write) between timed steps, outside the events.
+
+Prints ONE JSON line (rank 0).  metric = fill entries/s = nnz(L+U) / step time.
+--impl reference times the CPU oracle (the only reference this tier has), bounded samples.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from inputs import gen  # noqa: E402
+
+METRIC = "fill entries/s"
+UNIT = "entries/s"
+L2_FLUSH_BYTES = 256 << 20
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--config", type=int, default=2, help="BASELINE.json configs[C-1]")
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--rule", default="u", choices=["u", "glu3"])
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--cpu-sample-stride", type=int, default=0,
+                    help="oracle sample: every s-th row (0 = auto, ~10-30 s of CPU work)")
+    ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras)")
+    return ap.parse_args()
+
+
+# --------------------------------------------------------------------------- work units
+def work_units(rp):
+    """Method work of one traversal (reading R24).
+
+    TE = sum_i row_ptr[i+1] and SV = n(n-1)/2 are exact on connected natural-order grids
+    (pinned in tests/test_oracle_pins.py); for other inputs they are upper bounds."""
+    n = len(rp) - 1
+    te = int(rp[1:].sum())
+    sv = n * (n - 1) // 2
+    return te, sv
+
+
+def alg_bytes_per_pass(te, sv, n, nnz_lu, emit):
+    """4 B per traversed edge + 1 bit visited test-and-set, 8 B offsets + 8 B
+    queue push/pop per scanned vertex; per row 4 B count (count pass) or 8 B offset read and
+    4 B per emitted entry (emit pass)."""
+    b = 4 * te + te / 8 + 16 * sv
+    if emit:
+        b += 8 * (n + 1) + 4 * nnz_lu
+    else:
+        b += 4 * n
+    return b
+
+
+# --------------------------------------------------------------------------- clocks
+REASONS = ["gpu_idle", "applications_clocks_setting", "sw_power_cap", "hw_slowdown",
+           "sync_boost", "sw_thermal_slowdown", "hw_thermal_slowdown", "hw_power_brake_slowdown",
+           "display_clock_setting"]
+
+
+class ClockSampler:
+    def __init__(self, index):
+        self.index = index
+        self.samples = []
+        self.proc = None
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index),
+                 "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+                 "utilization.gpu", "--format=csv,noheader,nounits", "-lms", "200"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception:
+            self.proc = None
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) >= 4:
+                self.samples.append(parts)
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if not self.samples:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
+        sm, mx, reasons = [], None, set()
+        for s in self.samples:
+            try:
+                c, m, r, u = float(s[0]), float(s[1]), int(s[2], 16), float(s[3])
+            except ValueError:
+                continue
+            mx = m
+            if u > 0:
+                sm.append(c)
+            for b, name in enumerate(REASONS):
+                if r & (1 << b) and name != "gpu_idle":
+                    reasons.add(name)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(self.samples)}
+
+
+# --------------------------------------------------------------------------- CPU oracle
+def cpu_oracle_sample(rp, ci, stride, rule="u"):
+    """Time the oracle (as it stands) on every stride-th row (both passes, all host cores) and
+    on the full Kahn levelization; extrapolate the symbolic time by exact TE share."""
+    import oracle
+    n = len(rp) - 1
+    rows = np.arange(n - 1, -1, -stride, dtype=np.int32)
+    threads = os.cpu_count() or 1
+    t0 = time.perf_counter()
+    r = oracle.fill2(rp, ci, rows=rows, emit=True, threads=threads)
+    t_sym = time.perf_counter() - t0
+    te_total = int(rp[1:].sum())
+    te_sample = int(r["te"].sum())
+    scale = te_total / max(te_sample, 1)
+    t_sym_full = t_sym * scale
+    return dict(rows=rows, t_sample=t_sym, t_sym_full=t_sym_full, threads=threads,
+                entries_sample=int(r["counts"].sum()), te_sample=te_sample, scale=scale)
+
+
+def cpu_levels_time(rp, ci, rule, nnz_hint=None):
+    """Full-pattern oracle Kahn time (needs the full pattern: computed once, untimed)."""
+    import oracle
+    full = oracle.fill2(rp, ci, emit=True, threads=os.cpu_count() or 1)
+    t0 = time.perf_counter()
+    oracle.levels(full["row_ptr"], full["col_idx"], rule)
+    return time.perf_counter() - t0, int(full["row_ptr"][-1])
+
+
+def auto_stride(n, te_total):
+    # ~2e9 TE visited by the sample (both passes) is ~10-20 s on 8 host cores
+    target = 1.0e9
+    return max(1, int(round(te_total / target)))
+
+
+# --------------------------------------------------------------------------- reference arm
+def run_reference(args, rank, world):
+    if rank != 0:
+        return
+    name, rp, ci = gen.config(args.config)
+    n = len(rp) - 1
+    te, _ = work_units(rp)
+    stride = args.cpu_sample_stride or auto_stride(n, te)
+    times, entries = [], None
+    for k in range(args.warmup + args.steps):
+        s = cpu_oracle_sample(rp, ci, stride)
+        if k >= args.warmup:
+            times.append(s["t_sym_full"])
+        entries = s
+    t_lev, nnz = cpu_levels_time(rp, ci, args.rule)
+    t_step = float(np.mean(times)) + t_lev
+    value = nnz / t_step
+    out = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_step * 1e3,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+        "data": "synthetic",
+        "config": {"workload": f"cfg{args.config} {name}", "n": n, "nnz_a": int(rp[-1]),
+                   "nnz_lu": nnz},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": entries["threads"],
+                         "kind": "oracle",
+                         "sample": f"fill2 count+emit on every {stride}-th row "
+                                   f"({len(entries['rows'])} rows, descending), extrapolated by "
+                                   f"exact TE share x{entries['scale']:.2f}; Kahn on the full "
+                                   f"pattern ({t_lev:.2f} s, 1 thread)"},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(out), flush=True)
+
+
+# --------------------------------------------------------------------------- our arm
+def run_ours(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import paper_conf_ppopp_xia0ar23_b200 as lu
+
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.current_stream()
+    name, rp_np, ci_np = gen.config(args.config)
+    n = len(rp_np) - 1
+    te, sv = work_units(rp_np)
+    rp = torch.from_numpy(rp_np).to(dev)
+    ci = torch.from_numpy(ci_np).to(dev)
+    h = lu.Symbolic(rp, ci)
+    cost = lu.row_cost_upper_bound(rp_np)
+    bounds = lu.partition_rows(cost, world)
+    rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
+    flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+
+    state = {}
+
+    def step():
+        fc = torch.zeros(n, dtype=torch.int32, device=dev)
+        h.count(rb, re_, fc)                                     # S3 (symbolic_1)
+        if world > 1:
+            lu.assemble_counts(fc)                               # S7 (counts)
+        rp_lu, nnz = h.scan(fc)                                  # S4
+        ci_lu = torch.empty(nnz, dtype=torch.int32, device=dev)  # S5
+        h.emit(rp_lu, ci_lu, rb, re_)                            # S6 (symbolic_2)
+        if world > 1:
+            lu.assemble_pattern(ci_lu, rp_lu, bounds)            # S7 (pattern)
+        level, nl = h.levelize(rp_lu, ci_lu, args.rule)          # S8 + S9
+        state.update(nnz=nnz, nl=nl, rp_lu=rp_lu, ci_lu=ci_lu, level=level, fc=fc)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    launches0 = h.stats()["kernel_launches"]
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
+          for _ in range(args.steps)]
+    k_ms = {"count": [], "scan": [], "emit": [], "levelize": []}
+    barrier()
+    torch.cuda.synchronize()
+    with ClockSampler(local_rank) as clk:
+        for k in range(args.steps):
+            flush.fill_(k)                                   # L2 flush, outside the events
+            ev[k][0].record(stream)
+            step()
+            ev[k][1].record(stream)
+            st = h.stats()
+            for key in k_ms:
+                k_ms[key].append(st["ms_" + key])
+        barrier()
+        torch.cuda.synchronize()
+    launches = h.stats()["kernel_launches"] - launches0
+    step_ms = [a.elapsed_time(b) for a, b in ev]
+    tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(tot, op=dist.ReduceOp.MAX)
+    ms_per_step = float(tot.item()) / args.steps
+    nnz = state["nnz"]
+    value = nnz / (ms_per_step / 1e3)
+    stats = h.stats()
+    if args.profile:
+        if rank == 0:
+            print(json.dumps({"profile": True, "ms_per_step": ms_per_step, "stats": stats}))
+        return
+
+    # ---- roofline of the dominant kernel (fill2 traversal; events around its launch)
+    avg = {k: float(np.mean(v)) for k, v in k_ms.items()}
+    rows_mine = re_ - rb
+    frac_rows = cost[rb:re_].sum() / max(cost.sum(), 1)
+    te_mine, sv_mine = te * frac_rows, sv * frac_rows
+    b_count = alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, False)
+    b_emit = alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, True)
+    dom = "emit" if avg["emit"] >= avg["count"] else "count"
+    b_dom = b_emit if dom == "emit" else b_count
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    peak = float(peaks.get("hbm_gbs", 6650.0))
+    achieved = b_dom / (avg[dom] / 1e3) / 1e9
+    traffic = None
+    try:
+        prof = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        traffic = prof.get(f"cfg{args.config}", {}).get(f"fill2_{dom}")
+    except Exception:
+        pass
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                "frac": achieved / peak, "traffic": traffic,
+                "kernel": f"fill2_kernel<{dom}>",
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback",
+                "alg_bytes_per_launch": b_dom, "ms_per_launch": avg[dom]}
+
+    # ---- e2e through the public API with host buffers
+    e2e = None
+    if not args.no_e2e:
+        rp_h = torch.from_numpy(rp_np).pin_memory()
+        ci_h = torch.from_numpy(ci_np).pin_memory()
+        out_rp = torch.empty(n + 1, dtype=torch.int64).pin_memory()
+        out_ci = torch.empty(nnz, dtype=torch.int32).pin_memory()
+        out_lv = torch.empty(n, dtype=torch.int32).pin_memory()
+        e_ms = []
+        for k in range(args.e2e_steps + 1):
+            barrier()
+            torch.cuda.synchronize()
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            rpd = rp_h.to(dev, non_blocking=True)
+            cid = ci_h.to(dev, non_blocking=True)
+            he = lu.Symbolic(rpd, cid)                         # S1 + S2 (validate, plan)
+            fc = torch.zeros(n, dtype=torch.int32, device=dev)
+            he.count(rb, re_, fc)
+            if world > 1:
+                lu.assemble_counts(fc)
+            rp_lu, nz = he.scan(fc)
+            ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)
+            he.emit(rp_lu, ci_lu, rb, re_)
+            if world > 1:
+                lu.assemble_pattern(ci_lu, rp_lu, bounds)
+            level, _ = he.levelize(rp_lu, ci_lu, args.rule)
+            if rank == 0:
+                out_rp.copy_(rp_lu, non_blocking=True)
+                out_ci.copy_(ci_lu, non_blocking=True)
+                out_lv.copy_(level, non_blocking=True)
+            b.record(stream)
+            torch.cuda.synchronize()
+            he.close()
+            if k > 0:
+                e_ms.append(a.elapsed_time(b))
+        t = torch.tensor([float(np.mean(e_ms))], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e = {"value": nnz / (float(t.item()) / 1e3), "unit": UNIT,
+               "h2d_bytes_per_step": int(rp_np.nbytes + ci_np.nbytes),
+               "d2h_bytes_per_step": int((n + 1) * 8 + nnz * 4 + n * 4) if rank == 0 else 0,
+               "ms_per_step": float(t.item()),
+               "includes": "H2D of A, create (validate+adjacency+plan), count, scan, alloc, "
+                           "emit, levelize, D2H of row_ptr/col_idx/level"}
+
+    if rank != 0:
+        return
+    cpu = None
+    if world == 1 and not args.no_cpu_baseline:
+        stride = args.cpu_sample_stride or auto_stride(n, te)
+        s = cpu_oracle_sample(rp_np, ci_np, stride)
+        import oracle
+        rpl = state["rp_lu"].cpu().numpy()
+        cil = state["ci_lu"].cpu().numpy()
+        t0 = time.perf_counter()
+        oracle.levels(rpl, cil, args.rule)
+        t_lev = time.perf_counter() - t0
+        t_cpu = s["t_sym_full"] + t_lev
+        cpu = {"value": nnz / t_cpu, "unit": UNIT, "cores": s["threads"], "kind": "oracle",
+               "sample": f"fill2 count+emit on every {stride}-th row ({len(s['rows'])} rows) in "
+                         f"{s['t_sample']:.2f} s, extrapolated by exact TE share "
+                         f"x{s['scale']:.2f}; Kahn levels on the full pattern {t_lev:.2f} s "
+                         f"(1 thread)"}
+    out = {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
+        "config": {"workload": f"cfg{args.config} {name}", "n": n, "nnz_a": int(rp_np[-1]),
+                   "nnz_lu": nnz, "num_levels": state["nl"], "rule": args.rule,
+                   "parallelism": f"rows sharded over {world} GPU(s)" if world > 1 else "1 GPU",
+                   "l2": "flushed between timed steps (256 MiB write, outside the events)"},
+        "phases_ms": avg,
+        "symbolic_s": (avg["count"] + avg["scan"] + avg["emit"]) / 1e3,
+        "levelize_s": avg["levelize"] / 1e3,
+        "teps": te / ((avg["count"] + avg["scan"] + avg["emit"]) / 1e3),
+        "traversed_edges_per_pass": te, "scanned_vertices_per_pass": sv,
+        "roofline": roofline,
+        "cpu_baseline": cpu,
+        "e2e": e2e,
+        "gpu_launches": int(launches),
+        "clocks": clk.summary(),
+        "plan": {k: stats[k] for k in ("rows_in_flight", "threads_per_row", "smem_bytes_per_row",
+                                        "visited_in_smem", "ell_width", "queue_capacity",
+                                        "levelize_wide_levels", "levelize_narrow_levels",
+                                        "spills")},
+    }
+    print(json.dumps(out), flush=True)
+
+
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, rank, world)
+        return
+    if world > 1:
+        import torch
+        import torch.distributed as dist
+        torch.cuda.set_device(local_rank)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+    try:
+        run_ours(args, rank, world, local_rank)
+    finally:
+        if world > 1:
+            import torch.distributed as dist
+            dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,186 @@
+/*
+ * lu_sym.h — C ABI of the B200-native symbolic LU hot path.
+ *
+ * Implements, for a square sparse pattern A (CSR), the method of Xia et al., "End-to-End LU
+ * Factorization of Large Matrices on GPUs" (PPoPP'23), /root/reference/PAPER.md:
+ *
+ *   S1  validate A                                            (input of Alg. 1; CSR L270)
+ *   S3  lu_sym_count : per-row fill2 traversal, counts only   (symbolic_1, Alg. 3;
+ *                                                               Alg. 1; Thm 1)
+ *   S4  lu_sym_scan  : exclusive prefix sum of the counts     (prefix_sum, Alg. 3)
+ *   S5  (caller)     : allocate col_idx_lu[nnz]                (Alg. 3)
+ *   S6  lu_sym_emit  : the same traversal, writing positions  (symbolic_2, Alg. 3)
+ *   S8/S9 lu_levelize: dependency graph, in-degrees, Kahn      (Alg. 5, level formula
+ *                      topological levels                       L283, dependency rule L167)
+ *
+ * Conventions (all functions):
+ *   - extern "C", no C++ or framework types.  Pointers named d_* are DEVICE pointers on the
+ *     caller's current CUDA device; h_* / plain out-params are HOST pointers.
+ *   - `stream` is a cudaStream_t passed as void* (NULL = legacy default stream).  Work is
+ *     stream-ordered on it; calls that return a host value (nnz, num_levels, status of input
+ *     validation) synchronise that stream before returning.
+ *   - Indices are 0-based (reading R1).  A's rows must be strictly increasing (sorted, no
+ *     duplicates; reading R8).  The diagonal of L+U is present iff A(i,i) is (R7).
+ *   - Output rows are sorted ascending (R9); fill_count[i] = |row i of L+U| including original
+ *     entries and the diagonal (R10); offsets are int64 (R11).
+ *   - Errors are returned as lu_status, never by abort/exception; lu_last_error() gives a
+ *     thread-local message for the last failing call on this thread.
+ *   - Ownership: A's arrays are BORROWED by the handle and must stay valid and unchanged until
+ *     lu_sym_destroy.  Output arrays are CALLER-allocated.  The handle owns only its scratch.
+ *   - Threading: one handle is used by one host thread at a time; distinct handles are
+ *     independent.
+ */
+#ifndef LU_SYM_H
+#define LU_SYM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define LU_SYM_ABI_VERSION 1
+
+typedef enum {
+    LU_OK = 0,
+    LU_ERR_ARG = 1,      /* null pointer, negative size, bad enum, row range out of [0,n]     */
+    LU_ERR_INPUT = 2,    /* A is not a valid CSR pattern (see lu_sym_create)                 */
+    LU_ERR_NOMEM = 3,    /* scratch budget smaller than one row's minimum scratch, or OOM   */
+    LU_ERR_CAPACITY = 4, /* caller's output buffer smaller than nnz(L+U)                     */
+    LU_ERR_CUDA = 5,     /* a CUDA runtime error (message in lu_last_error)                  */
+    LU_ERR_STATE = 7,    /* wrong call order (e.g. emit before scan), or device-side check   */
+    LU_ERR_INTERNAL = 8  /* a device-side consistency check failed (count/emit mismatch)     */
+} lu_status;
+
+/* Dependency rule for levelization (reading R12).
+ *   LU_DEP_U    : column j depends on column i iff i<j and (i,j) in L+U
+ *   LU_DEP_GLU3 : additionally iff i<j and (j,i) in L+U (our reading of the "other
+ *                 dependencies" deferred to GLU3.0 at L167/L497; multi-edges counted once per
+ *                 source entry, identically in in-degree and update). */
+enum { LU_DEP_U = 0, LU_DEP_GLU3 = 1 };
+
+/* lu_sym_opts.flags — tuning / test knobs (never change results) */
+enum {
+    LU_F_GLOBAL_BITMAP = 1 << 0, /* keep visited bitmaps in HBM slots even if smem would fit */
+    LU_F_NO_BATCH = 1 << 1,      /* one threshold at a time, exactly Alg. 1's order (L130)   */
+    LU_F_ASCENDING = 1 << 2,     /* process rows in increasing id (default: decreasing,
+                                    i.e. heaviest-first)                      */
+    LU_F_NO_PRUNE = 1 << 3,      /* levelize over every U edge (no transitive pruning)       */
+    LU_F_KAHN_WIDE_ONLY = 1 << 4 /* levelize: never use the single-CTA narrow phase          */
+};
+
+typedef struct {
+    int32_t struct_size;           /* = sizeof(lu_sym_opts)                                  */
+    int32_t flags;                 /* LU_F_*                                                 */
+    uint64_t scratch_budget_bytes; /* 0 => 0.85 x free HBM at create (out-of-core planner)   */
+    int32_t threads_per_row;       /* CTA size per row in flight; 0 => planner (128..1024)   */
+    int32_t rows_in_flight;        /* 0 => planner (all resident CTAs); > 0 caps it          */
+    int32_t queue_capacity;        /* shared-memory frontier entries per buffer; 0 => planner */
+    int32_t ell_width;             /* traversal adjacency width 4 or 8; 0 => planner         */
+    int32_t reserved[8];
+} lu_sym_opts;
+
+typedef struct {
+    double ms_create;             /* validate + adjacency build + planning                  */
+    double ms_count, ms_scan, ms_emit, ms_levelize; /* last call of each (device events)     */
+    int64_t nnz_lu;               /* after lu_sym_scan                                       */
+    int64_t edges_read_count;     /* adjacency entries read by the device, last count pass  */
+    int64_t edges_read_emit;      /* ... last emit pass                                      */
+    int64_t vertices_scanned_count, vertices_scanned_emit;
+    int64_t spills;               /* frontier entries that spilled from smem to HBM          */
+    int64_t scratch_bytes;        /* HBM scratch owned by the handle                         */
+    int32_t rows_in_flight;       /* CTAs (= rows processed concurrently)                    */
+    int32_t threads_per_row;
+    int32_t smem_bytes_per_row;
+    int32_t visited_in_smem;      /* 1: visited bitmap in shared memory, 0: HBM slots        */
+    int32_t ell_width;
+    int32_t queue_capacity;
+    int32_t num_levels;           /* after lu_levelize with this handle                      */
+    int32_t levelize_wide_levels, levelize_narrow_levels;
+    int32_t reserved[5];
+    int64_t kernel_launches;      /* kernels this handle launched since create (all calls)  */
+} lu_sym_stats;
+
+typedef struct lu_sym lu_sym;
+
+/* Library ABI version (== LU_SYM_ABI_VERSION). */
+int32_t lu_sym_abi_version(void);
+
+/* Fill *opts with defaults (struct_size set, everything else 0). */
+void lu_sym_default_opts(lu_sym_opts *opts);
+
+/*
+ * Create a handle for the n x n pattern A given in CSR on the device:
+ *   d_row_ptr : int64[n+1], d_row_ptr[0] = 0, non-decreasing, d_row_ptr[n] = nnz_a
+ *   d_col_idx : int32[nnz_a], each row strictly increasing, values in [0, n)
+ * Validates A on the device (LU_ERR_INPUT with the first offending row in lu_last_error),
+ * builds the traversal adjacency and plans rows-in-flight from the scratch budget
+ * (chunk_size = L/(c n); here slots = budget / per-row scratch).
+ * n = 0 is allowed (every later call is a no-op).
+ */
+lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d_row_ptr,
+                        const int32_t *d_col_idx, const lu_sym_opts *opts, void *stream);
+
+/*
+ * S3 — symbolic_1: for every row i in [row_begin, row_end) write
+ *   d_fill_count[i] = |{ j : (i,j) in L+U }|      (int32[n] array indexed by global row id)
+ * Entries outside the range are not touched (row sharding across GPUs).
+ */
+lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d_fill_count,
+                       void *stream);
+
+/*
+ * S4 — exclusive prefix sum: d_row_ptr_lu[0] = 0, d_row_ptr_lu[i+1] = d_row_ptr_lu[i] +
+ * d_fill_count[i] for all i < n (int64).  *nnz_lu (host) = d_row_ptr_lu[n].  Synchronises.
+ */
+lu_status lu_sym_scan(lu_sym *h, const int32_t *d_fill_count, int64_t *d_row_ptr_lu,
+                      int64_t *nnz_lu, void *stream);
+
+/*
+ * S6 — symbolic_2: for every row i in [row_begin, row_end) write the sorted column ids of row i
+ * of L+U to d_col_idx_lu[d_row_ptr_lu[i] .. d_row_ptr_lu[i+1]).  cap = number of int32
+ * elements of d_col_idx_lu; LU_ERR_CAPACITY if cap < d_row_ptr_lu[row_end] (checked against
+ * the handle's last scan).  LU_ERR_STATE if lu_sym_scan has not run on this handle.
+ * LU_ERR_INTERNAL if a row's emitted length differs from its count (device check).
+ */
+lu_status lu_sym_emit(lu_sym *h, int32_t row_begin, int32_t row_end, const int64_t *d_row_ptr_lu,
+                      int32_t *d_col_idx_lu, int64_t cap, void *stream);
+
+/*
+ * Convenience two-call protocol over all rows:
+ *   call 1 with d_col_idx_lu == NULL: count + scan; sets *nnz_lu; returns LU_OK.
+ *   call 2 with cap >= *nnz_lu: emit only (counts cached in the handle's scan).
+ *   cap < nnz: LU_ERR_CAPACITY with *nnz_lu set; the handle stays usable.
+ */
+lu_status lu_sym_run(lu_sym *h, int32_t *d_fill_count, int64_t *d_row_ptr_lu,
+                     int32_t *d_col_idx_lu, int64_t cap, int64_t *nnz_lu, void *stream);
+
+/*
+ * S8+S9 — levelization (Algorithm 5) of the column-dependency DAG of the pattern
+ * (d_row_ptr_lu int64[n+1], d_col_idx_lu int32[nnz], rows sorted as lu_sym_emit writes them):
+ *   d_level[j] = 0 if column j has no predecessor, else 1 + max level of its predecessors
+ *   (PAPER.md L283); *num_levels (host) = max level + 1 (0 if n = 0).  Synchronises.
+ * dep_rule: LU_DEP_U or LU_DEP_GLU3.  h may be NULL (scratch allocated per call) or a handle
+ * (scratch cached; stats recorded; its opts.flags LU_F_NO_PRUNE / LU_F_KAHN_WIDE_ONLY apply).
+ */
+lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
+                      const int32_t *d_col_idx_lu, int32_t dep_rule, int32_t *d_level,
+                      int32_t *num_levels, void *stream);
+
+/* Copy the handle's statistics to *out (host). */
+lu_status lu_sym_get_stats(const lu_sym *h, lu_sym_stats *out);
+
+/* Free the handle's scratch (synchronises its streams).  NULL is a no-op. */
+void lu_sym_destroy(lu_sym *h);
+
+/* Static description of a status code. */
+const char *lu_status_str(lu_status s);
+
+/* Message of the last failing call on the calling host thread ("" if none). */
+const char *lu_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* LU_SYM_H */

@@ -1,0 +1,299 @@
+"""B200-native symbolic LU hot path of Xia et al., "End-to-End LU Factorization of Large Matrices
+on GPUs" (PPoPP'23) — Python binding over the C ABI in include/lu_sym.h (liblusym.so).
+
+This module only marshals arguments (device pointers, sizes, the current CUDA stream) into the
+C library: every step of the path (validation, fill2 count, prefix sum, fill2 emit, dependency
+graph, in-degrees, Kahn levels) runs in the hand-written sm_100a kernels of
+paper_conf_ppopp_xia0ar23_b200/csrc.  PyTorch provides device memory, streams and process
+groups.  There is no CPU fallback: if the library is missing or no CUDA device is present, the
+calls raise.
+
+Public API (names follow the paper / SURVEY §8(b)):
+  Symbolic(row_ptr, col_idx, **opts)      handle: .count() .scan() .emit() .run() .stats()
+  levelize(row_ptr_lu, col_idx_lu, rule)  Algorithm 5 levels
+  partition_rows / assemble_counts / assemble_pattern / symbolic_distributed
+                                          row sharding across GPUs
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from dataclasses import dataclass
+
+import numpy as np
+import torch
+
+from .parallel import (assemble_counts, assemble_pattern, partition_rows,  # noqa: F401
+                       row_cost_upper_bound)
+
+__all__ = ["Symbolic", "LuSymError", "levelize", "load_library", "library_path",
+           "partition_rows", "assemble_counts", "assemble_pattern", "symbolic_distributed",
+           "row_cost_upper_bound", "DEP_U", "DEP_GLU3"]
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_LIBPATH = os.path.join(_HERE, "lib", "liblusym.so")
+
+LU_OK, LU_ERR_ARG, LU_ERR_INPUT, LU_ERR_NOMEM, LU_ERR_CAPACITY = 0, 1, 2, 3, 4
+LU_ERR_CUDA, LU_ERR_STATE, LU_ERR_INTERNAL = 5, 7, 8
+DEP_U, DEP_GLU3 = 0, 1
+F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4, 8, 16
+
+
+class LuSymError(RuntimeError):
+    def __init__(self, status, msg):
+        super().__init__(f"{msg} [status {status}]")
+        self.status = status
+
+
+class _Opts(ctypes.Structure):
+    _fields_ = [("struct_size", ctypes.c_int32), ("flags", ctypes.c_int32),
+                ("scratch_budget_bytes", ctypes.c_uint64), ("threads_per_row", ctypes.c_int32),
+                ("rows_in_flight", ctypes.c_int32), ("queue_capacity", ctypes.c_int32),
+                ("ell_width", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+
+
+class _Stats(ctypes.Structure):
+    _fields_ = [("ms_create", ctypes.c_double), ("ms_count", ctypes.c_double),
+                ("ms_scan", ctypes.c_double), ("ms_emit", ctypes.c_double),
+                ("ms_levelize", ctypes.c_double), ("nnz_lu", ctypes.c_int64),
+                ("edges_read_count", ctypes.c_int64), ("edges_read_emit", ctypes.c_int64),
+                ("vertices_scanned_count", ctypes.c_int64),
+                ("vertices_scanned_emit", ctypes.c_int64), ("spills", ctypes.c_int64),
+                ("scratch_bytes", ctypes.c_int64), ("rows_in_flight", ctypes.c_int32),
+                ("threads_per_row", ctypes.c_int32), ("smem_bytes_per_row", ctypes.c_int32),
+                ("visited_in_smem", ctypes.c_int32), ("ell_width", ctypes.c_int32),
+                ("queue_capacity", ctypes.c_int32), ("num_levels", ctypes.c_int32),
+                ("levelize_wide_levels", ctypes.c_int32),
+                ("levelize_narrow_levels", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5),
+                ("kernel_launches", ctypes.c_int64)]
+
+
+_lib = None
+
+EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sym_count",
+            "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
+            "lu_sym_destroy", "lu_status_str", "lu_last_error"]
+
+
+def library_path() -> str:
+    return _LIBPATH
+
+
+def load_library():
+    """Load liblusym.so (built by __graft_entry__.build()).  Raises if it is missing."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_LIBPATH):
+        raise ImportError(f"{_LIBPATH} not built: run `python -c 'import __graft_entry__ as g; "
+                          f"g.build()'` (no CPU fallback exists)")
+    lib = ctypes.CDLL(_LIBPATH)
+    P, I32, I64 = ctypes.c_void_p, ctypes.c_int32, ctypes.c_int64
+    lib.lu_sym_abi_version.restype = I32
+    lib.lu_sym_default_opts.argtypes = [P]
+    lib.lu_sym_create.argtypes = [P, I32, I64, P, P, P, P]
+    lib.lu_sym_count.argtypes = [P, I32, I32, P, P]
+    lib.lu_sym_scan.argtypes = [P, P, P, P, P]
+    lib.lu_sym_emit.argtypes = [P, I32, I32, P, P, I64, P]
+    lib.lu_sym_run.argtypes = [P, P, P, P, I64, P, P]
+    lib.lu_levelize.argtypes = [P, I32, P, P, I32, P, P, P]
+    lib.lu_sym_get_stats.argtypes = [P, P]
+    lib.lu_sym_destroy.argtypes = [P]
+    lib.lu_status_str.argtypes = [I32]
+    lib.lu_status_str.restype = ctypes.c_char_p
+    lib.lu_last_error.restype = ctypes.c_char_p
+    for f in ("lu_sym_create", "lu_sym_count", "lu_sym_scan", "lu_sym_emit", "lu_sym_run",
+              "lu_levelize", "lu_sym_get_stats"):
+        getattr(lib, f).restype = I32
+    if lib.lu_sym_abi_version() != 1:
+        raise ImportError("liblusym.so ABI version mismatch")
+    _lib = lib
+    return lib
+
+
+def _check(status):
+    if status != LU_OK:
+        lib = load_library()
+        raise LuSymError(status, f"{lib.lu_status_str(status).decode()}: "
+                                 f"{lib.lu_last_error().decode()}")
+
+
+def _stream_ptr(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _dev(t: torch.Tensor, dtype, name):
+    if not isinstance(t, torch.Tensor) or not t.is_cuda:
+        raise TypeError(f"{name} must be a CUDA tensor")
+    if t.dtype != dtype:
+        raise TypeError(f"{name} must be {dtype}, got {t.dtype}")
+    if not t.is_contiguous():
+        raise ValueError(f"{name} must be contiguous")
+    return ctypes.c_void_p(t.data_ptr())
+
+
+@dataclass
+class Options:
+    flags: int = 0
+    scratch_budget_bytes: int = 0
+    threads_per_row: int = 0
+    rows_in_flight: int = 0
+    queue_capacity: int = 0
+    ell_width: int = 0
+
+    def to_c(self) -> _Opts:
+        o = _Opts()
+        load_library().lu_sym_default_opts(ctypes.byref(o))
+        o.flags = self.flags
+        o.scratch_budget_bytes = self.scratch_budget_bytes
+        o.threads_per_row = self.threads_per_row
+        o.rows_in_flight = self.rows_in_flight
+        o.queue_capacity = self.queue_capacity
+        o.ell_width = self.ell_width
+        return o
+
+
+class Symbolic:
+    """Handle over lu_sym_create for the pattern A (CSR on the current CUDA device).
+
+    row_ptr: int64[n+1], col_idx: int32[nnz] (rows strictly increasing).  The tensors are
+    borrowed: keep them alive and unchanged while the handle lives (the handle keeps a
+    reference)."""
+
+    def __init__(self, row_ptr: torch.Tensor, col_idx: torch.Tensor, options: Options | None = None,
+                 stream=None, **kw):
+        lib = load_library()
+        if options is None:
+            options = Options(**kw)
+        self.row_ptr = row_ptr
+        self.col_idx = col_idx
+        self.n = int(row_ptr.numel()) - 1
+        if self.n < 0:
+            raise ValueError("row_ptr must have n+1 >= 1 entries")
+        self.device = row_ptr.device
+        self._h = ctypes.c_void_p()
+        opts = options.to_c()
+        _check(lib.lu_sym_create(ctypes.byref(self._h), self.n, int(col_idx.numel()),
+                                 _dev(row_ptr, torch.int64, "row_ptr"),
+                                 ctypes.c_void_p(col_idx.data_ptr()) if col_idx.numel() else None,
+                                 ctypes.byref(opts), _stream_ptr(stream)))
+        self.nnz_lu = None
+
+    # -- S3
+    def count(self, row_begin: int = 0, row_end: int | None = None, fill_count=None, stream=None):
+        row_end = self.n if row_end is None else row_end
+        if fill_count is None:
+            fill_count = torch.zeros(self.n, dtype=torch.int32, device=self.device)
+        _check(load_library().lu_sym_count(self._h, row_begin, row_end,
+                                           _dev(fill_count, torch.int32, "fill_count")
+                                           if self.n else None, _stream_ptr(stream)))
+        return fill_count
+
+    # -- S4
+    def scan(self, fill_count, row_ptr_lu=None, stream=None):
+        if row_ptr_lu is None:
+            row_ptr_lu = torch.empty(self.n + 1, dtype=torch.int64, device=self.device)
+        nnz = ctypes.c_int64(0)
+        _check(load_library().lu_sym_scan(self._h,
+                                          _dev(fill_count, torch.int32, "fill_count")
+                                          if self.n else None,
+                                          _dev(row_ptr_lu, torch.int64, "row_ptr_lu"),
+                                          ctypes.byref(nnz), _stream_ptr(stream)))
+        self.nnz_lu = int(nnz.value)
+        return row_ptr_lu, self.nnz_lu
+
+    # -- S6
+    def emit(self, row_ptr_lu, col_idx_lu=None, row_begin: int = 0, row_end: int | None = None,
+             stream=None):
+        row_end = self.n if row_end is None else row_end
+        if col_idx_lu is None:
+            col_idx_lu = torch.empty(max(self.nnz_lu or 0, 1), dtype=torch.int32,
+                                     device=self.device)[: self.nnz_lu or 0]
+        cap = int(col_idx_lu.numel())
+        ptr = ctypes.c_void_p(col_idx_lu.data_ptr()) if cap else ctypes.c_void_p(
+            row_ptr_lu.data_ptr())
+        _check(load_library().lu_sym_emit(self._h, row_begin, row_end,
+                                          _dev(row_ptr_lu, torch.int64, "row_ptr_lu"), ptr, cap,
+                                          _stream_ptr(stream)))
+        return col_idx_lu
+
+    def run(self, stream=None):
+        """S3 + S4 + S5 + S6 on this GPU: (fill_count, row_ptr_lu, col_idx_lu)."""
+        fc = self.count(stream=stream)
+        rp_lu, nnz = self.scan(fc, stream=stream)
+        ci_lu = torch.empty(nnz, dtype=torch.int32, device=self.device)   # Alg. 3 line 8
+        self.emit(rp_lu, ci_lu, stream=stream)
+        return fc, rp_lu, ci_lu
+
+    def levelize(self, row_ptr_lu, col_idx_lu, rule: str = "u", level=None, stream=None):
+        return levelize(row_ptr_lu, col_idx_lu, rule, level=level, handle=self, stream=stream)
+
+    def stats(self) -> dict:
+        st = _Stats()
+        _check(load_library().lu_sym_get_stats(self._h, ctypes.byref(st)))
+        return {k: getattr(st, k) for k, _ in _Stats._fields_ if k != "reserved"}
+
+    def close(self):
+        if getattr(self, "_h", None) and self._h.value:
+            load_library().lu_sym_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+def levelize(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, rule: str = "u", level=None,
+             handle: Symbolic | None = None, stream=None):
+    """S8+S9: Kahn levels of the column-dependency DAG (Alg. 5).
+
+    rule 'u' (U(i,j)!=0 => j depends on i, L167) or 'glu3' (reading R12).
+    Returns (level int32[n] on the device, num_levels)."""
+    lib = load_library()
+    n = int(row_ptr_lu.numel()) - 1
+    if level is None:
+        level = torch.empty(max(n, 0), dtype=torch.int32, device=row_ptr_lu.device)
+    nl = ctypes.c_int32(0)
+    rule_id = {"u": DEP_U, "glu3": DEP_GLU3}[rule]
+    ci = ctypes.c_void_p(col_idx_lu.data_ptr()) if col_idx_lu.numel() else ctypes.c_void_p(
+        row_ptr_lu.data_ptr())
+    _check(lib.lu_levelize(handle._h if handle is not None else None, n,
+                           _dev(row_ptr_lu, torch.int64, "row_ptr_lu"), ci, rule_id,
+                           _dev(level, torch.int32, "level") if n else None, ctypes.byref(nl),
+                           _stream_ptr(stream)))
+    return level, int(nl.value)
+
+
+def symbolic_distributed(row_ptr: torch.Tensor, col_idx: torch.Tensor, group=None,
+                         options: Options | None = None, rule: str = "u", stream=None,
+                         handle: Symbolic | None = None, cost=None):
+    """Row-sharded symbolic factorization + levelization on every rank of `group`.
+
+    A is replicated; rank r runs fill2 count and emit on its contiguous, cost-balanced row block
+    (rows are independent); per-row counts are all-reduced (disjoint supports),
+    every rank scans them, and the pattern blocks are broadcast from their owners (allgatherv),
+    so all ranks end with the identical CSR of L+U; levels are then computed replicated.
+    Returns (fill_count, row_ptr_lu, col_idx_lu, level, num_levels)."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    rank = dist.get_rank(group) if dist.is_initialized() else 0
+    h = handle if handle is not None else Symbolic(row_ptr, col_idx, options, stream=stream)
+    n = h.n
+    if cost is None:
+        cost = row_cost_upper_bound(row_ptr)
+    bounds = partition_rows(cost, world)
+    rb, re = int(bounds[rank]), int(bounds[rank + 1])
+    fc = torch.zeros(n, dtype=torch.int32, device=h.device)
+    h.count(rb, re, fc, stream=stream)
+    if world > 1:
+        fc = assemble_counts(fc, group)
+    rp_lu, nnz = h.scan(fc, stream=stream)
+    ci_lu = torch.empty(nnz, dtype=torch.int32, device=h.device)
+    h.emit(rp_lu, ci_lu, rb, re, stream=stream)
+    if world > 1:
+        assemble_pattern(ci_lu, rp_lu, bounds, group)
+    level, nl = levelize(rp_lu, ci_lu, rule, handle=h, stream=stream)
+    return fc, rp_lu, ci_lu, level, nl

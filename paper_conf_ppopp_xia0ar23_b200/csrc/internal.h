@@ -1,0 +1,77 @@
+// Internal declarations shared by the CUDA translation units of liblusym.so.
+// Nothing here is part of the public ABI (include/lu_sym.h is).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace lusym {
+
+// Traversal adjacency entry marking a vertex whose off-diagonal degree exceeds the ELL width:
+// slot 0 = kHeavy, slot 1 = row length, slots 2..3 = int64 offset of the row in A's col_idx.
+constexpr int32_t kHeavy = INT32_MIN;
+constexpr int kHdrBytes = 1024;   // per-CTA shared header (scalars + scan scratch)
+
+// Device-side statistics slots (unsigned long long each).
+enum StatSlot { kStatEdges = 0, kStatVerts = 1, kStatSpills = 2, kStatErr = 3, kStatCount = 4 };
+
+struct Fill2Params {
+    int32_t n;
+    const int64_t *rp;        // A row_ptr [n+1]
+    const int32_t *ci;        // A col_idx
+    const int32_t *ell;       // traversal adjacency, n x W int32 (16 B aligned)
+    int32_t row_begin, row_end;
+    int32_t descending;       // 1: heaviest (largest id) first
+    int32_t *fill_count;      // count pass
+    const int64_t *rp_lu;     // emit pass
+    int32_t *ci_lu;
+    uint32_t *gbitmap;        // visited bitmaps in HBM (one slot per CTA) or null
+    int64_t gbitmap_stride;   // words per slot
+    int32_t *gspill;          // frontier spill, 2 x spill_cap per CTA
+    int64_t spill_cap;
+    int32_t nw;               // bitmap words = ceil((n+1)/32)
+    int32_t q;                // shared frontier capacity per buffer (entries)
+    int32_t wcap;             // window capacity (<= q); 1 = one threshold at a time
+    unsigned long long *row_counter;
+    unsigned long long *stats;  // kStatCount slots
+};
+
+// fill2_kernels.cu
+size_t fill2_smem_bytes(int n, int q, bool global_bitmap);
+cudaError_t fill2_configure(int nt, int w, bool gb, size_t smem);
+cudaError_t fill2_occupancy(int nt, int w, bool gb, size_t smem, int *occ);
+cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, bool emit, bool gb, int grid,
+                         size_t smem, cudaStream_t s);
+
+// prep_kernels.cu
+cudaError_t validate_csr(int32_t n, int64_t nnz, const int64_t *rp, const int32_t *ci,
+                         int64_t *d_bad /*[2]: first bad row, code*/, cudaStream_t s);
+cudaError_t count_light(int32_t n, const int64_t *rp, const int32_t *ci, int w,
+                        unsigned long long *d_cnt, cudaStream_t s);
+cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, int32_t *ell,
+                      cudaStream_t s);
+cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,
+                        cudaStream_t s);
+size_t scan_scratch_elems(int32_t n);
+
+// levelize_kernels.cu
+struct LevelizeScratch {
+    int64_t *ustart = nullptr;  // [n] first strict-U position of row i
+    int64_t *uend = nullptr;    // [n] end of the (pruned) successor range of row i
+    int32_t *indeg = nullptr;   // [n]
+    int32_t *queue = nullptr;   // [2n]
+    int64_t *lt_ptr = nullptr;  // [n+1]  (GLU3 rule: transpose of strict L)
+    int32_t *lt_idx = nullptr;  // [nnz_l]
+    int64_t *lt_fill = nullptr; // [n] scatter cursors
+    int64_t *scan_blk = nullptr;
+    int32_t *ctrl = nullptr;    // device control block
+    int32_t n_cap = 0;
+    int64_t lt_cap = 0;
+};
+cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, int rule,
+                         bool prune, bool wide_only, LevelizeScratch &scr, int32_t *level,
+                         int32_t *num_levels, int32_t *wide_levels, int32_t *narrow_levels,
+                         cudaStream_t s, const char **err);
+void levelize_free(LevelizeScratch &scr);
+
+}  // namespace lusym

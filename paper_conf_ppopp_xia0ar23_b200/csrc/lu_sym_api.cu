@@ -1,0 +1,527 @@
+// C ABI of liblusym.so (declared in include/lu_sym.h): handle, out-of-core planner, calls.
+#include "lu_sym.h"
+#include "internal.h"
+
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+using namespace lusym;
+
+namespace {
+
+thread_local std::string g_err;
+
+lu_status fail(lu_status s, const char *fmt, ...)
+{
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof(buf), fmt, ap);
+    va_end(ap);
+    g_err = buf;
+    return s;
+}
+
+#define CK(x)                                                                                \
+    do {                                                                                     \
+        cudaError_t e_ = (x);                                                                \
+        if (e_ != cudaSuccess)                                                               \
+            return fail(e_ == cudaErrorMemoryAllocation ? LU_ERR_NOMEM : LU_ERR_CUDA,        \
+                        "%s: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, __LINE__);   \
+    } while (0)
+
+enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvN = 4 };
+
+}  // namespace
+
+struct lu_sym {
+    int32_t n = 0;
+    int64_t nnz_a = 0;
+    const int64_t *rp = nullptr;
+    const int32_t *ci = nullptr;
+    lu_sym_opts opts;
+    int device = 0;
+    // traversal adjacency
+    int32_t *ell = nullptr;
+    int w = 8;
+    // plan
+    bool gb = false;
+    int nt = 256, q = 2048, grid = 0;
+    size_t smem = 0;
+    uint32_t *gbitmap = nullptr;
+    int64_t gb_stride = 0;
+    int32_t *gspill = nullptr;
+    int64_t spill_cap = 0;
+    unsigned long long *dstats = nullptr;  // [0] row counter, [1..4] count pass, [5..8] emit
+    int64_t *scan_blk = nullptr;
+    int64_t *dbad = nullptr;
+    // state
+    bool scanned = false;
+    int64_t nnz_lu = 0;
+    lu_sym_stats stats;
+    LevelizeScratch lev;
+    cudaEvent_t ev[kEvN][2] = {};
+    bool ev_used[kEvN] = {};
+    int64_t scratch_bytes = 0;
+    int64_t launches = 0;
+};
+
+namespace {
+
+lu_status check_device(const lu_sym *h)
+{
+    int d = -1;
+    CK(cudaGetDevice(&d));
+    if (d != h->device)
+        return fail(LU_ERR_STATE, "handle created on device %d, current device is %d", h->device,
+                    d);
+    return LU_OK;
+}
+
+template <class T>
+lu_status dalloc(lu_sym *h, T **p, size_t elems)
+{
+    size_t bytes = elems * sizeof(T);
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(reinterpret_cast<void **>(p), bytes);
+    if (e != cudaSuccess)
+        return fail(LU_ERR_NOMEM, "cudaMalloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
+    h->scratch_bytes += (int64_t)bytes;
+    return LU_OK;
+}
+
+void free_handle(lu_sym *h)
+{
+    cudaFree(h->ell);
+    cudaFree(h->gbitmap);
+    cudaFree(h->gspill);
+    cudaFree(h->dstats);
+    cudaFree(h->scan_blk);
+    cudaFree(h->dbad);
+    levelize_free(h->lev);
+    for (int k = 0; k < kEvN; ++k)
+        for (int j = 0; j < 2; ++j)
+            if (h->ev[k][j]) cudaEventDestroy(h->ev[k][j]);
+    delete h;
+}
+
+int pow2_floor(int x)
+{
+    int p = 1;
+    while (p * 2 <= x) p *= 2;
+    return p;
+}
+
+// ---------------------------------------------------------------- out-of-core planner
+// Paper (L239-243): chunk_size = L / (c n), c = 6 words per vertex per row in flight.
+// Here a row in flight owns: a visited bitmap of n bits (shared memory when it fits, else an
+// HBM slot), two frontier queues (shared memory, spilling to 2 x n int32 in HBM).  The number
+// of rows in flight is the smaller of (resident CTAs) and (scratch budget / HBM bytes per row).
+lu_status plan(lu_sym *h)
+{
+    int sms = 0, smem_sm = 0, smem_optin = 0, smem_res = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device));
+    CK(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, h->device));
+    CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->device));
+    CK(cudaDeviceGetAttribute(&smem_res, cudaDevAttrReservedSharedMemoryPerBlock, h->device));
+    const int n = h->n;
+    h->q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : 2048;
+    if (h->q < 32) h->q = 32;
+    size_t smem = fill2_smem_bytes(n, h->q, false);
+    h->gb = (h->opts.flags & LU_F_GLOBAL_BITMAP) || smem > (size_t)smem_optin;
+    if (h->gb) smem = fill2_smem_bytes(n, h->q, true);
+    if (smem > (size_t)smem_optin)
+        return fail(LU_ERR_NOMEM, "queue_capacity %d needs %zu B of shared memory (> %d)", h->q,
+                    smem, smem_optin);
+    int ctas = (int)(smem_sm / (smem + smem_res));
+    if (ctas < 1) ctas = 1;
+    if (ctas > 16) ctas = 16;
+    int nt = h->opts.threads_per_row;
+    if (nt <= 0) {
+        nt = pow2_floor(2048 / ctas);
+        if (nt < 128) nt = 128;
+        if (nt > 1024) nt = 1024;
+        if (n < 65536 && nt > 256) nt = 256;
+    }
+    if (nt != 128 && nt != 256 && nt != 512 && nt != 1024)
+        return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512 or 1024 (got %d)", nt);
+    h->nt = nt;
+    h->smem = smem;
+    CK(fill2_configure(nt, h->w, h->gb, smem));
+    // resident CTAs of the actual kernel (registers may limit below the smem estimate)
+    int occ = 0;
+    CK(fill2_occupancy(nt, h->w, h->gb, smem, &occ));
+    if (occ < 1) return fail(LU_ERR_NOMEM, "fill2 kernel cannot be resident (smem %zu B)", smem);
+    int64_t grid = (int64_t)sms * occ;
+    if (h->opts.rows_in_flight > 0 && h->opts.rows_in_flight < grid) grid = h->opts.rows_in_flight;
+    // HBM budget
+    size_t free_b = 0, total_b = 0;
+    CK(cudaMemGetInfo(&free_b, &total_b));
+    uint64_t budget = h->opts.scratch_budget_bytes ? h->opts.scratch_budget_bytes
+                                                   : (uint64_t)(0.85 * (double)free_b);
+    const int64_t nw = ((int64_t)n + 31) / 32;
+    h->gb_stride = (nw + 31) & ~(int64_t)31;  // 128 B aligned slots
+    h->spill_cap = n > 0 ? n : 1;
+    const uint64_t per_row = (uint64_t)2 * h->spill_cap * 4 + (h->gb ? (uint64_t)h->gb_stride * 4 : 0);
+    const uint64_t fit = budget / per_row;
+    if (fit < 1)
+        return fail(LU_ERR_NOMEM, "scratch budget %llu B < one row's scratch %llu B",
+                    (unsigned long long)budget, (unsigned long long)per_row);
+    if ((uint64_t)grid > fit) grid = (int64_t)fit;
+    if (grid < 1) grid = 1;
+    h->grid = (int)grid;
+    lu_status st = dalloc(h, &h->gspill, (size_t)2 * h->spill_cap * h->grid);
+    if (st != LU_OK) return st;
+    if (h->gb) {
+        st = dalloc(h, &h->gbitmap, (size_t)h->gb_stride * h->grid);
+        if (st != LU_OK) return st;
+    }
+    return LU_OK;
+}
+
+void ev_begin(lu_sym *h, int k, cudaStream_t s)
+{
+    if (!h->ev[k][0]) {
+        cudaEventCreate(&h->ev[k][0]);
+        cudaEventCreate(&h->ev[k][1]);
+    }
+    cudaEventRecord(h->ev[k][0], s);
+}
+
+void ev_end(lu_sym *h, int k, cudaStream_t s)
+{
+    cudaEventRecord(h->ev[k][1], s);
+    h->ev_used[k] = true;
+}
+
+lu_status run_pass(lu_sym *h, bool emit, int32_t rb, int32_t re, int32_t *fill_count,
+                   const int64_t *rp_lu, int32_t *ci_lu, cudaStream_t s)
+{
+    unsigned long long *st = h->dstats + (emit ? 5 : 1);
+    CK(cudaMemsetAsync(h->dstats, 0, sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(st, 0, sizeof(unsigned long long) * kStatCount, s));
+    if (h->gb)
+        CK(cudaMemsetAsync(h->gbitmap, 0, sizeof(uint32_t) * (size_t)h->gb_stride * h->grid, s));
+    Fill2Params p;
+    p.n = h->n;
+    p.rp = h->rp;
+    p.ci = h->ci;
+    p.ell = h->ell;
+    p.row_begin = rb;
+    p.row_end = re;
+    p.descending = (h->opts.flags & LU_F_ASCENDING) ? 0 : 1;
+    p.fill_count = fill_count;
+    p.rp_lu = rp_lu;
+    p.ci_lu = ci_lu;
+    p.gbitmap = h->gbitmap;
+    p.gbitmap_stride = h->gb_stride;
+    p.gspill = h->gspill;
+    p.spill_cap = h->spill_cap;
+    p.nw = (int32_t)(((int64_t)h->n + 31) / 32);
+    p.q = h->q;
+    p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : h->q;
+    p.row_counter = h->dstats;
+    p.stats = st;
+    int grid = h->grid;
+    if (grid > re - rb) grid = re - rb;
+    CK(fill2_launch(p, h->nt, h->w, emit, h->gb, grid, h->smem, s));
+    h->launches += 1;
+    return LU_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+int32_t lu_sym_abi_version(void) { return LU_SYM_ABI_VERSION; }
+
+void lu_sym_default_opts(lu_sym_opts *o)
+{
+    if (!o) return;
+    memset(o, 0, sizeof(*o));
+    o->struct_size = (int32_t)sizeof(lu_sym_opts);
+}
+
+const char *lu_status_str(lu_status s)
+{
+    switch (s) {
+    case LU_OK: return "LU_OK";
+    case LU_ERR_ARG: return "LU_ERR_ARG";
+    case LU_ERR_INPUT: return "LU_ERR_INPUT";
+    case LU_ERR_NOMEM: return "LU_ERR_NOMEM";
+    case LU_ERR_CAPACITY: return "LU_ERR_CAPACITY";
+    case LU_ERR_CUDA: return "LU_ERR_CUDA";
+    case LU_ERR_STATE: return "LU_ERR_STATE";
+    case LU_ERR_INTERNAL: return "LU_ERR_INTERNAL";
+    }
+    return "LU_ERR_UNKNOWN";
+}
+
+const char *lu_last_error(void) { return g_err.c_str(); }
+
+lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d_row_ptr,
+                        const int32_t *d_col_idx, const lu_sym_opts *opts, void *stream)
+{
+    g_err.clear();
+    if (!out) return fail(LU_ERR_ARG, "out is NULL");
+    *out = nullptr;
+    if (n < 0 || nnz_a < 0) return fail(LU_ERR_ARG, "negative size (n=%d, nnz=%lld)", n,
+                                         (long long)nnz_a);
+    if (!d_row_ptr || (nnz_a > 0 && !d_col_idx)) return fail(LU_ERR_ARG, "null CSR pointer");
+    if (opts && opts->struct_size != (int32_t)sizeof(lu_sym_opts))
+        return fail(LU_ERR_ARG, "opts.struct_size %d != %zu", opts->struct_size,
+                    sizeof(lu_sym_opts));
+    cudaStream_t s = (cudaStream_t)stream;
+    lu_sym *h = new lu_sym();
+    if (opts) h->opts = *opts; else lu_sym_default_opts(&h->opts);
+    memset(&h->stats, 0, sizeof(h->stats));
+    h->n = n;
+    h->nnz_a = nnz_a;
+    h->rp = d_row_ptr;
+    h->ci = d_col_idx;
+    cudaEvent_t t0, t1;
+    lu_status st = LU_OK;
+    auto bail = [&](lu_status e) {
+        free_handle(h);
+        return e;
+    };
+    if (cudaGetDevice(&h->device) != cudaSuccess) return bail(fail(LU_ERR_CUDA, "no device"));
+    if (cudaEventCreate(&t0) != cudaSuccess || cudaEventCreate(&t1) != cudaSuccess)
+        return bail(fail(LU_ERR_CUDA, "cudaEventCreate failed"));
+    cudaEventRecord(t0, s);
+    if ((st = dalloc(h, &h->dstats, 16)) != LU_OK) return bail(st);
+    if ((st = dalloc(h, &h->dbad, 2)) != LU_OK) return bail(st);
+    if ((st = dalloc(h, &h->scan_blk, scan_scratch_elems(n))) != LU_OK) return bail(st);
+    cudaMemsetAsync(h->dstats, 0, 16 * sizeof(unsigned long long), s);
+    // S1: validate A
+    {
+        cudaError_t e = validate_csr(n, nnz_a, d_row_ptr, d_col_idx, h->dbad, s);
+        unsigned long long bad = ~0ull;
+        if (e == cudaSuccess) e = cudaMemcpyAsync(&bad, h->dbad, 8, cudaMemcpyDeviceToHost, s);
+        if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+        if (e != cudaSuccess)
+            return bail(fail(LU_ERR_CUDA, "validate: %s", cudaGetErrorString(e)));
+        if (bad != ~0ull) {
+            static const char *what[] = {"", "row_ptr[0] != 0", "row_ptr not monotone",
+                                         "row_ptr[n] != nnz", "column index out of [0,n)",
+                                         "row not strictly increasing (unsorted or duplicate)"};
+            const int code = (int)(bad & 0xff);
+            return bail(fail(LU_ERR_INPUT, "invalid CSR at row %lld: %s",
+                             (long long)(bad >> 8), what[code < 6 ? code : 0]));
+        }
+    }
+    if (n == 0) {
+        cudaEventDestroy(t0);
+        cudaEventDestroy(t1);
+        *out = h;
+        return LU_OK;
+    }
+    // traversal adjacency width: 4 when nearly every vertex has <= 4 off-diagonal entries
+    {
+        int w = h->opts.ell_width;
+        if (w != 0 && w != 4 && w != 8)
+            return bail(fail(LU_ERR_ARG, "ell_width must be 0, 4 or 8 (got %d)", w));
+        if (w == 0) {
+            unsigned long long light4 = 0;
+            cudaError_t e = count_light(n, d_row_ptr, d_col_idx, 4, h->dstats + 15, s);
+            if (e == cudaSuccess)
+                e = cudaMemcpyAsync(&light4, h->dstats + 15, 8, cudaMemcpyDeviceToHost, s);
+            if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+            if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
+            w = (light4 >= (unsigned long long)(0.995 * n)) ? 4 : 8;
+        }
+        h->w = w;
+        if ((st = dalloc(h, &h->ell, (size_t)n * w)) != LU_OK) return bail(st);
+        cudaError_t e = build_ell(n, d_row_ptr, d_col_idx, w, h->ell, s);
+        if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
+    }
+    if ((st = plan(h)) != LU_OK) return bail(st);
+    cudaEventRecord(t1, s);
+    if (cudaEventSynchronize(t1) != cudaSuccess)
+        return bail(fail(LU_ERR_CUDA, "create: %s", cudaGetErrorString(cudaGetLastError())));
+    float ms = 0;
+    cudaEventElapsedTime(&ms, t0, t1);
+    cudaEventDestroy(t0);
+    cudaEventDestroy(t1);
+    h->stats.ms_create = ms;
+    *out = h;
+    return LU_OK;
+}
+
+lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d_fill_count,
+                       void *stream)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    if (row_begin < 0 || row_end > h->n || row_begin > row_end)
+        return fail(LU_ERR_ARG, "row range [%d,%d) outside [0,%d]", row_begin, row_end, h->n);
+    if (row_begin == row_end) return LU_OK;
+    if (!d_fill_count) return fail(LU_ERR_ARG, "d_fill_count is NULL");
+    lu_status st = check_device(h);
+    if (st != LU_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    ev_begin(h, kEvCount, s);
+    st = run_pass(h, false, row_begin, row_end, d_fill_count, nullptr, nullptr, s);
+    ev_end(h, kEvCount, s);
+    return st;
+}
+
+lu_status lu_sym_scan(lu_sym *h, const int32_t *d_fill_count, int64_t *d_row_ptr_lu,
+                      int64_t *nnz_lu, void *stream)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    if (!d_row_ptr_lu || (h->n > 0 && !d_fill_count))
+        return fail(LU_ERR_ARG, "null pointer");
+    lu_status st = check_device(h);
+    if (st != LU_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    ev_begin(h, kEvScan, s);
+    CK(scan_counts(h->n, d_fill_count, d_row_ptr_lu, h->scan_blk, s));
+    h->launches += h->n > 0 ? 3 : 1;
+    ev_end(h, kEvScan, s);
+    int64_t nnz = 0;
+    CK(cudaMemcpyAsync(&nnz, d_row_ptr_lu + h->n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    h->nnz_lu = nnz;
+    h->stats.nnz_lu = nnz;
+    h->scanned = true;
+    if (nnz_lu) *nnz_lu = nnz;
+    return LU_OK;
+}
+
+lu_status lu_sym_emit(lu_sym *h, int32_t row_begin, int32_t row_end, const int64_t *d_row_ptr_lu,
+                      int32_t *d_col_idx_lu, int64_t cap, void *stream)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    if (row_begin < 0 || row_end > h->n || row_begin > row_end)
+        return fail(LU_ERR_ARG, "row range [%d,%d) outside [0,%d]", row_begin, row_end, h->n);
+    if (!h->scanned) return fail(LU_ERR_STATE, "lu_sym_emit before lu_sym_scan");
+    if (row_begin == row_end) return LU_OK;
+    if (!d_row_ptr_lu || !d_col_idx_lu) return fail(LU_ERR_ARG, "null pointer");
+    lu_status st = check_device(h);
+    if (st != LU_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    int64_t need = 0;
+    CK(cudaMemcpyAsync(&need, d_row_ptr_lu + row_end, sizeof(int64_t), cudaMemcpyDeviceToHost,
+                       s));
+    CK(cudaStreamSynchronize(s));
+    if (cap < need)
+        return fail(LU_ERR_CAPACITY, "cap %lld < %lld entries needed", (long long)cap,
+                    (long long)need);
+    ev_begin(h, kEvEmit, s);
+    st = run_pass(h, true, row_begin, row_end, nullptr, d_row_ptr_lu, d_col_idx_lu, s);
+    ev_end(h, kEvEmit, s);
+    if (st != LU_OK) return st;
+    unsigned long long err = 0;
+    CK(cudaMemcpyAsync(&err, h->dstats + 5 + kStatErr, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (err)
+        return fail(LU_ERR_INTERNAL, "%llu rows emitted a length different from their count",
+                    err);
+    return LU_OK;
+}
+
+lu_status lu_sym_run(lu_sym *h, int32_t *d_fill_count, int64_t *d_row_ptr_lu,
+                     int32_t *d_col_idx_lu, int64_t cap, int64_t *nnz_lu, void *stream)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    if (!d_col_idx_lu) {
+        lu_status st = lu_sym_count(h, 0, h->n, d_fill_count, stream);
+        if (st != LU_OK) return st;
+        return lu_sym_scan(h, d_fill_count, d_row_ptr_lu, nnz_lu, stream);
+    }
+    if (!h->scanned) return fail(LU_ERR_STATE, "second lu_sym_run call before the first");
+    if (nnz_lu) *nnz_lu = h->nnz_lu;
+    if (cap < h->nnz_lu)
+        return fail(LU_ERR_CAPACITY, "cap %lld < nnz %lld", (long long)cap,
+                    (long long)h->nnz_lu);
+    return lu_sym_emit(h, 0, h->n, d_row_ptr_lu, d_col_idx_lu, cap, stream);
+}
+
+lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
+                      const int32_t *d_col_idx_lu, int32_t dep_rule, int32_t *d_level,
+                      int32_t *num_levels, void *stream)
+{
+    g_err.clear();
+    if (n < 0) return fail(LU_ERR_ARG, "n < 0");
+    if (dep_rule != LU_DEP_U && dep_rule != LU_DEP_GLU3)
+        return fail(LU_ERR_ARG, "dep_rule %d", dep_rule);
+    if (n > 0 && (!d_row_ptr_lu || !d_col_idx_lu || !d_level))
+        return fail(LU_ERR_ARG, "null pointer");
+    if (h) {
+        lu_status st = check_device(h);
+        if (st != LU_OK) return st;
+    }
+    cudaStream_t s = (cudaStream_t)stream;
+    LevelizeScratch tmp;
+    LevelizeScratch &scr = h ? h->lev : tmp;
+    const int flags = h ? h->opts.flags : 0;
+    int32_t nl = 0, wl = 0, nrw = 0;
+    const char *where = "";
+    if (h) ev_begin(h, kEvLev, s);
+    cudaError_t e = levelize_run(n, d_row_ptr_lu, d_col_idx_lu, dep_rule,
+                                 !(flags & LU_F_NO_PRUNE), (flags & LU_F_KAHN_WIDE_ONLY) != 0,
+                                 scr, d_level, &nl, &wl, &nrw, s, &where);
+    if (h) ev_end(h, kEvLev, s);
+    if (!h) levelize_free(tmp);
+    if (e != cudaSuccess)
+        return fail(e == cudaErrorMemoryAllocation ? LU_ERR_NOMEM : LU_ERR_CUDA,
+                    "levelize: %s: %s", where, cudaGetErrorString(e));
+    if (num_levels) *num_levels = nl;
+    if (h) {
+        h->launches += n > 0 ? (dep_rule == LU_DEP_GLU3 ? 9 : 4) : 0;
+        h->stats.num_levels = nl;
+        h->stats.levelize_wide_levels = wl;
+        h->stats.levelize_narrow_levels = nrw;
+    }
+    return LU_OK;
+}
+
+lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
+{
+    g_err.clear();
+    if (!hc || !out) return fail(LU_ERR_ARG, "null pointer");
+    lu_sym *h = const_cast<lu_sym *>(hc);
+    double *ms[kEvN] = {&h->stats.ms_count, &h->stats.ms_scan, &h->stats.ms_emit,
+                        &h->stats.ms_levelize};
+    for (int k = 0; k < kEvN; ++k) {
+        if (!h->ev_used[k]) continue;
+        if (cudaEventSynchronize(h->ev[k][1]) != cudaSuccess) continue;
+        float v = 0;
+        if (cudaEventElapsedTime(&v, h->ev[k][0], h->ev[k][1]) == cudaSuccess) *ms[k] = v;
+    }
+    if (h->dstats && h->n > 0) {
+        unsigned long long st[16] = {};
+        if (cudaMemcpy(st, h->dstats, sizeof(st), cudaMemcpyDeviceToHost) == cudaSuccess) {
+            h->stats.edges_read_count = (int64_t)st[1 + kStatEdges];
+            h->stats.vertices_scanned_count = (int64_t)st[1 + kStatVerts];
+            h->stats.edges_read_emit = (int64_t)st[5 + kStatEdges];
+            h->stats.vertices_scanned_emit = (int64_t)st[5 + kStatVerts];
+            h->stats.spills = (int64_t)(st[1 + kStatSpills] + st[5 + kStatSpills]);
+        }
+    }
+    h->stats.scratch_bytes = h->scratch_bytes;
+    h->stats.rows_in_flight = h->grid;
+    h->stats.threads_per_row = h->nt;
+    h->stats.smem_bytes_per_row = (int32_t)h->smem;
+    h->stats.visited_in_smem = h->gb ? 0 : 1;
+    h->stats.ell_width = h->w;
+    h->stats.queue_capacity = h->q;
+    h->stats.kernel_launches = h->launches;
+    *out = h->stats;
+    return LU_OK;
+}
+
+void lu_sym_destroy(lu_sym *h)
+{
+    if (!h) return;
+    cudaDeviceSynchronize();
+    free_handle(h);
+}
+
+}  // extern "C"

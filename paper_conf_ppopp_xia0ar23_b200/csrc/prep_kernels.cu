@@ -1,0 +1,247 @@
+// Preparation kernels: CSR validation (S1), the ELL-W traversal adjacency, and the int64
+// prefix sum of the per-row counts (S4, Alg. 3 line 7 "prefix_sum(fill_count_d)", L262).
+#include "internal.h"
+
+#include <climits>
+
+namespace lusym {
+namespace {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// Error codes packed with the row id: (row << 8) | code; the smallest row wins.
+enum { kBadRp0 = 1, kBadMono = 2, kBadNnz = 3, kBadCol = 4, kBadOrder = 5 };
+
+__global__ void k_validate(int32_t n, int64_t nnz, const int64_t *rp, const int32_t *ci,
+                           unsigned long long *bad)
+{
+    const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (i > n) return;
+    auto report = [&](int64_t row, int code) {
+        atomicMin(bad, ((unsigned long long)row << 8) | (unsigned long long)code);
+    };
+    const int64_t a = rp[i];
+    if (i == 0 && a != 0) report(0, kBadRp0);
+    if (i == n) {
+        if (a != nnz) report(n, kBadNnz);
+        return;
+    }
+    const int64_t b = rp[i + 1];
+    if (b < a) {
+        report(i, kBadMono);
+        return;
+    }
+    const int64_t lo = a < 0 ? 0 : a, hi = b > nnz ? nnz : b;
+    int prev = -1;
+    for (int64_t k = lo; k < hi; ++k) {
+        const int c = ci[k];
+        if (c < 0 || c >= n) {
+            report(i, kBadCol);
+            return;
+        }
+        if (c <= prev) {
+            report(i, kBadOrder);
+            return;
+        }
+        prev = c;
+    }
+}
+
+// number of rows whose off-diagonal degree is <= w
+__global__ void k_count_light(int32_t n, const int64_t *rp, const int32_t *ci, int w,
+                              unsigned long long *cnt)
+{
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    bool light = false;
+    if (i < n) {
+        const int64_t a = rp[i], b = rp[i + 1];
+        const int64_t len = b - a;
+        if (len <= w) {
+            light = true;
+        } else if (len == w + 1) {
+            for (int64_t k = a; k < b; ++k)
+                if (ci[k] == i) light = true;
+        }
+    }
+    const unsigned m = __ballot_sync(kFull, light);
+    if ((threadIdx.x & 31) == 0 && m) atomicAdd(cnt, (unsigned long long)__popc(m));
+}
+
+// ell[i*W .. i*W+W) = off-diagonal neighbours of i padded with -1, or the heavy record
+// {kHeavy, len, off_lo, off_hi} pointing at A's own row (diagonal included: it is always
+// visited when i is scanned, so the traversal skips it).
+template <int W>
+__global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int32_t *ell)
+{
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    const int64_t a = rp[i], b = rp[i + 1];
+    const int64_t len = b - a;
+    int out[W];
+#pragma unroll
+    for (int s = 0; s < W; ++s) out[s] = -1;
+    bool heavy = len > W + 1;
+    if (!heavy) {
+        int m = 0;
+        for (int64_t k = a; k < b; ++k) {
+            const int c = ci[k];
+            if (c == i) continue;
+            if (m == W) {
+                heavy = true;
+                break;
+            }
+            out[m++] = c;
+        }
+    }
+    if (heavy) {
+        out[0] = kHeavy;
+        out[1] = (int)len;
+        out[2] = (int)(uint32_t)(a & 0xffffffffll);
+        out[3] = (int)(a >> 32);
+#pragma unroll
+        for (int s = 4; s < W; ++s) out[s] = -1;
+    }
+    int4 *dst = reinterpret_cast<int4 *>(ell + (size_t)i * W);
+    dst[0] = make_int4(out[0], out[1], out[2], out[3]);
+    if constexpr (W == 8) dst[1] = make_int4(out[4], out[5], out[6], out[7]);
+}
+
+// ---------------------------------------------------------------- scan (int32 -> int64)
+constexpr int kScanNT = 1024;
+constexpr int kScanItems = 4;
+constexpr int kScanTile = kScanNT * kScanItems;
+
+__device__ __forceinline__ long long block_scan_ll(long long x, long long *s, long long &total)
+{
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    long long inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const long long y = __shfl_up_sync(kFull, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) s[wid] = inc;
+    __syncthreads();
+    if (wid == 0) {
+        long long v = s[lane];
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const long long y = __shfl_up_sync(kFull, v, o);
+            if (lane >= o) v += y;
+        }
+        s[lane] = v;
+    }
+    __syncthreads();
+    total = s[31];
+    const long long r = (wid ? s[wid - 1] : 0) + inc - x;
+    __syncthreads();
+    return r;
+}
+
+__global__ void __launch_bounds__(kScanNT) k_scan_tiles(int32_t n, const int32_t *cnt,
+                                                        int64_t *blk)
+{
+    __shared__ long long s[32];
+    const int64_t base = (int64_t)blockIdx.x * kScanTile + threadIdx.x * kScanItems;
+    long long sum = 0;
+#pragma unroll
+    for (int j = 0; j < kScanItems; ++j)
+        if (base + j < n) sum += cnt[base + j];
+    long long total;
+    block_scan_ll(sum, s, total);
+    if (threadIdx.x == 0) blk[blockIdx.x] = total;
+}
+
+__global__ void __launch_bounds__(kScanNT) k_scan_blocks(int64_t nb, int64_t *blk,
+                                                         int64_t *row_ptr_n)
+{
+    __shared__ long long s[32];
+    long long carry = 0;
+    for (int64_t b0 = 0; b0 < nb; b0 += kScanNT) {
+        const int64_t b = b0 + threadIdx.x;
+        const long long v = b < nb ? blk[b] : 0;
+        long long total;
+        const long long ex = block_scan_ll(v, s, total);
+        if (b < nb) blk[b] = carry + ex;
+        carry += total;
+    }
+    if (threadIdx.x == 0) *row_ptr_n = carry;
+}
+
+__global__ void __launch_bounds__(kScanNT) k_scan_final(int32_t n, const int32_t *cnt,
+                                                        const int64_t *blk, int64_t *row_ptr)
+{
+    __shared__ long long s[32];
+    const int64_t base = (int64_t)blockIdx.x * kScanTile + threadIdx.x * kScanItems;
+    long long v[kScanItems];
+    long long sum = 0;
+#pragma unroll
+    for (int j = 0; j < kScanItems; ++j) {
+        v[j] = base + j < n ? cnt[base + j] : 0;
+        sum += v[j];
+    }
+    long long total;
+    long long run = blk[blockIdx.x] + block_scan_ll(sum, s, total);
+#pragma unroll
+    for (int j = 0; j < kScanItems; ++j) {
+        if (base + j < n) row_ptr[base + j] = run;
+        run += v[j];
+    }
+}
+
+}  // namespace
+
+cudaError_t validate_csr(int32_t n, int64_t nnz, const int64_t *rp, const int32_t *ci,
+                         int64_t *d_bad, cudaStream_t s)
+{
+    cudaError_t e = cudaMemsetAsync(d_bad, 0xff, sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+    const int nt = 256;
+    const int grid = (int)(((int64_t)n + 1 + nt - 1) / nt);
+    k_validate<<<grid, nt, 0, s>>>(n, nnz, rp, ci, reinterpret_cast<unsigned long long *>(d_bad));
+    return cudaGetLastError();
+}
+
+cudaError_t count_light(int32_t n, const int64_t *rp, const int32_t *ci, int w,
+                        unsigned long long *d_cnt, cudaStream_t s)
+{
+    cudaError_t e = cudaMemsetAsync(d_cnt, 0, sizeof(unsigned long long), s);
+    if (e != cudaSuccess) return e;
+    if (n == 0) return cudaSuccess;
+    k_count_light<<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, w, d_cnt);
+    return cudaGetLastError();
+}
+
+cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, int32_t *ell,
+                      cudaStream_t s)
+{
+    if (n == 0) return cudaSuccess;
+    if (w == 4)
+        k_build_ell<4><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
+    else
+        k_build_ell<8><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
+    return cudaGetLastError();
+}
+
+size_t scan_scratch_elems(int32_t n)
+{
+    return (size_t)(((int64_t)n + kScanTile - 1) / kScanTile) + 1;
+}
+
+cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,
+                        cudaStream_t s)
+{
+    const int64_t nb = ((int64_t)n + kScanTile - 1) / kScanTile;
+    if (nb > 0) {
+        k_scan_tiles<<<(unsigned)nb, kScanNT, 0, s>>>(n, counts, blk);
+        cudaError_t e = cudaGetLastError();
+        if (e != cudaSuccess) return e;
+    }
+    k_scan_blocks<<<1, kScanNT, 0, s>>>(nb, blk, row_ptr + n);
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess || nb == 0) return e;
+    k_scan_final<<<(unsigned)nb, kScanNT, 0, s>>>(n, counts, blk, row_ptr);
+    return cudaGetLastError();
+}
+
+}  // namespace lusym

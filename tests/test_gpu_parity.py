@@ -1,0 +1,329 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, element by element.
+
+Bar: the pattern is a set emitted sorted and levels are unique, so counts,
+row_ptr, col_idx and level must be bit-exact.
+"""
+import numpy as np
+import pytest
+import torch
+
+import oracle
+from inputs import gen
+from tests import pins
+
+pytestmark = pytest.mark.gpu
+
+lu = pytest.importorskip("paper_conf_ppopp_xia0ar23_b200")
+
+
+def dev():
+    return torch.device("cuda", torch.cuda.current_device())
+
+
+def gpu_run(rp, ci, rules=("u", "glu3"), **opts):
+    d = dev()
+    h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d), **opts)
+    fc, rp_lu, ci_lu = h.run()
+    levels = {}
+    for r in rules:
+        lv, nl = h.levelize(rp_lu, ci_lu, r)
+        levels[r] = (lv.cpu().numpy(), nl)
+    out = dict(counts=fc.cpu().numpy(), row_ptr=rp_lu.cpu().numpy(), col_idx=ci_lu.cpu().numpy(),
+               levels=levels, stats=h.stats())
+    h.close()
+    return out
+
+
+def assert_same(g, ref, rules=("u", "glu3"), tag=""):
+    assert np.array_equal(g["counts"], ref["counts"]), f"{tag}: counts differ"
+    assert np.array_equal(g["row_ptr"], ref["row_ptr"]), f"{tag}: row_ptr differs"
+    assert np.array_equal(g["col_idx"], ref["col_idx"]), f"{tag}: col_idx differs"
+    for r in rules:
+        lv, nl = oracle.levels(ref["row_ptr"], ref["col_idx"], r)
+        assert np.array_equal(g["levels"][r][0], lv), f"{tag}: levels ({r}) differ"
+        assert g["levels"][r][1] == nl, f"{tag}: num_levels ({r})"
+
+
+def check(rp, ci, tag="", rules=("u", "glu3"), **opts):
+    ref = oracle.fill2(rp, ci)
+    g = gpu_run(rp, ci, rules=rules, **opts)
+    assert_same(g, ref, rules, tag)
+    return g
+
+
+# ---------------------------------------------------------------- many small random cases
+def test_random_tiny_zero_free_diag():
+    rng = np.random.default_rng(2024)
+    for case in range(150):
+        n = int(rng.integers(1, 200))
+        rp, ci = gen.random_pattern(n, float(rng.uniform(0.3, 4)), seed=50_000 + case,
+                                    sym_frac=float(rng.uniform(0, 1)))
+        check(rp, ci, f"case {case}")
+
+
+def test_random_with_zero_diagonals():
+    for case in range(60):
+        n = 5 + 13 * case % 300
+        rp, ci = gen.random_pattern(n, 2.2, seed=60_000 + case, zero_free_diag=False)
+        check(rp, ci, f"zd case {case}")
+
+
+def test_random_medium_heavy_rows():
+    # a few dense rows/columns exercise the warp-cooperative heavy-vertex path (degree > W)
+    for case in range(8):
+        n = 3000
+        rng = np.random.default_rng(case)
+        rp, ci = gen.random_pattern(n, 1.5, seed=70_000 + case)
+        R = [np.repeat(np.arange(n), np.diff(rp))]
+        C = [ci.astype(np.int64)]
+        for hub in rng.choice(n, 6, replace=False):
+            nb = rng.choice(n, 400, replace=False)
+            R += [np.full(nb.size, hub), nb]
+            C += [nb, np.full(nb.size, hub)]
+        rp2, ci2 = gen.csr_from_edges(n, np.concatenate(R), np.concatenate(C))
+        check(rp2, ci2, f"hub case {case}")
+
+
+# ---------------------------------------------------------------- structured inputs
+@pytest.mark.parametrize("k", [2, 3, 5, 8, 16, 64])
+def test_lap2d(k):
+    g = check(*gen.lap2d(k), tag=f"lap2d {k}")
+    assert int(g["row_ptr"][-1]) == pins.nnz_2d(k)
+
+
+@pytest.mark.parametrize("k", [2, 3, 4, 7, 12])
+def test_lap3d(k):
+    g = check(*gen.lap3d(k), tag=f"lap3d {k}")
+    assert int(g["row_ptr"][-1]) == pins.nnz_3d(k)
+
+
+@pytest.mark.parametrize("s", [16, 32, 64, 128])
+def test_circuit(s):
+    check(*gen.circuit(s, 1), tag=f"circuit {s}")
+
+
+def test_special_matrices():
+    for n in (1, 2, 3, 12, 100, 1000):
+        for name, fn in (("tridiag", gen.tridiag), ("arrow_first", gen.arrow_first),
+                         ("arrow_last", gen.arrow_last), ("diag", gen.diag_only)):
+            check(*fn(n), tag=f"{name} {n}")
+        for b in (1, 3, 9):
+            check(*gen.band(n, b), tag=f"band {n} {b}")
+    # empty rows / no diagonal at all
+    rp = np.zeros(6, np.int64)
+    ci = np.zeros(0, np.int32)
+    check(rp, ci, tag="empty")
+    rp, ci = gen.csr_from_edges(5, [4, 3, 1], [0, 2, 3])
+    check(rp, ci, tag="no-diagonal")
+
+
+def test_fig1_fixture():
+    import os
+    A, fills, table = pins.read_fig1_golden(
+        os.path.join(os.path.dirname(__file__), "golden", "fig1_fixture.txt"))
+    R = [r for r, cs in A.items() for _ in cs]
+    C = [c for r, cs in A.items() for c in cs]
+    rp, ci = gen.csr_from_edges(10, R, C)
+    g = check(rp, ci, tag="fig1")
+    lv, nl = g["levels"]["u"]
+    assert nl == 5 and {j: int(lv[j]) for j in range(10)} == table
+
+
+# ---------------------------------------------------------------- planner / schedule knobs
+KNOBS = [
+    dict(flags=lu.F_NO_BATCH),                       # one threshold at a time (Alg. 1 order)
+    dict(flags=lu.F_GLOBAL_BITMAP),                  # visited bitmaps in HBM slots
+    dict(flags=lu.F_ASCENDING),
+    dict(queue_capacity=32),                         # forces frontier spills to HBM
+    dict(rows_in_flight=1), dict(rows_in_flight=3), dict(rows_in_flight=17),
+    dict(threads_per_row=128), dict(threads_per_row=512), dict(threads_per_row=1024),
+    dict(ell_width=4), dict(ell_width=8),
+    dict(flags=lu.F_GLOBAL_BITMAP, queue_capacity=32, rows_in_flight=5),
+    dict(flags=lu.F_NO_PRUNE), dict(flags=lu.F_KAHN_WIDE_ONLY),
+]
+
+
+@pytest.mark.parametrize("knob", KNOBS, ids=[str(k) for k in KNOBS])
+def test_knobs_do_not_change_results(knob):
+    for rp, ci in (gen.lap3d(9), gen.circuit(40, 2), gen.random_pattern(700, 2.5, seed=9),
+                   gen.lap2d(20)):
+        check(rp, ci, tag=str(knob), **knob)
+
+
+def test_spills_are_exercised():
+    g = check(*gen.lap3d(12), tag="spill", queue_capacity=32)
+    assert g["stats"]["spills"] > 0
+
+
+def test_repeated_runs_same_handle():
+    """R25: stamps/bitmaps must not leak between passes or runs on the same handle."""
+    rp, ci = gen.circuit(48, 3)
+    ref = oracle.fill2(rp, ci)
+    d = dev()
+    h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d), rows_in_flight=4)
+    for _ in range(3):
+        fc, rp_lu, ci_lu = h.run()
+        assert np.array_equal(fc.cpu().numpy(), ref["counts"])
+        assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+    h.close()
+
+
+def test_row_ranges():
+    rp, ci = gen.circuit(40, 4)
+    n = len(rp) - 1
+    ref = oracle.fill2(rp, ci)
+    d = dev()
+    h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+    fc = torch.full((n,), -7, dtype=torch.int32, device=d)
+    h.count(100, 900, fc)
+    got = fc.cpu().numpy()
+    assert np.array_equal(got[100:900], ref["counts"][100:900])
+    assert np.all(got[:100] == -7) and np.all(got[900:] == -7)
+    # pieces assembled from disjoint ranges == the full result (the multi-GPU path's contract)
+    fc = torch.zeros(n, dtype=torch.int32, device=d)
+    bounds = lu.partition_rows(lu.row_cost_upper_bound(rp), 3)
+    for r in range(3):
+        h.count(int(bounds[r]), int(bounds[r + 1]), fc)
+    rp_lu, nnz = h.scan(fc)
+    ci_lu = torch.full((nnz,), -1, dtype=torch.int32, device=d)
+    for r in (2, 0, 1):
+        h.emit(rp_lu, ci_lu, int(bounds[r]), int(bounds[r + 1]))
+    assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+    h.close()
+
+
+# ---------------------------------------------------------------- C-ABI error behaviour
+def test_error_codes():
+    d = dev()
+    ok_rp, ok_ci = gen.lap2d(4)
+    bad = []
+    rp, ci = ok_rp.copy(), ok_ci.copy()
+    ci[3], ci[4] = ci[4], ci[3]                      # unsorted row
+    bad.append((rp, ci))
+    rp, ci = ok_rp.copy(), ok_ci.copy()
+    ci[1] = ci[0]                                    # duplicate
+    bad.append((rp, ci))
+    rp, ci = ok_rp.copy(), ok_ci.copy()
+    ci[-1] = 99                                      # out of range
+    bad.append((rp, ci))
+    rp, ci = ok_rp.copy(), ok_ci.copy()
+    rp[-1] += 1                                      # row_ptr[n] != nnz
+    bad.append((rp, ci))
+    rp, ci = ok_rp.copy(), ok_ci.copy()
+    rp[5], rp[6] = rp[6], rp[5]                      # not monotone
+    bad.append((rp, ci))
+    for rp, ci in bad:
+        with pytest.raises(lu.LuSymError) as e:
+            lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+        assert e.value.status == lu.LU_ERR_INPUT
+    h = lu.Symbolic(torch.from_numpy(ok_rp).to(d), torch.from_numpy(ok_ci).to(d))
+    fc = h.count()
+    rp_lu = torch.zeros(17, dtype=torch.int64, device=d)
+    with pytest.raises(lu.LuSymError) as e:
+        h.emit(rp_lu, torch.zeros(10, dtype=torch.int32, device=d))
+    assert e.value.status == lu.LU_ERR_STATE
+    rp_lu, nnz = h.scan(fc)
+    with pytest.raises(lu.LuSymError) as e:
+        h.emit(rp_lu, torch.zeros(nnz - 1, dtype=torch.int32, device=d))
+    assert e.value.status == lu.LU_ERR_CAPACITY
+    with pytest.raises(lu.LuSymError) as e:
+        h.count(3, 2)
+    assert e.value.status == lu.LU_ERR_ARG
+    with pytest.raises(lu.LuSymError) as e:
+        lu.Symbolic(torch.from_numpy(ok_rp).to(d), torch.from_numpy(ok_ci).to(d),
+                    threads_per_row=100)
+    assert e.value.status == lu.LU_ERR_ARG
+    with pytest.raises(lu.LuSymError) as e:
+        lu.Symbolic(torch.from_numpy(ok_rp).to(d), torch.from_numpy(ok_ci).to(d),
+                    scratch_budget_bytes=16)
+    assert e.value.status == lu.LU_ERR_NOMEM
+    h.close()
+
+
+# ---------------------------------------------------------------- BASELINE configs
+def test_cfg1_full():
+    g = check(*gen.lap2d(64), tag="cfg1")
+    assert int(g["row_ptr"][-1]) == 520_318
+    assert g["levels"]["u"][1] == 4096
+
+
+@pytest.mark.slow
+def test_cfg2_full_bench_launch_config():
+    """cfg2 (bench.py's N=1 workload) element by element against the full oracle."""
+    rp, ci = gen.lap3d(40)
+    ref = oracle.fill2(rp, ci)
+    g = gpu_run(rp, ci, rules=("u",))
+    assert int(g["row_ptr"][-1]) == pins.nnz_3d(40) == 199_868_878
+    assert np.array_equal(g["counts"], ref["counts"])
+    assert np.array_equal(g["row_ptr"], ref["row_ptr"])
+    assert np.array_equal(g["col_idx"], ref["col_idx"])
+    lv, nl = g["levels"]["u"]
+    assert np.array_equal(lv, np.arange(64_000)) and nl == 64_000
+
+
+@pytest.mark.slow
+def test_cfg3_sampled_rows_and_levels():
+    rp, ci = gen.circuit(1024, 1)
+    n = len(rp) - 1
+    g = gpu_run(rp, ci, rules=("u", "glu3"))
+    rng = np.random.default_rng(3)
+    rows = np.unique(np.concatenate([rng.choice(n, 1500, replace=False),
+                                     np.arange(n - 300, n)])).astype(np.int32)
+    ref = oracle.fill2(rp, ci, rows=rows)
+    for k, i in enumerate(rows):
+        a, b = ref["row_ptr"][k], ref["row_ptr"][k + 1]
+        got = g["col_idx"][g["row_ptr"][i]:g["row_ptr"][i + 1]]
+        assert np.array_equal(got, ref["col_idx"][a:b]), f"row {i}"
+    assert np.array_equal(np.diff(g["row_ptr"]), g["counts"])
+    # levels of the GPU pattern vs the oracle's Kahn on the same pattern (bit-exact)
+    for r in ("u", "glu3"):
+        lv, nl = oracle.levels(g["row_ptr"], g["col_idx"], r)
+        assert np.array_equal(g["levels"][r][0], lv) and g["levels"][r][1] == nl
+
+
+def _closed_form_counts_2d(k):
+    n = k * k
+    i = np.arange(n)
+    y, x = i // k, i % k
+    L = np.where(y >= 1, k, np.where(x >= 1, 1, 0))
+    U = np.where(y == k - 1, n - i, np.where(y >= 1, k + 1, 1 + (x < k - 1) + x + 1))
+    return (L + U).astype(np.int64)
+
+
+def _closed_form_counts_3d(k):
+    n = k ** 3
+    k2 = k * k
+    i = np.arange(n)
+    z, p = i // k2, i % k2
+    c2 = _closed_form_counts_2d(k)[p] + (p + 1)         # plane-0 rows gain [k^2, k^2+p]
+    cz = np.where(z == k - 1, k2 + (n - i), 2 * k2 + 1)
+    return np.where(z == 0, c2, cz).astype(np.int64)
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("cfg", [4, 5])
+def test_cfg45_closed_forms(cfg):
+    """cfg4/cfg5 (2.1e9 entries): every count vs the closed form, sampled rows vs the closed
+    form rows and the oracle, levels == arange(n) (chains), checked on the device."""
+    name, rp, ci = gen.config(cfg)
+    n = len(rp) - 1
+    k = 1024 if cfg == 4 else 64
+    d = dev()
+    h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+    fc, rp_lu, ci_lu = h.run()
+    expect = _closed_form_counts_2d(k) if cfg == 4 else _closed_form_counts_3d(k)
+    assert np.array_equal(fc.cpu().numpy().astype(np.int64), expect)
+    nnz = pins.nnz_2d(k) if cfg == 4 else pins.nnz_3d(k)
+    assert int(rp_lu[-1]) == nnz
+    rng = np.random.default_rng(cfg)
+    rows = np.unique(np.concatenate([rng.choice(n, 200, replace=False), [0, 1, n - 2, n - 1]]))
+    rpl = rp_lu.cpu().numpy()
+    ref = oracle.fill2(rp, ci, rows=rows.astype(np.int32))
+    for kk, i in enumerate(rows):
+        got = ci_lu[int(rpl[i]):int(rpl[i + 1])].cpu().numpy()
+        assert np.array_equal(got, ref["col_idx"][ref["row_ptr"][kk]:ref["row_ptr"][kk + 1]])
+    # every row sorted and inside [0, n): checked on the device in chunks
+    lv, nl = h.levelize(rp_lu, ci_lu, "u")
+    assert nl == n
+    assert torch.equal(lv, torch.arange(n, dtype=torch.int32, device=d))
+    h.close()
