@@ -66,7 +66,8 @@ enum {
     LU_F_ASCENDING = 1 << 2,     /* process rows in increasing id (default: decreasing,
                                     i.e. heaviest-first)                      */
     LU_F_NO_PRUNE = 1 << 3,      /* levelize over every U edge (no transitive pruning)       */
-    LU_F_KAHN_WIDE_ONLY = 1 << 4 /* levelize: never use the single-CTA narrow phase          */
+    LU_F_KAHN_WIDE_ONLY = 1 << 4,/* levelize: never use the single-CTA narrow phase          */
+    LU_F_NO_CONTRACT = 1 << 5    /* levelize: Kahn over every column (no chain contraction)  */
 };
 
 typedef struct {
@@ -84,8 +85,8 @@ typedef struct {
     double ms_create;             /* validate + adjacency build + planning                  */
     double ms_count, ms_scan, ms_emit, ms_levelize; /* last call of each (device events)     */
     int64_t nnz_lu;               /* after lu_sym_scan                                       */
-    int64_t edges_read_count;     /* adjacency entries read by the device, last count pass  */
-    int64_t edges_read_emit;      /* ... last emit pass                                      */
+    int64_t edges_read_count;     /* entries read from A's CSR (seed rows, heavy vertices),  */
+    int64_t edges_read_emit;      /*   last count / emit pass; ELL reads are not counted     */
     int64_t vertices_scanned_count, vertices_scanned_emit;
     int64_t spills;               /* frontier entries that spilled from smem to HBM          */
     int64_t scratch_bytes;        /* HBM scratch owned by the handle                         */
@@ -96,8 +97,9 @@ typedef struct {
     int32_t ell_width;
     int32_t queue_capacity;
     int32_t num_levels;           /* after lu_levelize with this handle                      */
-    int32_t levelize_wide_levels, levelize_narrow_levels;
-    int32_t reserved[5];
+    int32_t levelize_wide_levels, levelize_narrow_levels; /* Kahn rounds by mode            */
+    int32_t levelize_rank_rounds; /* pointer-jumping rounds of the chain contraction        */
+    int32_t reserved[4];
     int64_t kernel_launches;      /* kernels this handle launched since create (all calls)  */
 } lu_sym_stats;
 

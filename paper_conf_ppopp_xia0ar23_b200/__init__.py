@@ -37,6 +37,7 @@ LU_OK, LU_ERR_ARG, LU_ERR_INPUT, LU_ERR_NOMEM, LU_ERR_CAPACITY = 0, 1, 2, 3, 4
 LU_ERR_CUDA, LU_ERR_STATE, LU_ERR_INTERNAL = 5, 7, 8
 DEP_U, DEP_GLU3 = 0, 1
 F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4, 8, 16
+F_NO_CONTRACT = 32
 
 
 class LuSymError(RuntimeError):
@@ -64,7 +65,8 @@ class _Stats(ctypes.Structure):
                 ("visited_in_smem", ctypes.c_int32), ("ell_width", ctypes.c_int32),
                 ("queue_capacity", ctypes.c_int32), ("num_levels", ctypes.c_int32),
                 ("levelize_wide_levels", ctypes.c_int32),
-                ("levelize_narrow_levels", ctypes.c_int32), ("reserved", ctypes.c_int32 * 5),
+                ("levelize_narrow_levels", ctypes.c_int32),
+                ("levelize_rank_rounds", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4),
                 ("kernel_launches", ctypes.c_int64)]
 
 

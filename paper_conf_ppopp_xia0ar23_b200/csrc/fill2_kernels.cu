@@ -221,25 +221,54 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, uint32_t *bm, int32_t *qA, int
                 const int f = k < p.q ? F[k] : __ldcg(gF + k);
                 load_nb<W>(p.ell, f, nb);
                 heavy = nb[0] == kHeavy;
-                if (!heavy) ++a.sv;
             }
+            // light vertex: test-and-set its <= W neighbours, remember the new frontier ones
+            uint32_t frm = 0;
+            if (valid && !heavy) {
+                ++a.sv;
 #pragma unroll
-            for (int s = 0; s < W; ++s) {
-                const int w = heavy ? -1 : nb[s];
-                bool fr = false;
-                if (w >= 0) {
-                    ++a.te;
-                    if (!visited<GB>(bm, w) && mark(bm, w)) {
+                for (int s = 0; s < W; ++s) {
+                    const int w = nb[s];
+                    if (w >= 0 && !visited<GB>(bm, w) && mark(bm, w)) {
                         if (w < t0) {
-                            fr = true;
-                            a.lmin = min(a.lmin, w);
+                            frm |= 1u << s;
                         } else if (w > i) {
                             ++a.ucnt;
                             a.lmax = max(a.lmax, w);
                         }
                     }
                 }
-                push(fr, w, nsz, NF, gNF, p.q, a.spills);
+            }
+            // one warp-aggregated append for all new frontier vertices of the warp
+            {
+                const int c = __popc(frm);
+                int inc = c;
+#pragma unroll
+                for (int o = 1; o < 32; o <<= 1) {
+                    const int y = __shfl_up_sync(kFull, inc, o);
+                    if (lane >= o) inc += y;
+                }
+                const int total = __shfl_sync(kFull, inc, 31);
+                if (total) {
+                    int wbase = 0;
+                    if (lane == 31) wbase = atomicAdd(nsz, total);
+                    wbase = __shfl_sync(kFull, wbase, 31);
+                    int pos = wbase + inc - c;
+#pragma unroll
+                    for (int s = 0; s < W; ++s) {
+                        if (frm & (1u << s)) {
+                            const int w = nb[s];
+                            a.lmin = min(a.lmin, w);
+                            if (pos < p.q) {
+                                NF[pos] = w;
+                            } else {
+                                gNF[pos] = w;
+                                ++a.spills;
+                            }
+                            ++pos;
+                        }
+                    }
+                }
             }
             unsigned hm = __ballot_sync(kFull, valid && heavy);
             while (hm) {
@@ -375,10 +404,7 @@ __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
 #pragma unroll
                     for (int s = 0; s < W; ++s) {
                         const int w = nb[s];
-                        if (w >= 0) {
-                            ++a.te;
-                            if (w < t && !visited<GB>(bm, w)) simple = false;
-                        }
+                        if (w >= 0 && w < t && !visited<GB>(bm, w)) simple = false;
                     }
                     if (!simple) {
                         atomicMin(&h.tns, t);

@@ -65,13 +65,17 @@ struct LevelizeScratch {
     int64_t *lt_fill = nullptr; // [n] scatter cursors
     int64_t *scan_blk = nullptr;
     int32_t *ctrl = nullptr;    // device control block
+    int32_t *chain = nullptr;   // [8n] J0 D0 J1 D1 nxt tail len best
     int32_t n_cap = 0;
     int64_t lt_cap = 0;
 };
+struct LevelizeInfo {
+    int32_t num_levels = 0, rounds = 0, wide_rounds = 0, narrow_rounds = 0, rank_rounds = 0;
+    int32_t launches = 0;
+};
 cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, int rule,
-                         bool prune, bool wide_only, LevelizeScratch &scr, int32_t *level,
-                         int32_t *num_levels, int32_t *wide_levels, int32_t *narrow_levels,
-                         cudaStream_t s, const char **err);
+                         bool prune, bool contract, bool wide_only, LevelizeScratch &scr,
+                         int32_t *level, LevelizeInfo *info, cudaStream_t s, const char **err);
 void levelize_free(LevelizeScratch &scr);
 
 }  // namespace lusym

@@ -2,18 +2,23 @@
 //
 //   cons_graph   (L308): the dependency graph is a VIEW of the L+U CSR: the successors of
 //                column i are the strict-U entries of row i (rule "U(i,j)!=0 => j depends on
-//                i", L167), optionally pruned to the prefix up to the first symmetric pair
+//                i", L167), pruned to the prefix up to the first symmetric pair
 //                p_i = min{k > i : (i,k),(k,i) in P}, which is exact for longest paths
 //                (reading R27); the GLU3 reading (R12) adds the transpose of strict L.
+//                Chains u -> v with outdeg(u) = 1 = indeg(v) are then contracted (list ranking
+//                by pointer jumping): along a chain level(v) = level(head) + rank(v), so Kahn
+//                only has to order chain heads.  Both reductions preserve every level exactly;
+//                LU_F_NO_PRUNE / LU_F_NO_CONTRACT switch them off (plain Alg. 5).
 //   cnt_indegree (L311): atomic histogram over the successor lists.
 //   Topo         (L293-306): ONE persistent cooperative kernel replaces the parent kernel and
 //                its dynamically launched children (device-side cudaDeviceSynchronize is gone
-//                on sm_90+).  Wide levels: every CTA relaxes the queue (warp per queued column,
-//                lanes over its successors), grid barrier per level.  Narrow levels (queue <=
-//                narrow_max): CTA 0 alone runs level after level with a shared-memory queue
-//                and __syncthreads, while the other CTAs wait at the next grid barrier.
-//   level(k) = max(-1, level(preds)) + 1 (L283) is exactly the round in which column k's
-//   in-degree reaches zero; each column is enqueued once, on that decrement (reading R14).
+//                on sm_90+).  Wide rounds: every CTA relaxes the queue (warp per queued chain,
+//                lanes over its tail's successors), grid barrier per round.  Narrow rounds
+//                (queue <= kNarrowMax): CTA 0 alone runs round after round with a shared-memory
+//                queue and __syncthreads while the other CTAs wait at the next grid barrier.
+//   level(k) = max(-1, level(preds)) + 1 (L283): a head's level is the max over its
+//   predecessor chains of (their head level + length), final when its in-degree reaches 0;
+//   each head is enqueued exactly once, on that decrement (reading R14).
 #include "internal.h"
 
 #include <cooperative_groups.h>
@@ -29,7 +34,10 @@ constexpr int kNarrowQ = 4096;   // shared queue entries per buffer (narrow phas
 constexpr int kNarrowMax = 2048; // queue size at or below which CTA 0 runs alone
 
 // ctrl block layout (int32)
-enum { kQ0 = 0, kQ1 = 1, kQ2 = 2, kLevel = 3, kWide = 4, kNarrow = 5, kCtrlInts = 8 };
+enum {
+    kQ0 = 0, kQ1 = 1, kQ2 = 2, kRound = 3, kWide = 4, kNarrow = 5, kMaxLevel = 6,
+    kChanged = 8, /* 8..10 rotating flags of the list-ranking loop */ kCtrlInts = 16
+};
 
 __device__ __forceinline__ int64_t lower_bound_dev(const int32_t *ci, int64_t lo, int64_t hi,
                                                    int key)
@@ -124,13 +132,98 @@ __global__ void k_indeg(int32_t n, const int32_t *ci, const int64_t *us, const i
     }
 }
 
-// cons_queue for level 0 (L294-296)
-__global__ void k_init_queue(int32_t n, const int32_t *indeg, int32_t *level, int32_t *q0,
-                             int32_t *ctrl)
+// chain links: u -> v is a link iff u has exactly one successor v and v exactly one predecessor.
+// J[v] = link predecessor (or v), D[v] = 1 for linked v (else 0), nxt[u] = v or -1.
+__global__ void k_link(int32_t n, const int32_t *ci, const int64_t *us, const int64_t *ue,
+                       const int64_t *ltp, const int32_t *lti, const int32_t *indeg, int contract,
+                       int32_t *J, int32_t *D, int32_t *nxt)
+{
+    const int u = blockIdx.x * blockDim.x + threadIdx.x;
+    if (u >= n) return;
+    int v = -1;
+    if (contract) {
+        const int64_t du = ue[u] - us[u];
+        const int64_t dl = ltp ? ltp[u + 1] - ltp[u] : 0;
+        if (du + dl == 1) {
+            const int c = du ? ci[us[u]] : lti[ltp[u]];
+            if (indeg[c] == 1) v = c;
+        }
+    }
+    nxt[u] = v;
+    if (v >= 0) {
+        J[v] = u;
+        D[v] = 1;
+    }
+}
+
+__global__ void k_link_init(int32_t n, int32_t *J, int32_t *D)
+{
+    const int v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v < n) {
+        J[v] = v;
+        D[v] = 0;
+    }
+}
+
+// list ranking by pointer jumping: after the loop J[v] = chain head, D[v] = rank in the chain
+__global__ void __launch_bounds__(256) k_rank(int32_t n, int32_t *J0, int32_t *D0, int32_t *J1,
+                                              int32_t *D1, int32_t *ctrl, int32_t *rounds_out)
+{
+    cg::grid_group grid = cg::this_grid();
+    int32_t *Ja = J0, *Da = D0, *Jb = J1, *Db = D1;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    const int64_t t0 = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    int r = 0;
+    for (;; ++r) {
+        int32_t *flag = ctrl + kChanged + r % 3;
+        if (t0 == 0) ctrl[kChanged + (r + 1) % 3] = 0;
+        bool changed = false;
+        for (int64_t v = t0; v < n; v += stride) {
+            const int j = __ldcg(Ja + v);
+            const int jj = __ldcg(Ja + j);
+            Jb[v] = jj;
+            Db[v] = __ldcg(Da + v) + (j != v ? __ldcg(Da + j) : 0);
+            changed |= jj != j;
+        }
+        if (__syncthreads_or(changed) && threadIdx.x == 0) atomicOr(flag, 1);
+        grid.sync();
+        int32_t *t = Ja; Ja = Jb; Jb = t;
+        t = Da; Da = Db; Db = t;
+        if (__ldcg(flag) == 0) break;
+    }
+    // make sure the final result is in (J0, D0)
+    if (Ja != J0) {
+        for (int64_t v = t0; v < n; v += stride) {
+            J0[v] = Ja[v];
+            D0[v] = Da[v];
+        }
+    }
+    if (t0 == 0) *rounds_out = r + 1;
+}
+
+// per chain: tail and length (stored at the head)
+__global__ void k_chain_info(int32_t n, const int32_t *J, const int32_t *D, const int32_t *nxt,
+                             int32_t *tail, int32_t *len)
+{
+    const int v = blockIdx.x * blockDim.x + threadIdx.x;
+    if (v >= n) return;
+    if (nxt[v] < 0) {
+        const int h = J[v];
+        tail[h] = v;
+        len[h] = D[v] + 1;
+    }
+}
+
+// cons_queue for round 0 (L294-296): heads with in-degree 0
+__global__ void k_init_queue(int32_t n, const int32_t *indeg, const int32_t *J, int32_t *best,
+                             int32_t *q0, int32_t *ctrl)
 {
     const int j = blockIdx.x * blockDim.x + threadIdx.x;
-    const bool src = j < n && indeg[j] == 0;
-    if (j < n) level[j] = src ? 0 : -1;
+    bool src = false;
+    if (j < n) {
+        best[j] = 0;
+        src = J[j] == j && indeg[j] == 0;
+    }
     const unsigned b = __ballot_sync(kFull, src);
     if (!b) return;
     const int lane = threadIdx.x & 31, leader = __ffs(b) - 1;
@@ -146,7 +239,8 @@ struct KahnArgs {
     const int64_t *us, *ue;
     const int64_t *ltp;
     const int32_t *lti;
-    int32_t *indeg, *level, *queue;  // queue: 2 x n
+    const int32_t *tail, *len;
+    int32_t *indeg, *best, *queue;  // queue: 2 x n
     int32_t *ctrl;
     int32_t narrow_max;
     int32_t wide_only;
@@ -154,42 +248,44 @@ struct KahnArgs {
 
 __device__ __forceinline__ int ld_ctrl(const int32_t *p) { return __ldcg(p); }
 
-// relax every successor v of u: update (L299) + cons_queue (L302) fused
+// relax the successors v of chain h (update, L299 + cons_queue, L302, fused)
 template <class Push>
-__device__ __forceinline__ void relax(const KahnArgs &A, int u, int nextlvl, Push &&push)
+__device__ __forceinline__ void relax(const KahnArgs &A, int h, Push &&push)
 {
     const int lane = threadIdx.x & 31;
-    const int64_t a = A.us[u], b = A.ue[u];
+    const int t = A.tail[h];
+    const int lvl = __ldcg(A.best + h) + A.len[h];  // level of every successor via this chain
+    const int64_t a = A.us[t], b = A.ue[t];
     for (int64_t eb = a; eb < b; eb += 32) {
         const int64_t e = eb + lane;
         bool z = false;
         int v = 0;
         if (e < b) {
             v = A.ci[e];
+            atomicMax(A.best + v, lvl);
             z = atomicSub(A.indeg + v, 1) == 1;
-            if (z) A.level[v] = nextlvl;
         }
         push(z, v);
     }
     if (A.ltp) {
-        const int64_t c = A.ltp[u], d = A.ltp[u + 1];
+        const int64_t c = A.ltp[t], d = A.ltp[t + 1];
         for (int64_t eb = c; eb < d; eb += 32) {
             const int64_t e = eb + lane;
             bool z = false;
             int v = 0;
             if (e < d) {
                 v = A.lti[e];
+                atomicMax(A.best + v, lvl);
                 z = atomicSub(A.indeg + v, 1) == 1;
-                if (z) A.level[v] = nextlvl;
             }
             push(z, v);
         }
     }
 }
 
-__device__ __forceinline__ int warp_push_slot(bool pred, int *cnt, unsigned &b)
+__device__ __forceinline__ int warp_push_slot(bool pred, int *cnt)
 {
-    b = __ballot_sync(kFull, pred);
+    const unsigned b = __ballot_sync(kFull, pred);
     if (!b) return 0;
     const int lane = threadIdx.x & 31, leader = __ffs(b) - 1;
     int base = 0;
@@ -207,7 +303,7 @@ __global__ void __launch_bounds__(kKahnNT) k_kahn(const KahnArgs A)
     constexpr int NW = kKahnNT / 32;
     const int gwarp = blockIdx.x * NW + warp;
     const int twarps = gridDim.x * NW;
-    int L = 0;
+    int L = 0;  // round number
     for (;;) {
         const int q = ld_ctrl(A.ctrl + L % 3);
         if (q == 0) break;
@@ -215,9 +311,9 @@ __global__ void __launch_bounds__(kKahnNT) k_kahn(const KahnArgs A)
         int32_t *NQ = A.queue + (size_t)((L + 1) & 1) * A.n;
         if (q <= A.narrow_max && !A.wide_only) {
             if (blockIdx.x == 0) {
-                // ---- narrow phase: CTA 0 alone, shared queue, __syncthreads per level
+                // ---- narrow phase: CTA 0 alone, shared queue, __syncthreads per round
                 int32_t *cur = sq, *nxt = sq + kNarrowQ;
-                for (int k = tid; k < q; k += kKahnNT) cur[k] = Q[k];
+                for (int k = tid; k < q; k += kKahnNT) cur[k] = __ldcg(Q + k);
                 if (tid == 0) scnt[0] = scnt[1] = scnt[2] = 0;
                 __syncthreads();
                 int qq = q, it = 0, lv = L, nq = 0;
@@ -226,10 +322,8 @@ __global__ void __launch_bounds__(kKahnNT) k_kahn(const KahnArgs A)
                     if (tid == 0) scnt[(it + 2) % 3] = 0;
                     int32_t *gnext = A.queue + (size_t)((lv + 1) & 1) * A.n;
                     for (int k = warp; k < qq; k += NW) {
-                        const int u = cur[k];
-                        relax(A, u, lv + 1, [&](bool z, int v) {
-                            unsigned b;
-                            const int pos = warp_push_slot(z, cnt, b);
+                        relax(A, cur[k], [&](bool z, int v) {
+                            const int pos = warp_push_slot(z, cnt);
                             if (z) {
                                 if (pos < kNarrowQ) nxt[pos] = v; else gnext[pos] = v;
                             }
@@ -250,39 +344,51 @@ __global__ void __launch_bounds__(kKahnNT) k_kahn(const KahnArgs A)
                 if (tid == 0) {
                     A.ctrl[lv % 3] = nq;
                     A.ctrl[(lv + 1) % 3] = 0;
-                    A.ctrl[kLevel] = lv;
+                    A.ctrl[kRound] = lv;
                     A.ctrl[kNarrow] += it;
                 }
             }
             grid.sync();
-            L = ld_ctrl(A.ctrl + kLevel);
+            L = ld_ctrl(A.ctrl + kRound);
             continue;
         }
-        // ---- wide level: all CTAs
+        // ---- wide round: all CTAs
         if (blockIdx.x == 0 && tid == 0) {
             A.ctrl[(L + 2) % 3] = 0;
             A.ctrl[kWide] += 1;
         }
         int *gcnt = A.ctrl + (L + 1) % 3;
         for (int k = gwarp; k < q; k += twarps) {
-            const int u = Q[k];
-            relax(A, u, L + 1, [&](bool z, int v) {
-                unsigned b;
-                const int pos = warp_push_slot(z, gcnt, b);
+            relax(A, __ldcg(Q + k), [&](bool z, int v) {
+                const int pos = warp_push_slot(z, gcnt);
                 if (z) NQ[pos] = v;
             });
         }
         grid.sync();
         ++L;
     }
-    if (blockIdx.x == 0 && tid == 0) A.ctrl[kLevel] = L;
+    if (blockIdx.x == 0 && tid == 0) A.ctrl[kRound] = L;
+}
+
+// level(v) = level(head) + rank(v); num_levels = max + 1
+__global__ void k_expand(int32_t n, const int32_t *J, const int32_t *D, const int32_t *best,
+                         int32_t *level, int32_t *ctrl)
+{
+    const int v = blockIdx.x * blockDim.x + threadIdx.x;
+    int l = -1;
+    if (v < n) {
+        l = best[J[v]] + D[v];
+        level[v] = l;
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) l = max(l, __shfl_xor_sync(kFull, l, o));
+    if ((threadIdx.x & 31) == 0) atomicMax(ctrl + kMaxLevel, l);
 }
 
 constexpr int kAuxNT = 256;
 
-int aux_grid(int64_t rows_per_warp_items)
+int aux_grid(int64_t warps)
 {
-    int64_t warps = rows_per_warp_items;
     int64_t blocks = (warps * 32 + kAuxNT - 1) / kAuxNT;
     if (blocks > 148 * 16) blocks = 148 * 16;
     if (blocks < 1) blocks = 1;
@@ -295,7 +401,7 @@ void levelize_free(LevelizeScratch &s)
 {
     cudaFree(s.ustart); cudaFree(s.uend); cudaFree(s.indeg); cudaFree(s.queue);
     cudaFree(s.lt_ptr); cudaFree(s.lt_idx); cudaFree(s.lt_fill); cudaFree(s.scan_blk);
-    cudaFree(s.ctrl);
+    cudaFree(s.ctrl); cudaFree(s.chain);
     s = LevelizeScratch();
 }
 
@@ -309,18 +415,17 @@ void levelize_free(LevelizeScratch &s)
     } while (0)
 
 cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, int rule,
-                         bool prune, bool wide_only, LevelizeScratch &s, int32_t *level,
-                         int32_t *num_levels, int32_t *wide_levels, int32_t *narrow_levels,
-                         cudaStream_t st, const char **err)
+                         bool prune, bool contract, bool wide_only, LevelizeScratch &s,
+                         int32_t *level, LevelizeInfo *info, cudaStream_t st, const char **err)
 {
-    *num_levels = 0;
-    *wide_levels = *narrow_levels = 0;
+    *info = LevelizeInfo();
     if (n == 0) return cudaSuccess;
     if (s.n_cap < n) {
         cudaFree(s.ustart); cudaFree(s.uend); cudaFree(s.indeg); cudaFree(s.queue);
         cudaFree(s.lt_ptr); cudaFree(s.lt_fill); cudaFree(s.scan_blk); cudaFree(s.ctrl);
+        cudaFree(s.chain);
         s.ustart = s.uend = s.lt_ptr = s.lt_fill = s.scan_blk = nullptr;
-        s.indeg = s.queue = s.ctrl = nullptr;
+        s.indeg = s.queue = s.ctrl = s.chain = nullptr;
         LV_CK(cudaMalloc(&s.ustart, sizeof(int64_t) * n));
         LV_CK(cudaMalloc(&s.uend, sizeof(int64_t) * n));
         LV_CK(cudaMalloc(&s.indeg, sizeof(int32_t) * n));
@@ -329,13 +434,18 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
         LV_CK(cudaMalloc(&s.lt_fill, sizeof(int64_t) * n));
         LV_CK(cudaMalloc(&s.scan_blk, sizeof(int64_t) * scan_scratch_elems(n)));
         LV_CK(cudaMalloc(&s.ctrl, sizeof(int32_t) * kCtrlInts));
+        LV_CK(cudaMalloc(&s.chain, sizeof(int32_t) * 8 * (size_t)n));
         s.n_cap = n;
     }
+    int32_t *J0 = s.chain, *D0 = J0 + n, *J1 = D0 + n, *D1 = J1 + n, *nxt = D1 + n;
+    int32_t *tail = nxt + n, *len = tail + n, *best = len + n;
     const bool glu3 = rule == 1;
     const int g = aux_grid(n);
+    const int gt = (n + 255) / 256;
     // cons_graph: strict-U ranges (pruned for the U rule)
     k_urange<<<g, kAuxNT, 0, st>>>(n, rp_lu, ci_lu, (prune && !glu3) ? 1 : 0, s.ustart, s.uend);
     LV_CK(cudaGetLastError());
+    info->launches = 1;
     const int64_t *ltp = nullptr;
     const int32_t *lti = nullptr;
     if (glu3) {
@@ -361,19 +471,41 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
         LV_CK(cudaGetLastError());
         ltp = s.lt_ptr;
         lti = s.lt_idx;
+        info->launches += 5;
     }
     // cnt_indegree
     LV_CK(cudaMemsetAsync(s.indeg, 0, sizeof(int32_t) * n, st));
     k_indeg<<<g, kAuxNT, 0, st>>>(n, ci_lu, s.ustart, s.uend, ltp, lti, s.indeg);
     LV_CK(cudaGetLastError());
-    // cons_queue (level 0)
+    // chain contraction (list ranking)
     LV_CK(cudaMemsetAsync(s.ctrl, 0, sizeof(int32_t) * kCtrlInts, st));
-    k_init_queue<<<(n + 255) / 256, 256, 0, st>>>(n, s.indeg, level, s.queue, s.ctrl);
+    k_link_init<<<gt, 256, 0, st>>>(n, J0, D0);
     LV_CK(cudaGetLastError());
-    // Topo: persistent cooperative kernel
-    int dev = 0, sms = 0, occ = 0;
+    k_link<<<gt, 256, 0, st>>>(n, ci_lu, s.ustart, s.uend, ltp, lti, s.indeg, contract ? 1 : 0,
+                               J0, D0, nxt);
+    LV_CK(cudaGetLastError());
+    info->launches += 3;
+    int dev = 0, sms = 0;
     LV_CK(cudaGetDevice(&dev));
     LV_CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    if (contract) {
+        int occ = 0;
+        LV_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_rank, 256, 0));
+        int grid = sms * (occ < 4 ? occ : 4);
+        int32_t *rounds_dev = s.ctrl + 12;
+        int32_t nn = n;
+        void *args[] = {&nn, &J0, &D0, &J1, &D1, &s.ctrl, &rounds_dev};
+        LV_CK(cudaLaunchCooperativeKernel((const void *)k_rank, grid, 256, args, 0, st));
+        info->launches += 1;
+    }
+    k_chain_info<<<gt, 256, 0, st>>>(n, J0, D0, nxt, tail, len);
+    LV_CK(cudaGetLastError());
+    // cons_queue (round 0)
+    k_init_queue<<<gt, 256, 0, st>>>(n, s.indeg, J0, best, s.queue, s.ctrl);
+    LV_CK(cudaGetLastError());
+    info->launches += 2;
+    // Topo: persistent cooperative kernel over chain heads
+    int occ = 0;
     LV_CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_kahn, kKahnNT, 0));
     if (occ < 1) {
         *err = "k_kahn cannot be resident";
@@ -387,20 +519,27 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
     A.ue = s.uend;
     A.ltp = ltp;
     A.lti = lti;
+    A.tail = tail;
+    A.len = len;
     A.indeg = s.indeg;
-    A.level = level;
+    A.best = best;
     A.queue = s.queue;
     A.ctrl = s.ctrl;
     A.narrow_max = kNarrowMax;
     A.wide_only = wide_only ? 1 : 0;
     void *args[] = {&A};
     LV_CK(cudaLaunchCooperativeKernel((const void *)k_kahn, grid, kKahnNT, args, 0, st));
+    k_expand<<<gt, 256, 0, st>>>(n, J0, D0, best, level, s.ctrl);
+    LV_CK(cudaGetLastError());
+    info->launches += 2;
     int32_t ctrl[kCtrlInts];
     LV_CK(cudaMemcpyAsync(ctrl, s.ctrl, sizeof(ctrl), cudaMemcpyDeviceToHost, st));
     LV_CK(cudaStreamSynchronize(st));
-    *num_levels = ctrl[kLevel];
-    *wide_levels = ctrl[kWide];
-    *narrow_levels = ctrl[kNarrow];
+    info->num_levels = ctrl[kMaxLevel] + 1;
+    info->rounds = ctrl[kRound];
+    info->wide_rounds = ctrl[kWide];
+    info->narrow_rounds = ctrl[kNarrow];
+    info->rank_rounds = contract ? ctrl[12] : 0;
     return cudaSuccess;
 }
 

@@ -461,23 +461,25 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
     LevelizeScratch tmp;
     LevelizeScratch &scr = h ? h->lev : tmp;
     const int flags = h ? h->opts.flags : 0;
-    int32_t nl = 0, wl = 0, nrw = 0;
     const char *where = "";
+    LevelizeInfo info;
     if (h) ev_begin(h, kEvLev, s);
     cudaError_t e = levelize_run(n, d_row_ptr_lu, d_col_idx_lu, dep_rule,
-                                 !(flags & LU_F_NO_PRUNE), (flags & LU_F_KAHN_WIDE_ONLY) != 0,
-                                 scr, d_level, &nl, &wl, &nrw, s, &where);
+                                 !(flags & LU_F_NO_PRUNE), !(flags & LU_F_NO_CONTRACT),
+                                 (flags & LU_F_KAHN_WIDE_ONLY) != 0, scr, d_level, &info, s,
+                                 &where);
     if (h) ev_end(h, kEvLev, s);
     if (!h) levelize_free(tmp);
     if (e != cudaSuccess)
         return fail(e == cudaErrorMemoryAllocation ? LU_ERR_NOMEM : LU_ERR_CUDA,
                     "levelize: %s: %s", where, cudaGetErrorString(e));
-    if (num_levels) *num_levels = nl;
+    if (num_levels) *num_levels = info.num_levels;
     if (h) {
-        h->launches += n > 0 ? (dep_rule == LU_DEP_GLU3 ? 9 : 4) : 0;
-        h->stats.num_levels = nl;
-        h->stats.levelize_wide_levels = wl;
-        h->stats.levelize_narrow_levels = nrw;
+        h->launches += info.launches;
+        h->stats.num_levels = info.num_levels;
+        h->stats.levelize_wide_levels = info.wide_rounds;
+        h->stats.levelize_narrow_levels = info.narrow_rounds;
+        h->stats.levelize_rank_rounds = info.rank_rounds;
     }
     return LU_OK;
 }

@@ -139,7 +139,8 @@ KNOBS = [
     dict(threads_per_row=128), dict(threads_per_row=512), dict(threads_per_row=1024),
     dict(ell_width=4), dict(ell_width=8),
     dict(flags=lu.F_GLOBAL_BITMAP, queue_capacity=32, rows_in_flight=5),
-    dict(flags=lu.F_NO_PRUNE), dict(flags=lu.F_KAHN_WIDE_ONLY),
+    dict(flags=lu.F_NO_PRUNE), dict(flags=lu.F_KAHN_WIDE_ONLY), dict(flags=lu.F_NO_CONTRACT),
+    dict(flags=lu.F_NO_CONTRACT | lu.F_NO_PRUNE | lu.F_KAHN_WIDE_ONLY),
 ]
 
 
