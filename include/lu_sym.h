@@ -67,7 +67,9 @@ enum {
                                     i.e. heaviest-first)                      */
     LU_F_NO_PRUNE = 1 << 3,      /* levelize over every U edge (no transitive pruning)       */
     LU_F_KAHN_WIDE_ONLY = 1 << 4,/* levelize: never use the single-CTA narrow phase          */
-    LU_F_NO_CONTRACT = 1 << 5    /* levelize: Kahn over every column (no chain contraction)  */
+    LU_F_NO_CONTRACT = 1 << 5,   /* levelize: Kahn over every column (no chain contraction)  */
+    LU_F_TWO_PASS = 1 << 6       /* no staging pool: emit re-runs the traversal (Alg. 3 as
+                                    printed, symbolic_2 repeats symbolic_1's work)           */
 };
 
 typedef struct {
@@ -78,7 +80,10 @@ typedef struct {
     int32_t rows_in_flight;        /* 0 => planner (all resident CTAs); > 0 caps it          */
     int32_t queue_capacity;        /* shared-memory frontier entries per buffer; 0 => planner */
     int32_t ell_width;             /* traversal adjacency width 4 or 8; 0 => planner         */
-    int32_t reserved[8];
+    uint64_t pool_bytes;           /* HBM staging pool for the rows found by lu_sym_count, so
+                                      lu_sym_emit places them instead of re-traversing;
+                                      0 => min(32 GiB, what the budget leaves)              */
+    int32_t reserved[6];
 } lu_sym_opts;
 
 typedef struct {
@@ -99,7 +104,9 @@ typedef struct {
     int32_t num_levels;           /* after lu_levelize with this handle                      */
     int32_t levelize_wide_levels, levelize_narrow_levels; /* Kahn rounds by mode            */
     int32_t levelize_rank_rounds; /* pointer-jumping rounds of the chain contraction        */
-    int32_t reserved[4];
+    int32_t reserved[2];
+    int64_t pool_bytes;           /* staging pool size (0: two-pass mode)                    */
+    int64_t rows_retraversed;     /* rows of the last emit that were not staged              */
     int64_t kernel_launches;      /* kernels this handle launched since create (all calls)  */
 } lu_sym_stats;
 

@@ -37,7 +37,7 @@ LU_OK, LU_ERR_ARG, LU_ERR_INPUT, LU_ERR_NOMEM, LU_ERR_CAPACITY = 0, 1, 2, 3, 4
 LU_ERR_CUDA, LU_ERR_STATE, LU_ERR_INTERNAL = 5, 7, 8
 DEP_U, DEP_GLU3 = 0, 1
 F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4, 8, 16
-F_NO_CONTRACT = 32
+F_NO_CONTRACT, F_TWO_PASS = 32, 64
 
 
 class LuSymError(RuntimeError):
@@ -50,7 +50,8 @@ class _Opts(ctypes.Structure):
     _fields_ = [("struct_size", ctypes.c_int32), ("flags", ctypes.c_int32),
                 ("scratch_budget_bytes", ctypes.c_uint64), ("threads_per_row", ctypes.c_int32),
                 ("rows_in_flight", ctypes.c_int32), ("queue_capacity", ctypes.c_int32),
-                ("ell_width", ctypes.c_int32), ("reserved", ctypes.c_int32 * 8)]
+                ("ell_width", ctypes.c_int32), ("pool_bytes", ctypes.c_uint64),
+                ("reserved", ctypes.c_int32 * 6)]
 
 
 class _Stats(ctypes.Structure):
@@ -66,7 +67,8 @@ class _Stats(ctypes.Structure):
                 ("queue_capacity", ctypes.c_int32), ("num_levels", ctypes.c_int32),
                 ("levelize_wide_levels", ctypes.c_int32),
                 ("levelize_narrow_levels", ctypes.c_int32),
-                ("levelize_rank_rounds", ctypes.c_int32), ("reserved", ctypes.c_int32 * 4),
+                ("levelize_rank_rounds", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2),
+                ("pool_bytes", ctypes.c_int64), ("rows_retraversed", ctypes.c_int64),
                 ("kernel_launches", ctypes.c_int64)]
 
 
@@ -143,6 +145,7 @@ class Options:
     rows_in_flight: int = 0
     queue_capacity: int = 0
     ell_width: int = 0
+    pool_bytes: int = 0
 
     def to_c(self) -> _Opts:
         o = _Opts()
@@ -153,6 +156,7 @@ class Options:
         o.rows_in_flight = self.rows_in_flight
         o.queue_capacity = self.queue_capacity
         o.ell_width = self.ell_width
+        o.pool_bytes = self.pool_bytes
         return o
 
 

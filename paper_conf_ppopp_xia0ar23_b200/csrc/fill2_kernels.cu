@@ -33,6 +33,7 @@ struct Hdr {
     int row, minseed, diag, tns, newmin, ucnt, lmin, lmax;
     int cnt[3];
     int pad;
+    long long stage_off;
     int scan[40];
 };
 static_assert(sizeof(Hdr) <= kHdrBytes, "header too large");
@@ -309,7 +310,9 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, uint32_t *bm, int32_t *qA, int
     }
 }
 
-template <int NT, int W, bool EMIT, bool GB>
+// MODE: kCount (symbolic_1, counts only), kStage (counts + rows staged into the HBM pool, so
+// symbolic_2 becomes a placement copy), kEmit (symbolic_2 by traversal, into the final CSR).
+template <int NT, int W, int MODE, bool GB>
 __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
 {
     extern __shared__ __align__(16) unsigned char smem[];
@@ -334,8 +337,11 @@ __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
         if (tid == 0) {
             const unsigned long long c = atomicAdd(p.row_counter, 1ull);
             int r = -1;
-            if (c < (unsigned long long)nrows)
+            if (p.row_list) {
+                if (c < (unsigned long long)p.list_len) r = p.row_list[c];
+            } else if (c < (unsigned long long)nrows) {
                 r = p.descending ? p.row_end - 1 - (int)c : p.row_begin + (int)c;
+            }
             h.row = r;
             h.minseed = r;
             h.diag = 0;
@@ -371,10 +377,16 @@ __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
 
         int ptr = h.minseed - 1;  // every unprocessed threshold is > ptr
         int Lcnt = 0;
-        int64_t obase = 0, oend = 0;
-        if constexpr (EMIT) {
-            obase = p.rp_lu[i];
-            oend = p.rp_lu[i + 1];
+        // destination of the L entries (written in threshold order, i.e. sorted)
+        int32_t *ldst = nullptr;
+        int64_t lcap = 0;
+        if constexpr (MODE == kEmit) {
+            const int64_t obase = p.rp_lu[i];
+            ldst = p.ci_lu + obase;
+            lcap = p.rp_lu[i + 1] - obase;
+        } else if constexpr (MODE == kStage) {
+            ldst = p.stg + (size_t)blockIdx.x * p.spill_cap;
+            lcap = p.n;
         }
         // ---- thresholds in increasing order (L130)
         for (;;) {
@@ -464,9 +476,9 @@ __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
             const int m = min(tns, h.newmin);
             const int last = qA[wc - 1];
             if (m > last) {  // the whole window is processed
-                if constexpr (EMIT)
+                if constexpr (MODE != kCount)
                     for (int k = tid; k < wc; k += NT)
-                        if (obase + Lcnt + k < oend) p.ci_lu[obase + Lcnt + k] = qA[k];
+                        if (Lcnt + k < lcap) ldst[Lcnt + k] = qA[k];
                 Lcnt += wc;
                 ptr = last;
                 __syncthreads();
@@ -479,13 +491,13 @@ __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
                 if (qA[mid] < m) lo = mid + 1; else hi = mid;
             }
             const int e = lo;
-            if constexpr (EMIT)
+            if constexpr (MODE != kCount)
                 for (int k = tid; k < e; k += NT)
-                    if (obase + Lcnt + k < oend) p.ci_lu[obase + Lcnt + k] = qA[k];
+                    if (Lcnt + k < lcap) ldst[Lcnt + k] = qA[k];
             Lcnt += e;
             if (m == tns) {  // smallest pending threshold needs a below-exploration
-                if constexpr (EMIT)
-                    if (tid == 0 && obase + Lcnt < oend) p.ci_lu[obase + Lcnt] = m;
+                if constexpr (MODE != kCount)
+                    if (tid == 0 && Lcnt < lcap) ldst[Lcnt] = m;
                 Lcnt += 1;
                 __syncthreads();
                 bfs<NT, W, GB>(p, h, bm, qA, qB, gA, gB, i, m, a);
@@ -502,14 +514,33 @@ __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
         if (a.lmax > i) atomicMax(&h.lmax, a.lmax);
         __syncthreads();
         const int ucnt = h.ucnt, diag = h.diag, gmin = h.lmin, gmax = h.lmax;
-        if constexpr (!EMIT) {
-            if (tid == 0) p.fill_count[i] = Lcnt + diag + ucnt;
+        const int len = Lcnt + diag + ucnt;
+        if constexpr (MODE == kCount) {
+            if (tid == 0) p.fill_count[i] = len;
+        } else if constexpr (MODE == kStage) {
+            // reserve len entries of the pool; rows that do not fit are re-traversed by emit
+            if (tid == 0) {
+                p.fill_count[i] = len;
+                const unsigned long long off = atomicAdd(p.pool_cursor, (unsigned long long)len);
+                const bool fits = off + (unsigned long long)len <= (unsigned long long)p.pool_cap;
+                h.stage_off = fits ? (long long)off : -1ll;
+                p.row_off[i] = fits ? (int64_t)off : -1;
+                if (!fits) p.unstaged[atomicAdd(p.unstaged_cnt, 1ull)] = i;
+            }
+            __syncthreads();
+            const long long off = h.stage_off;
+            if (off >= 0) {
+                int32_t *dst = p.pool + off;
+                for (int k = tid; k < Lcnt; k += NT) dst[k] = ldst[k];
+                if (diag && tid == 0) dst[Lcnt] = i;
+                emit_bits<NT, GB>(bm, i + 1, gmax + 1, dst + Lcnt + diag, h.scan);
+            }
         } else {
-            if (oend - obase != (int64_t)Lcnt + diag + ucnt) {
+            if (lcap != (int64_t)len) {
                 if (tid == 0) atomicAdd(p.stats + kStatErr, 1ull);
             } else {
-                if (diag && tid == 0) p.ci_lu[obase + Lcnt] = i;
-                emit_bits<NT, GB>(bm, i + 1, gmax + 1, p.ci_lu + obase + Lcnt + diag, h.scan);
+                if (diag && tid == 0) ldst[Lcnt] = i;
+                emit_bits<NT, GB>(bm, i + 1, gmax + 1, ldst + Lcnt + diag, h.scan);
             }
         }
         // ---- clear the dirty word range (fill(:) = 0 for the next row, L115)
@@ -532,38 +563,52 @@ __global__ void __launch_bounds__(NT) fill2_kernel(const Fill2Params p)
     }
 }
 
-template <int NT, int W, bool EMIT, bool GB>
-cudaError_t launch_one(const Fill2Params &p, int grid, size_t smem, cudaStream_t s)
+template <int NT, int W, bool GB>
+cudaError_t launch_one(const Fill2Params &p, int mode, int grid, size_t smem, cudaStream_t s)
 {
-    fill2_kernel<NT, W, EMIT, GB><<<grid, NT, smem, s>>>(p);
+    if (mode == kCount)
+        fill2_kernel<NT, W, kCount, GB><<<grid, NT, smem, s>>>(p);
+    else if (mode == kStage)
+        fill2_kernel<NT, W, kStage, GB><<<grid, NT, smem, s>>>(p);
+    else
+        fill2_kernel<NT, W, kEmit, GB><<<grid, NT, smem, s>>>(p);
     return cudaGetLastError();
 }
 
-template <int NT, int W, bool GB>
-cudaError_t configure_one(size_t smem)
+template <int NT, int W, int MODE, bool GB>
+cudaError_t configure_mode(size_t smem)
 {
-    cudaError_t e = cudaFuncSetAttribute(fill2_kernel<NT, W, false, GB>,
+    cudaError_t e = cudaFuncSetAttribute(fill2_kernel<NT, W, MODE, GB>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(fill2_kernel<NT, W, true, GB>,
-                             cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    cudaFuncSetAttribute(fill2_kernel<NT, W, false, GB>,
-                         cudaFuncAttributePreferredSharedMemoryCarveout, 100);
-    cudaFuncSetAttribute(fill2_kernel<NT, W, true, GB>,
+    cudaFuncSetAttribute(fill2_kernel<NT, W, MODE, GB>,
                          cudaFuncAttributePreferredSharedMemoryCarveout, 100);
     return cudaSuccess;
 }
 
 template <int NT, int W, bool GB>
+cudaError_t configure_one(size_t smem)
+{
+    cudaError_t e = configure_mode<NT, W, kCount, GB>(smem);
+    if (e == cudaSuccess) e = configure_mode<NT, W, kStage, GB>(smem);
+    if (e == cudaSuccess) e = configure_mode<NT, W, kEmit, GB>(smem);
+    return e;
+}
+
+template <int NT, int W, bool GB>
 cudaError_t occupancy_one(size_t smem, int *occ)
 {
-    int a = 0, b = 0;
+    int a = 0, b = 0, c = 0;
     cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(
-        &a, fill2_kernel<NT, W, false, GB>, NT, smem);
-    if (e != cudaSuccess) return e;
-    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fill2_kernel<NT, W, true, GB>, NT, smem);
+        &a, fill2_kernel<NT, W, kCount, GB>, NT, smem);
+    if (e == cudaSuccess)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&b, fill2_kernel<NT, W, kStage, GB>, NT,
+                                                          smem);
+    if (e == cudaSuccess)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c, fill2_kernel<NT, W, kEmit, GB>, NT,
+                                                          smem);
     *occ = a < b ? a : b;
+    *occ = *occ < c ? *occ : c;
     return e;
 }
 
@@ -601,13 +646,11 @@ cudaError_t fill2_occupancy(int nt, int w, bool gb, size_t smem, int *occ)
     return cudaErrorInvalidValue;
 }
 
-cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, bool emit, bool gb, int grid,
+cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, int mode, bool gb, int grid,
                          size_t smem, cudaStream_t s)
 {
 #define LCH(NTV, WV, GBV)                                                                    \
-    LUSYM_DISPATCH(NTV, WV, GBV,                                                             \
-                   (emit ? launch_one<NTV, WV, true, GBV>(p, grid, smem, s)                  \
-                         : launch_one<NTV, WV, false, GBV>(p, grid, smem, s)))
+    LUSYM_DISPATCH(NTV, WV, GBV, (launch_one<NTV, WV, GBV>(p, mode, grid, smem, s)))
     LCH(128, 4, false) LCH(128, 4, true) LCH(128, 8, false) LCH(128, 8, true)
     LCH(256, 4, false) LCH(256, 4, true) LCH(256, 8, false) LCH(256, 8, true)
     LCH(512, 4, false) LCH(512, 4, true) LCH(512, 8, false) LCH(512, 8, true)

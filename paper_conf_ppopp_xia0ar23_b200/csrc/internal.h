@@ -34,13 +34,25 @@ struct Fill2Params {
     int32_t wcap;             // window capacity (<= q); 1 = one threshold at a time
     unsigned long long *row_counter;
     unsigned long long *stats;  // kStatCount slots
+    // rows taken from row_list[0..list_len) instead of [row_begin, row_end) when non-null
+    const int32_t *row_list;
+    int32_t list_len;
+    // staging (kStage): per-CTA L buffer (spill_cap entries), pool, per-row pool offset
+    int32_t *stg;
+    int32_t *pool;
+    int64_t pool_cap;
+    int64_t *row_off;
+    unsigned long long *pool_cursor;
+    int32_t *unstaged;
+    unsigned long long *unstaged_cnt;
 };
+enum Fill2Mode { kCount = 0, kEmit = 1, kStage = 2 };
 
 // fill2_kernels.cu
 size_t fill2_smem_bytes(int n, int q, bool global_bitmap);
 cudaError_t fill2_configure(int nt, int w, bool gb, size_t smem);
 cudaError_t fill2_occupancy(int nt, int w, bool gb, size_t smem, int *occ);
-cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, bool emit, bool gb, int grid,
+cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, int mode, bool gb, int grid,
                          size_t smem, cudaStream_t s);
 
 // prep_kernels.cu
@@ -53,6 +65,14 @@ cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, in
 cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,
                         cudaStream_t s);
 size_t scan_scratch_elems(int32_t n);
+
+// place_kernels.cu — symbolic_2 for staged rows: copy pool rows to their CSR slots
+cudaError_t place_rows(int32_t row_begin, int32_t row_end, const int64_t *rp_lu,
+                       const int64_t *row_off, const int32_t *pool, int32_t *ci_lu,
+                       int64_t base, int64_t total, cudaStream_t s);
+// rows of [row_begin, row_end) with row_off < 0 -> list[0..*cnt)
+cudaError_t collect_unstaged(int32_t row_begin, int32_t row_end, const int64_t *row_off,
+                             int32_t *list, unsigned long long *cnt, cudaStream_t s);
 
 // levelize_kernels.cu
 struct LevelizeScratch {

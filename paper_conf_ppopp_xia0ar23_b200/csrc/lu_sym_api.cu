@@ -6,6 +6,8 @@
 #include <cstdio>
 #include <cstring>
 #include <string>
+#include <utility>
+#include <vector>
 
 using namespace lusym;
 
@@ -33,6 +35,7 @@ lu_status fail(lu_status s, const char *fmt, ...)
     } while (0)
 
 enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvN = 4 };
+enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11 };
 
 }  // namespace
 
@@ -54,9 +57,19 @@ struct lu_sym {
     int64_t gb_stride = 0;
     int32_t *gspill = nullptr;
     int64_t spill_cap = 0;
-    unsigned long long *dstats = nullptr;  // [0] row counter, [1..4] count pass, [5..8] emit
+    unsigned long long *dstats = nullptr;  // [0] row counter, [1..4] count pass, [5..8] emit,
+                                           // [9] pool cursor, [10] unstaged rows, [11] list n
     int64_t *scan_blk = nullptr;
     int64_t *dbad = nullptr;
+    uint64_t budget = 0;
+    // staging (count writes every row to the pool; emit places it)
+    bool staging = true;
+    int32_t *stg = nullptr;      // per CTA: L entries of the row in flight (spill_cap each)
+    int32_t *pool = nullptr;
+    int64_t pool_cap = 0;        // entries; -1 = no pool could be allocated
+    int64_t *row_off = nullptr;  // [n] pool offset of each staged row, -1 = not staged
+    int32_t *unstaged = nullptr; // [n] rows that overflowed the pool / row list for re-traversal
+    std::vector<std::pair<int32_t, int32_t>> staged;  // row ranges staged since the last reset
     // state
     bool scanned = false;
     int64_t nnz_lu = 0;
@@ -100,6 +113,10 @@ void free_handle(lu_sym *h)
     cudaFree(h->dstats);
     cudaFree(h->scan_blk);
     cudaFree(h->dbad);
+    cudaFree(h->stg);
+    cudaFree(h->pool);
+    cudaFree(h->row_off);
+    cudaFree(h->unstaged);
     levelize_free(h->lev);
     for (int k = 0; k < kEvN; ++k)
         for (int j = 0; j < 2; ++j)
@@ -164,7 +181,10 @@ lu_status plan(lu_sym *h)
     const int64_t nw = ((int64_t)n + 31) / 32;
     h->gb_stride = (nw + 31) & ~(int64_t)31;  // 128 B aligned slots
     h->spill_cap = n > 0 ? n : 1;
-    const uint64_t per_row = (uint64_t)2 * h->spill_cap * 4 + (h->gb ? (uint64_t)h->gb_stride * 4 : 0);
+    h->staging = !(h->opts.flags & LU_F_TWO_PASS);
+    h->budget = budget;
+    const uint64_t per_row = (uint64_t)(h->staging ? 3 : 2) * h->spill_cap * 4 +
+                             (h->gb ? (uint64_t)h->gb_stride * 4 : 0);
     const uint64_t fit = budget / per_row;
     if (fit < 1)
         return fail(LU_ERR_NOMEM, "scratch budget %llu B < one row's scratch %llu B",
@@ -177,6 +197,11 @@ lu_status plan(lu_sym *h)
     if (h->gb) {
         st = dalloc(h, &h->gbitmap, (size_t)h->gb_stride * h->grid);
         if (st != LU_OK) return st;
+    }
+    if ((st = dalloc(h, &h->unstaged, (size_t)n)) != LU_OK) return st;
+    if (h->staging) {
+        if ((st = dalloc(h, &h->stg, (size_t)h->spill_cap * h->grid)) != LU_OK) return st;
+        if ((st = dalloc(h, &h->row_off, (size_t)n)) != LU_OK) return st;
     }
     return LU_OK;
 }
@@ -196,9 +221,11 @@ void ev_end(lu_sym *h, int k, cudaStream_t s)
     h->ev_used[k] = true;
 }
 
-lu_status run_pass(lu_sym *h, bool emit, int32_t rb, int32_t re, int32_t *fill_count,
-                   const int64_t *rp_lu, int32_t *ci_lu, cudaStream_t s)
+lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_count,
+                   const int64_t *rp_lu, int32_t *ci_lu, cudaStream_t s,
+                   const int32_t *row_list = nullptr, int32_t list_len = 0)
 {
+    const bool emit = mode == kEmit;
     unsigned long long *st = h->dstats + (emit ? 5 : 1);
     CK(cudaMemsetAsync(h->dstats, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(st, 0, sizeof(unsigned long long) * kStatCount, s));
@@ -224,10 +251,51 @@ lu_status run_pass(lu_sym *h, bool emit, int32_t rb, int32_t re, int32_t *fill_c
     p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : h->q;
     p.row_counter = h->dstats;
     p.stats = st;
+    p.row_list = row_list;
+    p.list_len = list_len;
+    p.stg = h->stg;
+    p.pool = h->pool;
+    p.pool_cap = h->pool_cap;
+    p.row_off = h->row_off;
+    p.pool_cursor = h->dstats + kSlotPoolCursor;
+    p.unstaged = h->unstaged;
+    p.unstaged_cnt = h->dstats + kSlotUnstaged;
+    int rows = row_list ? list_len : re - rb;
     int grid = h->grid;
-    if (grid > re - rb) grid = re - rb;
-    CK(fill2_launch(p, h->nt, h->w, emit, h->gb, grid, h->smem, s));
+    if (grid > rows) grid = rows;
+    if (grid < 1) return LU_OK;
+    CK(fill2_launch(p, h->nt, h->w, mode, h->gb, grid, h->smem, s));
     h->launches += 1;
+    return LU_OK;
+}
+
+// Staging pool (HBM): allocated on the first staged count, kept for the handle's lifetime.
+lu_status ensure_pool(lu_sym *h)
+{
+    if (h->pool || h->pool_cap < 0) return LU_OK;
+    size_t free_b = 0, total_b = 0;
+    CK(cudaMemGetInfo(&free_b, &total_b));
+    uint64_t want = h->opts.pool_bytes;
+    if (want == 0) {
+        const uint64_t budget = h->budget > (uint64_t)h->scratch_bytes
+                                    ? h->budget - (uint64_t)h->scratch_bytes : 0;
+        want = budget < (32ull << 30) ? budget : (32ull << 30);
+        if (want > (uint64_t)(0.9 * (double)free_b)) want = (uint64_t)(0.9 * (double)free_b);
+    }
+    int64_t cap = (int64_t)(want / sizeof(int32_t));
+    if (cap < 1) {
+        h->pool_cap = -1;  // no room: every row is re-traversed by emit
+        return LU_OK;
+    }
+    cudaError_t e = cudaMalloc(&h->pool, (size_t)cap * sizeof(int32_t));
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        h->pool = nullptr;
+        h->pool_cap = -1;
+        return LU_OK;
+    }
+    h->pool_cap = cap;
+    h->scratch_bytes += cap * (int64_t)sizeof(int32_t);
     return LU_OK;
 }
 
@@ -363,7 +431,25 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
     if (st != LU_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
     ev_begin(h, kEvCount, s);
-    st = run_pass(h, false, row_begin, row_end, d_fill_count, nullptr, nullptr, s);
+    int mode = kCount;
+    if (h->staging) {
+        st = ensure_pool(h);
+        if (st != LU_OK) return st;
+        if (h->pool) {
+            mode = kStage;
+            bool overlap = false;
+            for (auto &r : h->staged)
+                if (row_begin < r.second && r.first < row_end) overlap = true;
+            if (overlap || h->staged.empty()) {  // restart the pool
+                h->staged.clear();
+                CK(cudaMemsetAsync(h->row_off, 0xff, sizeof(int64_t) * (size_t)h->n, s));
+                CK(cudaMemsetAsync(h->dstats + kSlotPoolCursor, 0, 2 * sizeof(unsigned long long),
+                                   s));
+            }
+            h->staged.emplace_back(row_begin, row_end);
+        }
+    }
+    st = run_pass(h, mode, row_begin, row_end, d_fill_count, nullptr, nullptr, s);
     ev_end(h, kEvCount, s);
     return st;
 }
@@ -413,9 +499,31 @@ lu_status lu_sym_emit(lu_sym *h, int32_t row_begin, int32_t row_end, const int64
         return fail(LU_ERR_CAPACITY, "cap %lld < %lld entries needed", (long long)cap,
                     (long long)need);
     ev_begin(h, kEvEmit, s);
-    st = run_pass(h, true, row_begin, row_end, nullptr, d_row_ptr_lu, d_col_idx_lu, s);
+    int64_t retraverse = row_end - row_begin;
+    if (h->staging && !h->staged.empty()) {
+        // symbolic_2 for the staged rows: place them; re-traverse only the others
+        int64_t first = 0;
+        CK(cudaMemcpyAsync(&first, d_row_ptr_lu + row_begin, sizeof(int64_t),
+                           cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        CK(place_rows(row_begin, row_end, d_row_ptr_lu, h->row_off, h->pool, d_col_idx_lu, first,
+                      need - first, s));
+        CK(collect_unstaged(row_begin, row_end, h->row_off, h->unstaged, h->dstats + kSlotList,
+                            s));
+        unsigned long long nun = 0;
+        CK(cudaMemcpyAsync(&nun, h->dstats + kSlotList, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        h->launches += 2;
+        retraverse = (int64_t)nun;
+        if (nun > 0)
+            st = run_pass(h, kEmit, row_begin, row_end, nullptr, d_row_ptr_lu, d_col_idx_lu, s,
+                          h->unstaged, (int32_t)nun);
+    } else {
+        st = run_pass(h, kEmit, row_begin, row_end, nullptr, d_row_ptr_lu, d_col_idx_lu, s);
+    }
     ev_end(h, kEvEmit, s);
     if (st != LU_OK) return st;
+    h->stats.rows_retraversed = retraverse;
     unsigned long long err = 0;
     CK(cudaMemcpyAsync(&err, h->dstats + 5 + kStatErr, 8, cudaMemcpyDeviceToHost, s));
     CK(cudaStreamSynchronize(s));
@@ -515,6 +623,7 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
     h->stats.ell_width = h->w;
     h->stats.queue_capacity = h->q;
     h->stats.kernel_launches = h->launches;
+    h->stats.pool_bytes = h->pool ? h->pool_cap * (int64_t)sizeof(int32_t) : 0;
     *out = h->stats;
     return LU_OK;
 }

@@ -141,6 +141,9 @@ KNOBS = [
     dict(flags=lu.F_GLOBAL_BITMAP, queue_capacity=32, rows_in_flight=5),
     dict(flags=lu.F_NO_PRUNE), dict(flags=lu.F_KAHN_WIDE_ONLY), dict(flags=lu.F_NO_CONTRACT),
     dict(flags=lu.F_NO_CONTRACT | lu.F_NO_PRUNE | lu.F_KAHN_WIDE_ONLY),
+    dict(flags=lu.F_TWO_PASS),                       # Alg. 3 as printed: emit re-traverses
+    dict(pool_bytes=4096),                           # pool overflow: most rows re-traversed
+    dict(pool_bytes=200_000),                        # partial staging
 ]
 
 
@@ -149,6 +152,13 @@ def test_knobs_do_not_change_results(knob):
     for rp, ci in (gen.lap3d(9), gen.circuit(40, 2), gen.random_pattern(700, 2.5, seed=9),
                    gen.lap2d(20)):
         check(rp, ci, tag=str(knob), **knob)
+
+
+def test_pool_overflow_falls_back_to_traversal():
+    g = check(*gen.circuit(64, 5), tag="pool", pool_bytes=64_000)
+    assert 0 < g["stats"]["rows_retraversed"] < 4096
+    g = check(*gen.circuit(64, 5), tag="pool-full")
+    assert g["stats"]["rows_retraversed"] == 0 and g["stats"]["pool_bytes"] > 0
 
 
 def test_spills_are_exercised():
