@@ -50,6 +50,9 @@ def parse():
     ap.add_argument("--cpu-sample-stride", type=int, default=0,
                     help="oracle sample: every s-th row (0 = auto, ~10-30 s of CPU work)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras)")
+    ap.add_argument("--flags", type=int, default=0, help="lu_sym_opts.flags (LU_F_*)")
+    ap.add_argument("--threads-per-row", type=int, default=0)
+    ap.add_argument("--queue-capacity", type=int, default=0)
     return ap.parse_args()
 
 
@@ -218,7 +221,9 @@ def run_ours(args, rank, world, local_rank):
     te, sv = work_units(rp_np)
     rp = torch.from_numpy(rp_np).to(dev)
     ci = torch.from_numpy(ci_np).to(dev)
-    h = lu.Symbolic(rp, ci)
+    sym_opts = dict(flags=args.flags, threads_per_row=args.threads_per_row,
+                    queue_capacity=args.queue_capacity)
+    h = lu.Symbolic(rp, ci, **sym_opts)
     cost = lu.row_cost_upper_bound(rp_np)
     bounds = lu.partition_rows(cost, world)
     rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
@@ -321,7 +326,7 @@ def run_ours(args, rank, world, local_rank):
             a.record(stream)
             rpd = rp_h.to(dev, non_blocking=True)
             cid = ci_h.to(dev, non_blocking=True)
-            he = lu.Symbolic(rpd, cid)                         # S1 + S2 (validate, plan)
+            he = lu.Symbolic(rpd, cid, **sym_opts)             # S1 + S2 (validate, plan)
             fc = torch.zeros(n, dtype=torch.int32, device=dev)
             he.count(rb, re_, fc)
             if world > 1:

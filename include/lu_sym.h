@@ -179,6 +179,14 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
 /* Copy the handle's statistics to *out (host). */
 lu_status lu_sym_get_stats(const lu_sym *h, lu_sym_stats *out);
 
+/*
+ * Diagnostics (the paper's Fig. 3 per-row frontier profile, L249/L272): with d_prof != NULL
+ * (device int64[4 n], borrowed) every later lu_sym_count records, for each row i it processes,
+ * d_prof[4i+0] = SM clock cycles spent on the row, [4i+1] = vertices scanned, [4i+2] = BFS runs
+ * (non-simple thresholds), [4i+3] = threshold windows.  NULL switches recording off.
+ */
+lu_status lu_sym_set_row_profile(lu_sym *h, int64_t *d_prof);
+
 /* Free the handle's scratch (synchronises its streams).  NULL is a no-op. */
 void lu_sym_destroy(lu_sym *h);
 

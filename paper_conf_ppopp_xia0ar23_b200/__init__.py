@@ -76,7 +76,7 @@ _lib = None
 
 EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sym_count",
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
-            "lu_sym_destroy", "lu_status_str", "lu_last_error"]
+            "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile"]
 
 
 def library_path() -> str:
@@ -103,6 +103,8 @@ def load_library():
     lib.lu_levelize.argtypes = [P, I32, P, P, I32, P, P, P]
     lib.lu_sym_get_stats.argtypes = [P, P]
     lib.lu_sym_destroy.argtypes = [P]
+    lib.lu_sym_set_row_profile.argtypes = [P, P]
+    lib.lu_sym_set_row_profile.restype = I32
     lib.lu_status_str.argtypes = [I32]
     lib.lu_status_str.restype = ctypes.c_char_p
     lib.lu_last_error.restype = ctypes.c_char_p
@@ -234,6 +236,17 @@ class Symbolic:
 
     def levelize(self, row_ptr_lu, col_idx_lu, rule: str = "u", level=None, stream=None):
         return levelize(row_ptr_lu, col_idx_lu, rule, level=level, handle=self, stream=stream)
+
+    def set_row_profile(self, prof):
+        """Record a per-row profile on later count passes into prof (int64[n, 4] on the device:
+        cycles, vertices scanned, BFS runs, threshold windows); None switches it off."""
+        ptr = None
+        if prof is not None:
+            if prof.dtype != torch.int64 or prof.numel() < 4 * self.n or not prof.is_cuda:
+                raise ValueError("prof must be a CUDA int64 tensor with 4*n elements")
+            ptr = ctypes.c_void_p(prof.data_ptr())
+        self._prof = prof
+        _check(load_library().lu_sym_set_row_profile(self._h, ptr))
 
     def stats(self) -> dict:
         st = _Stats()

@@ -1,0 +1,745 @@
+// fill2 traversal kernels (S3 count / S6 emit) for sm_100a — device code, instantiated per CTA
+// size in fill2_nt*.cu.
+//
+// One CTA owns one source row at a time ("symbolic factorization from each
+// source row is independent") and pulls rows from a device counter, heaviest (largest id)
+// first (L272: per-row work grows with the row id).  Per row it runs Algorithm 1 (L110-161):
+//
+//   seed    : mark src and every v in A(src,:)                                  (L116-129)
+//   loop    : thresholds in strictly increasing order (L130) — taken as a sorted WINDOW of the
+//             marked-but-unprocessed vertices in (ptr, src) (reading R4), and
+//             * "simple" thresholds (all below-neighbours already visited) are scanned in
+//               parallel: their unvisited above-neighbours are pattern entries (reading R5b);
+//             * the smallest non-simple threshold t0 runs a level-synchronous BFS over
+//               unvisited vertices < t0 (L131-158); order inside a level is free (R5).
+//   output  : L(src,:) = thresholds in the order the pointer passes them (already sorted),
+//             U(src,:) = visited bits in (src, n) scanned upward (sorted), diagonal iff in A.
+//
+// Visited state: 1 bit per vertex, in shared memory when n/8 bytes fit next to the frontier
+// queues (else in an HBM slot per CTA, reading R3/R25: zeroed per pass, cleared per row over
+// the dirty word range only).  Frontier levels are lists in shared memory, spilling to a
+// per-CTA HBM region of capacity n.  Adjacency is read through an ELL-W copy of A without the
+// diagonal (one 128/256-bit load per scanned vertex); vertices of larger degree are scanned by
+// a whole warp from A's CSR.
+#pragma once
+
+#include "internal.h"
+
+#include <climits>
+
+namespace lusym {
+namespace f2 {
+
+constexpr unsigned kFull = 0xffffffffu;
+constexpr int kSmallWin = 32;  // threshold window after a window was cut short
+
+struct Hdr {
+    int row, minseed, diag, tns, newmin, ucnt, lmin, lmax;
+    int cnt[3];
+    int pad;
+    long long stage_off;
+    int scan[40];
+};
+static_assert(sizeof(Hdr) <= kHdrBytes, "header too large");
+
+template <int NT>
+__device__ __forceinline__ int block_scan_excl(int x, int *s, int &total)
+{
+    constexpr int NW = NT / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    int inc = x;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+        const int y = __shfl_up_sync(kFull, inc, o);
+        if (lane >= o) inc += y;
+    }
+    if (lane == 31) s[wid] = inc;
+    __syncthreads();
+    if (wid == 0) {
+        int v = lane < NW ? s[lane] : 0;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+            const int y = __shfl_up_sync(kFull, v, o);
+            if (lane >= o) v += y;
+        }
+        if (lane < NW) s[lane] = v;
+    }
+    __syncthreads();
+    total = s[NW - 1];
+    const int r = (wid ? s[wid - 1] : 0) + inc - x;
+    __syncthreads();
+    return r;
+}
+
+template <bool GB>
+__device__ __forceinline__ uint32_t bm_word(const uint32_t *bm, int w)
+{
+    if (GB) return __ldcg(bm + w);
+    return bm[w];
+}
+
+template <bool GB>
+__device__ __forceinline__ bool visited(const uint32_t *bm, int v)
+{
+    return (bm_word<GB>(bm, v >> 5) >> (v & 31)) & 1u;
+}
+
+// test-and-set (reading R26): true iff this call set the bit.  The level-1 summary sm gets bit
+// w when visited word w first becomes non-zero, so scans and clears skip empty stretches.
+__device__ __forceinline__ bool mark(uint32_t *bm, uint32_t *sm, int v)
+{
+    const uint32_t b = 1u << (v & 31);
+    const uint32_t old = atomicOr(bm + (v >> 5), b);
+    if (old == 0) atomicOr(sm + (v >> 10), 1u << ((v >> 5) & 31));
+    return !(old & b);
+}
+
+template <int W>
+__device__ __forceinline__ void load_nb(const int32_t *ell, int f, int (&nb)[W])
+{
+    if constexpr (W == 8) {
+        // one 256-bit load per adjacency row (LDG.E.256 on sm_100a)
+        asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+            : "=r"(nb[0]), "=r"(nb[1]), "=r"(nb[2]), "=r"(nb[3]), "=r"(nb[4]), "=r"(nb[5]),
+              "=r"(nb[6]), "=r"(nb[7])
+            : "l"(ell + (size_t)f * W));
+    } else {
+        const int4 a = __ldg(reinterpret_cast<const int4 *>(ell + (size_t)f * W));
+        nb[0] = a.x; nb[1] = a.y; nb[2] = a.z; nb[3] = a.w;
+    }
+}
+
+__device__ __forceinline__ int64_t heavy_off(int lo, int hi)
+{
+    return (int64_t)(uint32_t)lo | ((int64_t)hi << 32);
+}
+
+// warp-aggregated append to a list (smem, spilling to HBM past q entries)
+__device__ __forceinline__ void push(bool pred, int w, int *cnt, int32_t *NF, int32_t *gNF, int q,
+                                     unsigned long long &spills)
+{
+    const unsigned b = __ballot_sync(kFull, pred);
+    if (b == 0) return;
+    const int lane = threadIdx.x & 31;
+    const int leader = __ffs(b) - 1;
+    int base = 0;
+    if (lane == leader) base = atomicAdd(cnt, __popc(b));
+    base = __shfl_sync(kFull, base, leader);
+    if (pred) {
+        const int pos = base + __popc(b & ((1u << lane) - 1u));
+        if (pos < q) {
+            NF[pos] = w;
+        } else {
+            gNF[pos] = w;
+            ++spills;
+        }
+    }
+}
+
+// Smallest visited word index >= w0 whose summary bit is set (may exceed whi within the last
+// summary word), INT_MAX if none up to whi.  Block-uniform; sred: NT/32 ints of scratch.
+template <int NT>
+__device__ int next_word(const uint32_t *sm, int w0, int whi, int *sred)
+{
+    const int shi = whi >> 5;
+    for (int sb = w0 >> 5; sb <= shi; sb += NT) {
+        const int sidx = sb + (int)threadIdx.x;
+        int cand = INT_MAX;
+        if (sidx <= shi) {
+            uint32_t sw = sm[sidx];
+            if (sidx == (w0 >> 5)) sw &= kFull << (w0 & 31);
+            if (sw) cand = (sidx << 5) + __ffs(sw) - 1;
+        }
+        cand = __reduce_min_sync(kFull, cand);
+        if ((threadIdx.x & 31) == 0) sred[threadIdx.x >> 5] = cand;
+        __syncthreads();
+        int r = INT_MAX;
+#pragma unroll
+        for (int k = 0; k < NT / 32; ++k) r = min(r, sred[k]);
+        __syncthreads();
+        if (r != INT_MAX) return r;
+    }
+    return INT_MAX;
+}
+
+// Set bits of (bm & ~dm) in [lo, hi) (dm may be null), in increasing order.  Returns how many
+// there are (at most cap when CAPPED).  WRITE: stores them at dst[base + k] for base + k < dcap.
+// One visited word per thread per chunk; on ranges wider than a chunk the level-1 summary sm
+// skips empty stretches before each chunk.  Block-uniform.
+template <int NT, bool GB, bool WRITE, bool CAPPED>
+__device__ int scan_bits(const uint32_t *bm, const uint32_t *sm, const uint32_t *dm, int lo,
+                         int hi, int32_t *dst, int64_t base, int64_t dcap, int cap, int *sscan)
+{
+    if (lo >= hi) return 0;
+    const int wlo = lo >> 5, whi = (hi - 1) >> 5;
+    const bool wide = whi - wlo >= NT;
+    int count = 0;
+    for (int w0 = wlo; w0 <= whi; w0 += NT) {
+        if (wide) {
+            w0 = next_word<NT>(sm, w0, whi, sscan);
+            if (w0 > whi) break;
+        }
+        const int w = w0 + (int)threadIdx.x;
+        uint32_t word = 0;
+        if (w <= whi) {
+            word = bm_word<GB>(bm, w);
+            if (w == wlo) word &= kFull << (lo & 31);
+            if (w == whi) {
+                const int hb = (hi - 1) & 31;
+                word &= (hb == 31) ? kFull : ((2u << hb) - 1u);
+            }
+            if (dm && word) word &= ~__ldcg(dm + w);
+        }
+        int total;
+        int pos = count + block_scan_excl<NT>(__popc(word), sscan, total);
+        if (WRITE)
+            for (; word; word &= word - 1, ++pos) {
+                const int64_t o = base + pos;
+                if (o < dcap) dst[o] = (w << 5) + __ffs(word) - 1;
+            }
+        count += total;
+        if (CAPPED && count >= cap) break;
+    }
+    if (WRITE) __syncthreads();
+    return CAPPED && count > cap ? cap : count;
+}
+
+// Pending thresholds not yet finished: the first cap set bits of bm & ~dm in [lo, hi), sorted.
+template <int NT, bool GB>
+__device__ __forceinline__ int collect(const uint32_t *bm, const uint32_t *sm, const uint32_t *dm,
+                                       int lo, int hi, int32_t *out, int cap, int *sscan)
+{
+    return scan_bits<NT, GB, true, true>(bm, sm, dm, lo, hi, out, 0, cap, cap, sscan);
+}
+
+// Count the set bits in [lo, hi) and, if WRITE, store them in increasing order at dst[base ..]
+// (bounded by cap).  Returns the count.
+template <int NT, bool GB, bool WRITE>
+__device__ __forceinline__ int emit_range(const uint32_t *bm, const uint32_t *sm, int lo, int hi,
+                                          int32_t *dst, int base, int64_t cap, int *sscan)
+{
+    return scan_bits<NT, GB, WRITE, false>(bm, sm, nullptr, lo, hi, dst, base, cap, 0, sscan);
+}
+
+// Zero the visited words [wlo, whi] and their summary bits (walk the summary if wide).
+template <int NT>
+__device__ void clear_words(uint32_t *bm, uint32_t *sm, int wlo, int whi)
+{
+    if (whi < wlo) return;
+    if (whi - wlo < 4 * NT) {
+        for (int w = wlo + (int)threadIdx.x; w <= whi; w += NT) bm[w] = 0;
+    } else {
+        for (int sidx = (wlo >> 5) + (int)threadIdx.x; sidx <= (whi >> 5); sidx += NT)
+            for (uint32_t t = sm[sidx]; t; t &= t - 1) bm[(sidx << 5) + __ffs(t) - 1] = 0;
+    }
+    __syncthreads();
+    for (int sidx = (wlo >> 5) + (int)threadIdx.x; sidx <= (whi >> 5); sidx += NT) sm[sidx] = 0;
+}
+
+struct RowAcc {
+    int ucnt, lmin, lmax;
+    unsigned long long te, sv, spills;
+};
+
+// Scan the vertices L[0..cnt) (smem, HBM past q) of one BFS level below t0: test-and-set every
+// neighbour; new ones below t0 form the next level (appended to NF), new ones above t0 are
+// pattern entries (L130-147).
+template <int NT, int W, bool GB>
+__device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, uint32_t *sm,
+                                           const int32_t *L,
+                                           const int32_t *gL, int cnt, int *ncnt, int32_t *NF,
+                                           int32_t *gNF, const int i, const int t0, int &nmin,
+                                           RowAcc &a)
+{
+    const int tid = threadIdx.x, lane = tid & 31;
+    for (int base = 0; base < cnt; base += NT) {
+        const int k = base + tid;
+        const bool valid = k < cnt;
+        int nb[W];
+#pragma unroll
+        for (int s = 0; s < W; ++s) nb[s] = -1;
+        bool heavy = false;
+        if (valid) {
+            const int f = k < p.q ? L[k] : __ldcg(gL + k);
+            load_nb<W>(p.ell, f, nb);
+            heavy = nb[0] == kHeavy;
+        }
+        uint32_t frm = 0;
+        if (valid && !heavy) {
+            ++a.sv;
+#pragma unroll
+            for (int s = 0; s < W; ++s) {
+                const int w = nb[s];
+                if (w >= 0 && !visited<GB>(bm, w) && mark(bm, sm, w)) {
+                    if (w < t0) {
+                        frm |= 1u << s;
+                    } else if (w > i) {
+                        ++a.ucnt;
+                        a.lmax = max(a.lmax, w);
+                    }
+                }
+            }
+        }
+        {
+            // one warp-aggregated append for all new frontier vertices of the warp
+            const int c = __popc(frm);
+            int inc = c;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int y = __shfl_up_sync(kFull, inc, o);
+                if (lane >= o) inc += y;
+            }
+            const int total = __shfl_sync(kFull, inc, 31);
+            if (total) {
+                int wbase = 0;
+                if (lane == 31) wbase = atomicAdd(ncnt, total);
+                wbase = __shfl_sync(kFull, wbase, 31);
+                int pos = wbase + inc - c;
+#pragma unroll
+                for (int s = 0; s < W; ++s) {
+                    if (frm & (1u << s)) {
+                        const int w = nb[s];
+                        nmin = min(nmin, w);
+                        if (pos < p.q) {
+                            NF[pos] = w;
+                        } else {
+                            gNF[pos] = w;
+                            ++a.spills;
+                        }
+                        ++pos;
+                    }
+                }
+            }
+        }
+        // heavy vertices (degree > W): one warp each, over A's CSR row
+        unsigned hm = __ballot_sync(kFull, valid && heavy);
+        while (hm) {
+            const int src = __ffs(hm) - 1;
+            hm &= hm - 1;
+            const int len = __shfl_sync(kFull, nb[1], src);
+            const int64_t off =
+                heavy_off(__shfl_sync(kFull, nb[2], src), __shfl_sync(kFull, nb[3], src));
+            if (lane == 0) {
+                a.te += len;
+                ++a.sv;
+            }
+            for (int eb = 0; eb < len; eb += 32) {
+                const int e = eb + lane;
+                bool fr = false;
+                int w = -1;
+                if (e < len) {
+                    w = __ldg(p.ci + off + e);
+                    if (!visited<GB>(bm, w) && mark(bm, sm, w)) {
+                        if (w < t0) {
+                            fr = true;
+                            nmin = min(nmin, w);
+                        } else if (w > i) {
+                            ++a.ucnt;
+                            a.lmax = max(a.lmax, w);
+                        }
+                    }
+                }
+                push(fr, w, ncnt, NF, gNF, p.q, a.spills);
+            }
+        }
+    }
+}
+
+// Level-synchronous BFS from threshold t0 over unvisited vertices < t0 (Alg. 1).
+template <int NT, int W, bool GB>
+__device__ void bfs(const Fill2Params &p, Hdr &h, uint32_t *bm, uint32_t *sm, int32_t *qA,
+                    int32_t *qB,
+                    int32_t *gA, int32_t *gB, const int i, const int t0, RowAcc &a)
+{
+    const int tid = threadIdx.x;
+    int32_t *F = qA, *NF = qB, *gF = gA, *gNF = gB;
+    if (tid == 0) {
+        F[0] = t0;
+        h.cnt[1] = h.cnt[2] = 0;
+    }
+    __syncthreads();
+    int fsize = 1;
+    for (int lev = 0;; ++lev) {
+        int *ncnt = &h.cnt[(lev + 1) % 3];
+        if (tid == 0) h.cnt[(lev + 2) % 3] = 0;
+        int nmin = INT_MAX;
+        scan_level<NT, W, GB>(p, bm, sm, F, gF, fsize, ncnt, NF, gNF, i, t0, nmin, a);
+        a.lmin = min(a.lmin, nmin);
+        __syncthreads();
+        fsize = *ncnt;
+        if (fsize == 0) break;
+        int32_t *t = F; F = NF; NF = t;
+        t = gF; gF = gNF; gNF = t;
+    }
+}
+
+// MODE: kCount (symbolic_1, counts only), kStage (counts + rows staged into the HBM pool, so
+// symbolic_2 becomes a placement copy), kEmit (symbolic_2 by traversal, into the final CSR).
+template <int NT, int W, int MODE, int VIS>
+__global__ void __launch_bounds__(NT, 2048 / NT) fill2_kernel(const Fill2Params p)
+{
+    constexpr bool GB = VIS == kVisGlobal;
+    extern __shared__ __align__(16) unsigned char smem[];
+    Hdr &h = *reinterpret_cast<Hdr *>(smem);
+    int32_t *qA = reinterpret_cast<int32_t *>(smem + kHdrBytes);
+    int32_t *qB = qA + p.q;
+    uint32_t *sm = reinterpret_cast<uint32_t *>(qB + p.q);  // summary (p.sw words)
+    uint32_t *bm;
+    if constexpr (GB)
+        bm = p.gbitmap + (size_t)blockIdx.x * p.gbitmap_stride;
+    else
+        bm = sm + p.sw;
+    int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
+    int32_t *gB = gA + p.spill_cap;
+    const int tid = threadIdx.x, lane = tid & 31;
+    for (int w = tid; w < p.sw; w += NT) sm[w] = 0;
+    if constexpr (!GB)
+        for (int w = tid; w < p.nw; w += NT) bm[w] = 0;
+
+    RowAcc a;
+    a.te = a.sv = a.spills = 0;
+    const int nrows = p.row_end - p.row_begin;
+    for (;;) {
+        if (tid == 0) {
+            const unsigned long long c = atomicAdd(p.row_counter, 1ull);
+            int r = -1;
+            if (p.row_list) {
+                if (c < (unsigned long long)p.list_len) r = p.row_list[c];
+            } else if (c < (unsigned long long)nrows) {
+                r = p.descending ? p.row_end - 1 - (int)c : p.row_begin + (int)c;
+            }
+            h.row = r;
+            h.minseed = r;
+            h.diag = 0;
+            h.ucnt = 0;
+            h.lmin = r;
+            h.lmax = r;
+        }
+        __syncthreads();
+        const int i = h.row;
+        if (i < 0) break;
+        const long long t_row = p.row_prof ? clock64() : 0;
+        const unsigned long long sv_row = a.sv;
+        int n_bfs = 0, n_win = 0;
+        a.ucnt = 0;
+        a.lmin = i;
+        a.lmax = i;
+
+        // ---- seed: fill(src) = src; for v in A(src,:) fill(v) = src  (L116-129)
+        const int64_t rb = p.rp[i], re = p.rp[i + 1];
+        for (int64_t k = rb + tid; k < re; k += NT) {
+            const int v = __ldg(p.ci + k);
+            ++a.te;
+            mark(bm, sm, v);
+            if (v < i) {
+                atomicMin(&h.minseed, v);
+                a.lmin = min(a.lmin, v);
+            } else if (v > i) {
+                ++a.ucnt;
+                a.lmax = max(a.lmax, v);
+            } else {
+                h.diag = 1;
+            }
+        }
+        if (tid == 0) mark(bm, sm, i);
+        __syncthreads();
+
+        int ptr = h.minseed - 1;  // every unprocessed threshold is > ptr
+        int Lcnt = 0;
+        // destination of the L entries (written in threshold order, i.e. sorted)
+        int32_t *ldst = nullptr;
+        int64_t lcap = 0;
+        if constexpr (MODE == kEmit) {
+            const int64_t obase = p.rp_lu[i];
+            ldst = p.ci_lu + obase;
+            lcap = p.rp_lu[i + 1] - obase;
+        } else if constexpr (MODE == kStage) {
+            ldst = p.stg + (size_t)blockIdx.x * p.spill_cap;
+            lcap = p.n;
+        }
+        // "done" marks (HBM slot of this CTA) of simple thresholds processed ahead of the pointer,
+        // so a re-collected window skips them; non-simple ones are re-checked, in a window that
+        // shrinks to kSmallWin after it was cut short and doubles back while it is consumed
+        uint32_t *dm = p.dbitmap + (size_t)blockIdx.x * p.gbitmap_stride;
+        bool dused = false;
+        int cap = p.wcap;
+        // ---- thresholds in increasing order (L130)
+        for (;;) {
+            const int wc = collect<NT, GB>(bm, sm, dused ? dm : nullptr, ptr + 1, i, qA, cap,
+                                           h.scan);
+            if (wc == 0) break;
+            ++n_win;
+            if (tid == 0) {
+                h.tns = INT_MAX;
+                h.newmin = INT_MAX;
+            }
+            __syncthreads();
+            int nm = INT_MAX;
+            for (int base = 0; base < wc; base += NT) {
+                const int k = base + tid;
+                const bool valid = k < wc;
+                const int t = valid ? qA[k] : 0;
+                int nb[W];
+#pragma unroll
+                for (int s = 0; s < W; ++s) nb[s] = -1;
+                bool heavy = false, done = false;
+                if (valid) {
+                    load_nb<W>(p.ell, t, nb);
+                    heavy = nb[0] == kHeavy;
+                }
+                if (valid && !heavy) {
+                    ++a.sv;
+                    bool simple = true;
+#pragma unroll
+                    for (int s = 0; s < W; ++s) {
+                        const int w = nb[s];
+                        if (w >= 0 && w < t && !visited<GB>(bm, w)) simple = false;
+                    }
+                    if (!simple) {
+                        atomicMin(&h.tns, t);
+                    } else {
+                        done = true;
+#pragma unroll
+                        for (int s = 0; s < W; ++s) {
+                            const int w = nb[s];
+                            if (w > t && !visited<GB>(bm, w) && mark(bm, sm, w)) {
+                                if (w < i) {
+                                    nm = min(nm, w);
+                                } else {
+                                    ++a.ucnt;
+                                    a.lmax = max(a.lmax, w);
+                                }
+                            }
+                        }
+                    }
+                }
+                unsigned hm = __ballot_sync(kFull, valid && heavy);
+                while (hm) {
+                    const int src = __ffs(hm) - 1;
+                    hm &= hm - 1;
+                    const int tt = __shfl_sync(kFull, t, src);
+                    const int len = __shfl_sync(kFull, nb[1], src);
+                    const int64_t off = heavy_off(__shfl_sync(kFull, nb[2], src),
+                                                  __shfl_sync(kFull, nb[3], src));
+                    bool ok = true;
+                    for (int e = lane; e < len; e += 32) {
+                        const int w = __ldg(p.ci + off + e);
+                        if (w < tt && !visited<GB>(bm, w)) ok = false;
+                    }
+                    ok = __all_sync(kFull, ok);
+                    if (lane == 0) {
+                        a.te += len;
+                        ++a.sv;
+                    }
+                    if (lane == src) done = ok;
+                    if (!ok) {
+                        if (lane == 0) atomicMin(&h.tns, tt);
+                    } else {
+                        for (int e = lane; e < len; e += 32) {
+                            const int w = __ldg(p.ci + off + e);
+                            if (w > tt && !visited<GB>(bm, w) && mark(bm, sm, w)) {
+                                if (w < i) {
+                                    nm = min(nm, w);
+                                } else {
+                                    ++a.ucnt;
+                                    a.lmax = max(a.lmax, w);
+                                }
+                            }
+                        }
+                    }
+                }
+                if (valid) qB[k] = done ? 1 : 0;
+            }
+            if (nm != INT_MAX) atomicMin(&h.newmin, nm);
+            __syncthreads();
+            // m = smallest pending threshold now: a non-simple candidate (tns) or a vertex just
+            // marked by a simple one (newmin)
+            const int tns = h.tns, newmin = h.newmin;
+            const int m = min(tns, newmin);
+            const int last = qA[wc - 1];
+            const int nptr = m > last ? last : (m == tns ? m : m - 1);
+            // every visited bit in (ptr, nptr] is an L entry now (no BFS has marked below m yet):
+            // emit / count them in increasing order as the pointer passes (L122-143)
+            Lcnt += emit_range<NT, GB, MODE != kCount>(bm, sm, ptr + 1, nptr + 1, ldst, Lcnt, lcap,
+                                                       h.scan);
+            if (nptr < last) {  // simple candidates beyond the pointer are finished: mark them
+                for (int k = tid; k < wc; k += NT) {
+                    const int t = qA[k];
+                    if (t > nptr && qB[k]) atomicOr(dm + (t >> 5), 1u << (t & 31));
+                }
+                dused = true;
+            }
+            __syncthreads();
+            if (m <= last && m == tns) {  // smallest pending threshold: below-exploration
+                bfs<NT, W, GB>(p, h, bm, sm, qA, qB, gA, gB, i, m, a);
+                ++n_bfs;
+            }
+            cap = m <= last ? min(cap, kSmallWin) : min(2 * cap, p.wcap);
+            ptr = nptr;
+        }
+        // thresholds finished ahead of the pointer and never re-collected: the rest of (ptr, i)
+        Lcnt += emit_range<NT, GB, MODE != kCount>(bm, sm, ptr + 1, i, ldst, Lcnt, lcap, h.scan);
+        if (dused)  // leave the done map zero for the next row
+            for (int w = (h.minseed >> 5) + tid; w <= ((i - 1) >> 5); w += NT) dm[w] = 0;
+
+        // ---- U part, diagonal, count / emission
+        if (a.ucnt) atomicAdd(&h.ucnt, a.ucnt);
+        if (a.lmin < i) atomicMin(&h.lmin, a.lmin);
+        if (a.lmax > i) atomicMax(&h.lmax, a.lmax);
+        __syncthreads();
+        const int ucnt = h.ucnt, diag = h.diag, gmin = h.lmin, gmax = h.lmax;
+        const int len = Lcnt + diag + ucnt;
+        if constexpr (MODE == kCount) {
+            if (tid == 0) p.fill_count[i] = len;
+        } else if constexpr (MODE == kStage) {
+            // reserve len entries of the pool; rows that do not fit are re-traversed by emit
+            if (tid == 0) {
+                p.fill_count[i] = len;
+                const unsigned long long off = atomicAdd(p.pool_cursor, (unsigned long long)len);
+                const bool fits = off + (unsigned long long)len <= (unsigned long long)p.pool_cap;
+                h.stage_off = fits ? (long long)off : -1ll;
+                p.row_off[i] = fits ? (int64_t)off : -1;
+                if (!fits) p.unstaged[atomicAdd(p.unstaged_cnt, 1ull)] = i;
+            }
+            __syncthreads();
+            const long long off = h.stage_off;
+            if (off >= 0) {
+                int32_t *dst = p.pool + off;
+                for (int k = tid; k < Lcnt; k += NT) dst[k] = ldst[k];
+                if (diag && tid == 0) dst[Lcnt] = i;
+                emit_range<NT, GB, true>(bm, sm, i + 1, gmax + 1, dst + Lcnt + diag, 0, INT64_MAX,
+                                         h.scan);
+            }
+        } else {
+            if (lcap != (int64_t)len) {
+                if (tid == 0) atomicAdd(p.stats + kStatErr, 1ull);
+            } else {
+                if (diag && tid == 0) ldst[Lcnt] = i;
+                emit_range<NT, GB, true>(bm, sm, i + 1, gmax + 1, ldst + Lcnt + diag, 0, INT64_MAX,
+                                         h.scan);
+            }
+        }
+        if (p.row_prof) {
+            unsigned long long dsv = a.sv - sv_row;
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) dsv += __shfl_xor_sync(kFull, dsv, o);
+            if (lane == 0 && dsv) atomicAdd(reinterpret_cast<unsigned long long *>(p.row_prof) +
+                                                4 * (size_t)i + 1, dsv);
+            if (tid == 0) {
+                p.row_prof[4 * (size_t)i + 0] = clock64() - t_row;
+                p.row_prof[4 * (size_t)i + 2] = n_bfs;
+                p.row_prof[4 * (size_t)i + 3] = n_win;
+            }
+        }
+        // ---- clear the dirty word range (fill(:) = 0 for the next row, L115)
+        clear_words<NT>(bm, sm, gmin >> 5, gmax >> 5);
+        __syncthreads();
+    }
+
+    // flush statistics
+    unsigned long long te = a.te, sv = a.sv, sp = a.spills;
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+        te += __shfl_xor_sync(kFull, te, o);
+        sv += __shfl_xor_sync(kFull, sv, o);
+        sp += __shfl_xor_sync(kFull, sp, o);
+    }
+    if (lane == 0) {
+        atomicAdd(p.stats + kStatEdges, te);
+        atomicAdd(p.stats + kStatVerts, sv);
+        if (sp) atomicAdd(p.stats + kStatSpills, sp);
+    }
+}
+
+template <int NT, int W, int VIS>
+cudaError_t launch_w_vis(const Fill2Params &p, int mode, int grid, size_t smem, cudaStream_t s)
+{
+    if (mode == kCount)
+        fill2_kernel<NT, W, kCount, VIS><<<grid, NT, smem, s>>>(p);
+    else if (mode == kStage)
+        fill2_kernel<NT, W, kStage, VIS><<<grid, NT, smem, s>>>(p);
+    else
+        fill2_kernel<NT, W, kEmit, VIS><<<grid, NT, smem, s>>>(p);
+    return cudaGetLastError();
+}
+
+template <int NT, int W, int VIS>
+cudaError_t configure_w_vis(size_t smem)
+{
+    const void *fns[3] = {(const void *)fill2_kernel<NT, W, kCount, VIS>,
+                          (const void *)fill2_kernel<NT, W, kStage, VIS>,
+                          (const void *)fill2_kernel<NT, W, kEmit, VIS>};
+    for (const void *f : fns) {
+        cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)smem);
+        if (e != cudaSuccess) return e;
+        cudaFuncSetAttribute(f, cudaFuncAttributePreferredSharedMemoryCarveout, 100);
+    }
+    return cudaSuccess;
+}
+
+template <int NT, int W, int VIS>
+cudaError_t occupancy_w_vis(size_t smem, int *occ)
+{
+    const void *fns[3] = {(const void *)fill2_kernel<NT, W, kCount, VIS>,
+                          (const void *)fill2_kernel<NT, W, kStage, VIS>,
+                          (const void *)fill2_kernel<NT, W, kEmit, VIS>};
+    int best = 1 << 30;
+    for (const void *f : fns) {
+        int o = 0;
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, f, NT, smem);
+        if (e != cudaSuccess) return e;
+        best = o < best ? o : best;
+    }
+    *occ = best;
+    return cudaSuccess;
+}
+
+template <int NT, template <int, int, int> class Op, class... Args>
+cudaError_t dispatch_w_vis(int w, int vis, Args... args)
+{
+    if (w == 4 && vis == kVisSmem) return Op<NT, 4, kVisSmem>::run(args...);
+    if (w == 4 && vis == kVisGlobal) return Op<NT, 4, kVisGlobal>::run(args...);
+    if (w == 8 && vis == kVisSmem) return Op<NT, 8, kVisSmem>::run(args...);
+    if (w == 8 && vis == kVisGlobal) return Op<NT, 8, kVisGlobal>::run(args...);
+    return cudaErrorInvalidValue;
+}
+
+template <int NT, int W, int VIS>
+struct LaunchOp {
+    static cudaError_t run(const Fill2Params *p, int mode, int grid, size_t smem, cudaStream_t s)
+    {
+        return launch_w_vis<NT, W, VIS>(*p, mode, grid, smem, s);
+    }
+};
+template <int NT, int W, int VIS>
+struct ConfigOp {
+    static cudaError_t run(size_t smem) { return configure_w_vis<NT, W, VIS>(smem); }
+};
+template <int NT, int W, int VIS>
+struct OccOp {
+    static cudaError_t run(size_t smem, int *occ) { return occupancy_w_vis<NT, W, VIS>(smem, occ); }
+};
+
+}  // namespace f2
+
+// Explicit per-NT entry points (one translation unit per CTA size: fill2_nt<NT>.cu).
+#define LUSYM_F2_INSTANTIATE(NTV)                                                            \
+    template <>                                                                              \
+    cudaError_t fill2_launch_nt<NTV>(const Fill2Params &p, int w, int mode, int vis,         \
+                                     int grid, size_t smem, cudaStream_t s)                  \
+    {                                                                                        \
+        return f2::dispatch_w_vis<NTV, f2::LaunchOp>(w, vis, &p, mode, grid, smem, s);       \
+    }                                                                                        \
+    template <>                                                                              \
+    cudaError_t fill2_configure_nt<NTV>(int w, int vis, size_t smem)                         \
+    {                                                                                        \
+        return f2::dispatch_w_vis<NTV, f2::ConfigOp>(w, vis, smem);                          \
+    }                                                                                        \
+    template <>                                                                              \
+    cudaError_t fill2_occupancy_nt<NTV>(int w, int vis, size_t smem, int *occ)               \
+    {                                                                                        \
+        return f2::dispatch_w_vis<NTV, f2::OccOp>(w, vis, smem, occ);                        \
+    }
+
+}  // namespace lusym

@@ -26,10 +26,12 @@ struct Fill2Params {
     const int64_t *rp_lu;     // emit pass
     int32_t *ci_lu;
     uint32_t *gbitmap;        // visited bitmaps in HBM (one slot per CTA) or null
+    uint32_t *dbitmap;        // "threshold done" bitmaps in HBM (one slot per CTA)
     int64_t gbitmap_stride;   // words per slot
     int32_t *gspill;          // frontier spill, 2 x spill_cap per CTA
     int64_t spill_cap;
-    int32_t nw;               // bitmap words = ceil((n+1)/32)
+    int32_t nw;               // visited bitmap words = ceil(n/32)
+    int32_t sw;               // summary words = ceil(nw/32) (shared memory)
     int32_t q;                // shared frontier capacity per buffer (entries)
     int32_t wcap;             // window capacity (<= q); 1 = one threshold at a time
     unsigned long long *row_counter;
@@ -45,15 +47,29 @@ struct Fill2Params {
     unsigned long long *pool_cursor;
     int32_t *unstaged;
     unsigned long long *unstaged_cnt;
+    // optional per-row profile (4 x int64 per row: cycles, vertices scanned, BFS runs, windows)
+    int64_t *row_prof;
 };
 enum Fill2Mode { kCount = 0, kEmit = 1, kStage = 2 };
 
-// fill2_kernels.cu
-size_t fill2_smem_bytes(int n, int q, bool global_bitmap);
-cudaError_t fill2_configure(int nt, int w, bool gb, size_t smem);
-cudaError_t fill2_occupancy(int nt, int w, bool gb, size_t smem, int *occ);
-cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, int mode, bool gb, int grid,
+// Visited storage of a row in flight (frontiers are lists in shared memory, spilling to HBM).
+//   kVisSmem   : visited bitmap in shared memory
+//   kVisGlobal : visited bitmap in an HBM slot per CTA (n too large for shared memory)
+enum Fill2Vis { kVisSmem = 0, kVisGlobal = 1 };
+
+// fill2_kernels.cu (host dispatch; kernels instantiated in fill2_nt*.cu)
+size_t fill2_smem_bytes(int n, int q, int vis);
+cudaError_t fill2_configure(int nt, int w, int vis, size_t smem);
+cudaError_t fill2_occupancy(int nt, int w, int vis, size_t smem, int *occ);
+cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, int mode, int vis, int grid,
                          size_t smem, cudaStream_t s);
+template <int NT>
+cudaError_t fill2_launch_nt(const Fill2Params &p, int w, int mode, int vis, int grid, size_t smem,
+                            cudaStream_t s);
+template <int NT>
+cudaError_t fill2_configure_nt(int w, int vis, size_t smem);
+template <int NT>
+cudaError_t fill2_occupancy_nt(int w, int vis, size_t smem, int *occ);
 
 // prep_kernels.cu
 cudaError_t validate_csr(int32_t n, int64_t nnz, const int64_t *rp, const int32_t *ci,

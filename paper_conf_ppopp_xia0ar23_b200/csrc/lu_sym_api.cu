@@ -51,9 +51,11 @@ struct lu_sym {
     int w = 8;
     // plan
     bool gb = false;
+    int vis = kVisSmem;
     int nt = 256, q = 2048, grid = 0;
     size_t smem = 0;
     uint32_t *gbitmap = nullptr;
+    uint32_t *dbitmap = nullptr;
     int64_t gb_stride = 0;
     int32_t *gspill = nullptr;
     int64_t spill_cap = 0;
@@ -79,6 +81,7 @@ struct lu_sym {
     bool ev_used[kEvN] = {};
     int64_t scratch_bytes = 0;
     int64_t launches = 0;
+    int64_t *row_prof = nullptr;  // borrowed, set by lu_sym_set_row_profile
 };
 
 namespace {
@@ -109,6 +112,7 @@ void free_handle(lu_sym *h)
 {
     cudaFree(h->ell);
     cudaFree(h->gbitmap);
+    cudaFree(h->dbitmap);
     cudaFree(h->gspill);
     cudaFree(h->dstats);
     cudaFree(h->scan_blk);
@@ -146,9 +150,16 @@ lu_status plan(lu_sym *h)
     const int n = h->n;
     h->q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : 2048;
     if (h->q < 32) h->q = 32;
-    size_t smem = fill2_smem_bytes(n, h->q, false);
-    h->gb = (h->opts.flags & LU_F_GLOBAL_BITMAP) || smem > (size_t)smem_optin;
-    if (h->gb) smem = fill2_smem_bytes(n, h->q, true);
+    // visited bitmap in shared memory when it fits next to the queues, else HBM slots
+    const size_t smem_list = fill2_smem_bytes(n, h->q, kVisSmem);
+    if (h->opts.flags & LU_F_GLOBAL_BITMAP)
+        h->vis = kVisGlobal;
+    else if (smem_list <= (size_t)smem_optin)
+        h->vis = kVisSmem;
+    else
+        h->vis = kVisGlobal;
+    h->gb = h->vis == kVisGlobal;
+    size_t smem = fill2_smem_bytes(n, h->q, h->vis);
     if (smem > (size_t)smem_optin)
         return fail(LU_ERR_NOMEM, "queue_capacity %d needs %zu B of shared memory (> %d)", h->q,
                     smem, smem_optin);
@@ -166,10 +177,10 @@ lu_status plan(lu_sym *h)
         return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512 or 1024 (got %d)", nt);
     h->nt = nt;
     h->smem = smem;
-    CK(fill2_configure(nt, h->w, h->gb, smem));
+    CK(fill2_configure(nt, h->w, h->vis, smem));
     // resident CTAs of the actual kernel (registers may limit below the smem estimate)
     int occ = 0;
-    CK(fill2_occupancy(nt, h->w, h->gb, smem, &occ));
+    CK(fill2_occupancy(nt, h->w, h->vis, smem, &occ));
     if (occ < 1) return fail(LU_ERR_NOMEM, "fill2 kernel cannot be resident (smem %zu B)", smem);
     int64_t grid = (int64_t)sms * occ;
     if (h->opts.rows_in_flight > 0 && h->opts.rows_in_flight < grid) grid = h->opts.rows_in_flight;
@@ -184,7 +195,7 @@ lu_status plan(lu_sym *h)
     h->staging = !(h->opts.flags & LU_F_TWO_PASS);
     h->budget = budget;
     const uint64_t per_row = (uint64_t)(h->staging ? 3 : 2) * h->spill_cap * 4 +
-                             (h->gb ? (uint64_t)h->gb_stride * 4 : 0);
+                             (uint64_t)(h->gb ? 2 : 1) * h->gb_stride * 4;
     const uint64_t fit = budget / per_row;
     if (fit < 1)
         return fail(LU_ERR_NOMEM, "scratch budget %llu B < one row's scratch %llu B",
@@ -198,6 +209,7 @@ lu_status plan(lu_sym *h)
         st = dalloc(h, &h->gbitmap, (size_t)h->gb_stride * h->grid);
         if (st != LU_OK) return st;
     }
+    if ((st = dalloc(h, &h->dbitmap, (size_t)h->gb_stride * h->grid)) != LU_OK) return st;
     if ((st = dalloc(h, &h->unstaged, (size_t)n)) != LU_OK) return st;
     if (h->staging) {
         if ((st = dalloc(h, &h->stg, (size_t)h->spill_cap * h->grid)) != LU_OK) return st;
@@ -231,6 +243,7 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     CK(cudaMemsetAsync(st, 0, sizeof(unsigned long long) * kStatCount, s));
     if (h->gb)
         CK(cudaMemsetAsync(h->gbitmap, 0, sizeof(uint32_t) * (size_t)h->gb_stride * h->grid, s));
+    CK(cudaMemsetAsync(h->dbitmap, 0, sizeof(uint32_t) * (size_t)h->gb_stride * h->grid, s));
     Fill2Params p;
     p.n = h->n;
     p.rp = h->rp;
@@ -243,10 +256,12 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     p.rp_lu = rp_lu;
     p.ci_lu = ci_lu;
     p.gbitmap = h->gbitmap;
+    p.dbitmap = h->dbitmap;
     p.gbitmap_stride = h->gb_stride;
     p.gspill = h->gspill;
     p.spill_cap = h->spill_cap;
     p.nw = (int32_t)(((int64_t)h->n + 31) / 32);
+    p.sw = (p.nw + 31) / 32;
     p.q = h->q;
     p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : h->q;
     p.row_counter = h->dstats;
@@ -260,11 +275,14 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     p.pool_cursor = h->dstats + kSlotPoolCursor;
     p.unstaged = h->unstaged;
     p.unstaged_cnt = h->dstats + kSlotUnstaged;
+    p.row_prof = h->row_prof;
+    if (h->row_prof && mode != kEmit)
+        CK(cudaMemsetAsync(h->row_prof + 4 * (size_t)rb, 0, sizeof(int64_t) * 4 * (size_t)(re - rb), s));
     int rows = row_list ? list_len : re - rb;
     int grid = h->grid;
     if (grid > rows) grid = rows;
     if (grid < 1) return LU_OK;
-    CK(fill2_launch(p, h->nt, h->w, mode, h->gb, grid, h->smem, s));
+    CK(fill2_launch(p, h->nt, h->w, mode, h->vis, grid, h->smem, s));
     h->launches += 1;
     return LU_OK;
 }
@@ -625,6 +643,14 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
     h->stats.kernel_launches = h->launches;
     h->stats.pool_bytes = h->pool ? h->pool_cap * (int64_t)sizeof(int32_t) : 0;
     *out = h->stats;
+    return LU_OK;
+}
+
+lu_status lu_sym_set_row_profile(lu_sym *h, int64_t *d_prof)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    h->row_prof = d_prof;
     return LU_OK;
 }
 

@@ -142,6 +142,7 @@ KNOBS = [
     dict(flags=lu.F_NO_PRUNE), dict(flags=lu.F_KAHN_WIDE_ONLY), dict(flags=lu.F_NO_CONTRACT),
     dict(flags=lu.F_NO_CONTRACT | lu.F_NO_PRUNE | lu.F_KAHN_WIDE_ONLY),
     dict(flags=lu.F_TWO_PASS),                       # Alg. 3 as printed: emit re-traverses
+    dict(flags=lu.F_TWO_PASS, queue_capacity=64),
     dict(pool_bytes=4096),                           # pool overflow: most rows re-traversed
     dict(pool_bytes=200_000),                        # partial staging
 ]
