@@ -167,8 +167,10 @@ def cpu_levels_time(rp, ci, rule, nnz_hint=None):
 
 
 def auto_stride(n, te_total):
-    # ~2e9 TE visited by the sample (both passes) is ~10-20 s on 8 host cores
-    target = 1.0e9
+    """Row stride of the oracle sample: about 10-30 s of CPU work on the box's host cores.
+    The oracle visits ~6e8 TE/s per core over its two passes (count + emit)."""
+    cores = os.cpu_count() or 1
+    target = 6e8 * cores * 15.0 / 2
     return max(1, int(round(te_total / target)))
 
 
@@ -287,10 +289,15 @@ def run_ours(args, rank, world, local_rank):
     rows_mine = re_ - rb
     frac_rows = cost[rb:re_].sum() / max(cost.sum(), 1)
     te_mine, sv_mine = te * frac_rows, sv * frac_rows
-    b_count = alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, False)
-    b_emit = alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, True)
+    # the count pass runs the traversal and stages every row (staged mode), so its algorithmic
+    # bytes are the traversal's plus the pattern it writes; emit is then a placement copy
+    staged = stats["pool_bytes"] > 0
+    b_count = alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, staged)
+    b_emit = (8.0 * nnz * frac_rows + 8 * rows_mine) if staged else \
+        alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, True)
     dom = "emit" if avg["emit"] >= avg["count"] else "count"
     b_dom = b_emit if dom == "emit" else b_count
+    kname = {"count": "stage" if staged else "count", "emit": "place" if staged else "emit"}[dom]
     peaks = {}
     try:
         peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
@@ -301,12 +308,13 @@ def run_ours(args, rank, world, local_rank):
     traffic = None
     try:
         prof = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        traffic = prof.get(f"cfg{args.config}", {}).get(f"fill2_{dom}")
+        traffic = prof.get(f"cfg{args.config}", {}).get(
+            f"fill2_{kname}" if kname in ("stage", "count", "emit") else "k_place")
     except Exception:
         pass
     roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                 "frac": achieved / peak, "traffic": traffic,
-                "kernel": f"fill2_kernel<{dom}>",
+                "kernel": f"fill2_kernel<{kname}>" if kname != "place" else "k_place",
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback",
                 "alg_bytes_per_launch": b_dom, "ms_per_launch": avg[dom]}
 
