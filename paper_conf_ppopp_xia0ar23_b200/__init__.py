@@ -31,7 +31,8 @@ __all__ = ["Symbolic", "LuSymError", "levelize", "load_library", "library_path",
            "row_cost_upper_bound", "DEP_U", "DEP_GLU3"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-_LIBPATH = os.path.join(_HERE, "lib", "liblusym.so")
+# LUSYM_LIB selects an alternative build of the same library (kernel-variant experiments)
+_LIBPATH = os.environ.get("LUSYM_LIB") or os.path.join(_HERE, "lib", "liblusym.so")
 
 LU_OK, LU_ERR_ARG, LU_ERR_INPUT, LU_ERR_NOMEM, LU_ERR_CAPACITY = 0, 1, 2, 3, 4
 LU_ERR_CUDA, LU_ERR_STATE, LU_ERR_INTERNAL = 5, 7, 8

@@ -30,6 +30,19 @@
 namespace lusym {
 namespace f2 {
 
+#ifndef LUSYM_LAYOUT_CONST
+#define LUSYM_LAYOUT_CONST 1
+#endif
+#ifndef LUSYM_SWZ
+#define LUSYM_SWZ 1
+#endif
+#ifndef LUSYM_SHPTX
+#define LUSYM_SHPTX 0
+#endif
+#ifndef LUSYM_THREADS_PER_SM  // register budget: 65536 / this
+#define LUSYM_THREADS_PER_SM 2048
+#endif
+
 constexpr unsigned kFull = 0xffffffffu;
 constexpr int kSmallWin = 32;  // threshold window after a window was cut short
 
@@ -71,11 +84,21 @@ __device__ __forceinline__ int block_scan_excl(int x, int *s, int &total)
     return r;
 }
 
+// Shared-memory bitmaps are stored with the word index XOR-swizzled inside each group of 32
+// words, so that words 32 (or a multiple of 32) apart — grid neighbours at +-k for k a
+// multiple of 1024 — fall into different banks.
+template <bool GB>
+__device__ __forceinline__ int phys(int w)
+{
+    if (GB || !LUSYM_SWZ) return w;
+    return w ^ ((w >> 5) & 31);
+}
+
 template <bool GB>
 __device__ __forceinline__ uint32_t bm_word(const uint32_t *bm, int w)
 {
     if (GB) return __ldcg(bm + w);
-    return bm[w];
+    return bm[phys<GB>(w)];
 }
 
 template <bool GB>
@@ -86,10 +109,11 @@ __device__ __forceinline__ bool visited(const uint32_t *bm, int v)
 
 // test-and-set (reading R26): true iff this call set the bit.  The level-1 summary sm gets bit
 // w when visited word w first becomes non-zero, so scans and clears skip empty stretches.
+template <bool GB>
 __device__ __forceinline__ bool mark(uint32_t *bm, uint32_t *sm, int v)
 {
     const uint32_t b = 1u << (v & 31);
-    const uint32_t old = atomicOr(bm + (v >> 5), b);
+    const uint32_t old = atomicOr(bm + phys<GB>(v >> 5), b);
     if (old == 0) atomicOr(sm + (v >> 10), 1u << ((v >> 5) & 31));
     return !(old & b);
 }
@@ -107,6 +131,34 @@ __device__ __forceinline__ void load_nb(const int32_t *ell, int f, int (&nb)[W])
         const int4 a = __ldg(reinterpret_cast<const int4 *>(ell + (size_t)f * W));
         nb[0] = a.x; nb[1] = a.y; nb[2] = a.z; nb[3] = a.w;
     }
+}
+
+// Shared-memory bitmap access through 32-bit shared-window addresses (computed once per BFS
+// level), so the hot neighbour test is LDS + shift + test without re-deriving the CTA's shared
+// base for every neighbour.
+__device__ __forceinline__ uint32_t lds_u32(uint32_t addr)
+{
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
+    return v;
+}
+
+__device__ __forceinline__ uint32_t atoms_or(uint32_t addr, uint32_t b)
+{
+    uint32_t old;
+    asm volatile("atom.shared.or.b32 %0, [%1], %2;" : "=r"(old) : "r"(addr), "r"(b) : "memory");
+    return old;
+}
+
+// test-and-set of v in a shared bitmap at window address bmw (summary at smw); see mark()
+__device__ __forceinline__ bool visit_s(uint32_t bmw, uint32_t smw, int v)
+{
+    const uint32_t wa = bmw + 4u * (uint32_t)phys<false>(v >> 5);
+    const uint32_t b = 1u << (v & 31);
+    if (lds_u32(wa) & b) return false;
+    const uint32_t old = atoms_or(wa, b);
+    if (old == 0) atoms_or(smw + 4u * (uint32_t)(v >> 10), 1u << ((v >> 5) & 31));
+    return !(old & b);
 }
 
 __device__ __forceinline__ int64_t heavy_off(int lo, int hi)
@@ -222,15 +274,15 @@ __device__ __forceinline__ int emit_range(const uint32_t *bm, const uint32_t *sm
 }
 
 // Zero the visited words [wlo, whi] and their summary bits (walk the summary if wide).
-template <int NT>
+template <int NT, bool GB>
 __device__ void clear_words(uint32_t *bm, uint32_t *sm, int wlo, int whi)
 {
     if (whi < wlo) return;
     if (whi - wlo < 4 * NT) {
-        for (int w = wlo + (int)threadIdx.x; w <= whi; w += NT) bm[w] = 0;
+        for (int w = wlo + (int)threadIdx.x; w <= whi; w += NT) bm[phys<GB>(w)] = 0;
     } else {
         for (int sidx = (wlo >> 5) + (int)threadIdx.x; sidx <= (whi >> 5); sidx += NT)
-            for (uint32_t t = sm[sidx]; t; t &= t - 1) bm[(sidx << 5) + __ffs(t) - 1] = 0;
+            for (uint32_t t = sm[sidx]; t; t &= t - 1) bm[phys<GB>((sidx << 5) + __ffs(t) - 1)] = 0;
     }
     __syncthreads();
     for (int sidx = (wlo >> 5) + (int)threadIdx.x; sidx <= (whi >> 5); sidx += NT) sm[sidx] = 0;
@@ -252,6 +304,10 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, u
                                            RowAcc &a)
 {
     const int tid = threadIdx.x, lane = tid & 31;
+#if LUSYM_SHPTX
+    const uint32_t bmw = GB ? 0u : (uint32_t)__cvta_generic_to_shared(bm);
+    const uint32_t smw = (uint32_t)__cvta_generic_to_shared(sm);
+#endif
     for (int base = 0; base < cnt; base += NT) {
         const int k = base + tid;
         const bool valid = k < cnt;
@@ -270,7 +326,16 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, u
 #pragma unroll
             for (int s = 0; s < W; ++s) {
                 const int w = nb[s];
-                if (w >= 0 && !visited<GB>(bm, w) && mark(bm, sm, w)) {
+#if LUSYM_SHPTX
+                bool nw;
+                if constexpr (GB)
+                    nw = w >= 0 && !visited<GB>(bm, w) && mark<GB>(bm, sm, w);
+                else
+                    nw = w >= 0 && visit_s(bmw, smw, w);
+                if (nw) {
+#else
+                if (w >= 0 && !visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
+#endif
                     if (w < t0) {
                         frm |= 1u << s;
                     } else if (w > i) {
@@ -329,7 +394,7 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, u
                 int w = -1;
                 if (e < len) {
                     w = __ldg(p.ci + off + e);
-                    if (!visited<GB>(bm, w) && mark(bm, sm, w)) {
+                    if (!visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
                         if (w < t0) {
                             fr = true;
                             nmin = min(nmin, w);
@@ -376,19 +441,35 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, uint32_t *bm, uint32_t *sm, in
 // MODE: kCount (symbolic_1, counts only), kStage (counts + rows staged into the HBM pool, so
 // symbolic_2 becomes a placement copy), kEmit (symbolic_2 by traversal, into the final CSR).
 template <int NT, int W, int MODE, int VIS>
-__global__ void __launch_bounds__(NT, 2048 / NT) fill2_kernel(const Fill2Params p)
+__global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(const Fill2Params p)
 {
     constexpr bool GB = VIS == kVisGlobal;
     extern __shared__ __align__(16) unsigned char smem[];
     Hdr &h = *reinterpret_cast<Hdr *>(smem);
-    int32_t *qA = reinterpret_cast<int32_t *>(smem + kHdrBytes);
-    int32_t *qB = qA + p.q;
-    uint32_t *sm = reinterpret_cast<uint32_t *>(qB + p.q);  // summary (p.sw words)
+    // shared layout: header | visited bitmap (at a constant offset, so the hot bit tests need
+    // no address arithmetic beyond the word index) | summary | two frontier queues
     uint32_t *bm;
+    uint32_t *sm;
+    int32_t *qA, *qB;
+#if LUSYM_LAYOUT_CONST
+    if constexpr (GB) {
+        bm = p.gbitmap + (size_t)blockIdx.x * p.gbitmap_stride;
+        sm = reinterpret_cast<uint32_t *>(smem + kHdrBytes);
+    } else {
+        bm = reinterpret_cast<uint32_t *>(smem + kHdrBytes);
+        sm = bm + p.nw;
+    }
+    qA = reinterpret_cast<int32_t *>(sm + p.sw);
+    qB = qA + p.q;
+#else
+    qA = reinterpret_cast<int32_t *>(smem + kHdrBytes);
+    qB = qA + p.q;
+    sm = reinterpret_cast<uint32_t *>(qB + p.q);
     if constexpr (GB)
         bm = p.gbitmap + (size_t)blockIdx.x * p.gbitmap_stride;
     else
         bm = sm + p.sw;
+#endif
     int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
     int32_t *gB = gA + p.spill_cap;
     const int tid = threadIdx.x, lane = tid & 31;
@@ -430,7 +511,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) fill2_kernel(const Fill2Params 
         for (int64_t k = rb + tid; k < re; k += NT) {
             const int v = __ldg(p.ci + k);
             ++a.te;
-            mark(bm, sm, v);
+            mark<GB>(bm, sm, v);
             if (v < i) {
                 atomicMin(&h.minseed, v);
                 a.lmin = min(a.lmin, v);
@@ -441,7 +522,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) fill2_kernel(const Fill2Params 
                 h.diag = 1;
             }
         }
-        if (tid == 0) mark(bm, sm, i);
+        if (tid == 0) mark<GB>(bm, sm, i);
         __syncthreads();
 
         int ptr = h.minseed - 1;  // every unprocessed threshold is > ptr
@@ -502,7 +583,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) fill2_kernel(const Fill2Params 
 #pragma unroll
                         for (int s = 0; s < W; ++s) {
                             const int w = nb[s];
-                            if (w > t && !visited<GB>(bm, w) && mark(bm, sm, w)) {
+                            if (w > t && !visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
                                 if (w < i) {
                                     nm = min(nm, w);
                                 } else {
@@ -537,7 +618,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) fill2_kernel(const Fill2Params 
                     } else {
                         for (int e = lane; e < len; e += 32) {
                             const int w = __ldg(p.ci + off + e);
-                            if (w > tt && !visited<GB>(bm, w) && mark(bm, sm, w)) {
+                            if (w > tt && !visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
                                 if (w < i) {
                                     nm = min(nm, w);
                                 } else {
@@ -632,7 +713,7 @@ __global__ void __launch_bounds__(NT, 2048 / NT) fill2_kernel(const Fill2Params 
             }
         }
         // ---- clear the dirty word range (fill(:) = 0 for the next row, L115)
-        clear_words<NT>(bm, sm, gmin >> 5, gmax >> 5);
+        clear_words<NT, GB>(bm, sm, gmin >> 5, gmax >> 5);
         __syncthreads();
     }
 

@@ -6,10 +6,11 @@ namespace lusym {
 
 size_t fill2_smem_bytes(int n, int q, int vis)
 {
+    // header | visited bitmap (kVisSmem) | level-1 summary | two frontier queues
     size_t b = kHdrBytes + 2 * (size_t)q * sizeof(int32_t);
     const size_t words = (size_t)((n + 31) / 32);
-    b += (words + 31) / 32 * sizeof(uint32_t);  // level-1 summary
-    if (vis == kVisSmem) b += words * sizeof(uint32_t);
+    b += (words + 31) / 32 * sizeof(uint32_t);
+    if (vis == kVisSmem) b += (words + 31) / 32 * 32 * sizeof(uint32_t);  // whole swizzle groups
     return (b + 15) & ~(size_t)15;
 }
 

@@ -148,40 +148,59 @@ lu_status plan(lu_sym *h)
     CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->device));
     CK(cudaDeviceGetAttribute(&smem_res, cudaDevAttrReservedSharedMemoryPerBlock, h->device));
     const int n = h->n;
-    h->q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : 2048;
-    if (h->q < 32) h->q = 32;
-    // visited bitmap in shared memory when it fits next to the queues, else HBM slots
-    const size_t smem_list = fill2_smem_bytes(n, h->q, kVisSmem);
+    // visited bitmap in shared memory when it fits next to minimal queues, else HBM slots
     if (h->opts.flags & LU_F_GLOBAL_BITMAP)
         h->vis = kVisGlobal;
-    else if (smem_list <= (size_t)smem_optin)
+    else if (fill2_smem_bytes(n, h->opts.queue_capacity > 0 ? h->opts.queue_capacity : 256,
+                              kVisSmem) <= (size_t)smem_optin)
         h->vis = kVisSmem;
     else
         h->vis = kVisGlobal;
     h->gb = h->vis == kVisGlobal;
-    size_t smem = fill2_smem_bytes(n, h->q, h->vis);
-    if (smem > (size_t)smem_optin)
-        return fail(LU_ERR_NOMEM, "queue_capacity %d needs %zu B of shared memory (> %d)", h->q,
-                    smem, smem_optin);
-    int ctas = (int)(smem_sm / (smem + smem_res));
-    if (ctas < 1) ctas = 1;
-    if (ctas > 16) ctas = 16;
-    int nt = h->opts.threads_per_row;
-    if (nt <= 0) {
-        nt = pow2_floor(2048 / ctas);
-        if (nt < 128) nt = 128;
-        if (nt > 1024) nt = 1024;
-        if (n < 65536 && nt > 256) nt = 256;
+    // CTA size and shared queue capacity: the traversal is latency-bound, so maximise resident
+    // threads first, then rows in flight (CTAs), then queue capacity (fewer spills).
+    // Frontier levels larger than the queue spill to the CTA's HBM region.
+    const int nts[4] = {128, 256, 512, 1024};
+    const int qs[4] = {512, 1024, 2048, 4096};
+    int best_nt = 0, best_q = 0, best_occ = 0;
+    long best_key = -1;
+    for (int a = 0; a < 4; ++a) {
+        const int nt = nts[a];
+        if (h->opts.threads_per_row > 0 && nt != h->opts.threads_per_row) continue;
+        for (int b = 0; b < 4; ++b) {
+            const int q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : qs[b];
+            if (h->opts.queue_capacity > 0 && b > 0) break;
+            const size_t smem = fill2_smem_bytes(n, q < 32 ? 32 : q, h->vis);
+            if (smem > (size_t)smem_optin) continue;
+            CK(fill2_configure(nt, h->w, h->vis, smem));
+            int occ = 0;
+            CK(fill2_occupancy(nt, h->w, h->vis, smem, &occ));
+            if (occ < 1) continue;
+            // small matrices: rows are short, prefer small CTAs; large rows want big levels
+            const long key = ((long)occ * nt << 24) | ((long)occ << 14) | q;
+            if (key > best_key) {
+                best_key = key;
+                best_nt = nt;
+                best_q = q < 32 ? 32 : q;
+                best_occ = occ;
+            }
+        }
     }
-    if (nt != 128 && nt != 256 && nt != 512 && nt != 1024)
-        return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512 or 1024 (got %d)", nt);
-    h->nt = nt;
-    h->smem = smem;
-    CK(fill2_configure(nt, h->w, h->vis, smem));
-    // resident CTAs of the actual kernel (registers may limit below the smem estimate)
-    int occ = 0;
-    CK(fill2_occupancy(nt, h->w, h->vis, smem, &occ));
-    if (occ < 1) return fail(LU_ERR_NOMEM, "fill2 kernel cannot be resident (smem %zu B)", smem);
+    if (best_key < 0) {
+        if (h->opts.threads_per_row > 0 && h->opts.threads_per_row != 128 &&
+            h->opts.threads_per_row != 256 && h->opts.threads_per_row != 512 &&
+            h->opts.threads_per_row != 1024)
+            return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512 or 1024 (got %d)",
+                        h->opts.threads_per_row);
+        return fail(LU_ERR_NOMEM, "no resident fill2 configuration (queue_capacity %d)",
+                    h->opts.queue_capacity);
+    }
+    h->nt = best_nt;
+    h->q = best_q;
+    h->smem = fill2_smem_bytes(n, h->q, h->vis);
+    const int occ = best_occ;
+    (void)smem_res;
+    (void)pow2_floor;
     int64_t grid = (int64_t)sms * occ;
     if (h->opts.rows_in_flight > 0 && h->opts.rows_in_flight < grid) grid = h->opts.rows_in_flight;
     // HBM budget
@@ -260,7 +279,7 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     p.gbitmap_stride = h->gb_stride;
     p.gspill = h->gspill;
     p.spill_cap = h->spill_cap;
-    p.nw = (int32_t)(((int64_t)h->n + 31) / 32);
+    p.nw = (int32_t)((((int64_t)h->n + 31) / 32 + 31) / 32 * 32);  // whole swizzle groups
     p.sw = (p.nw + 31) / 32;
     p.q = h->q;
     p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : h->q;
