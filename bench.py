@@ -327,24 +327,38 @@ def run_ours(args, rank, world, local_rank):
         out_ci = torch.empty(nnz, dtype=torch.int32).pin_memory()
         out_lv = torch.empty(n, dtype=torch.int32).pin_memory()
         e_ms = []
+        e_phase = {}
         for k in range(args.e2e_steps + 1):
             barrier()
             torch.cuda.synchronize()
             a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            marks = []
+
+            def mark(tag):
+                ev_ = torch.cuda.Event(enable_timing=True)
+                ev_.record(stream)
+                marks.append((tag, ev_))
+
             a.record(stream)
             rpd = rp_h.to(dev, non_blocking=True)
             cid = ci_h.to(dev, non_blocking=True)
+            mark("h2d")
             he = lu.Symbolic(rpd, cid, **sym_opts)             # S1 + S2 (validate, plan)
+            mark("create")
             fc = torch.zeros(n, dtype=torch.int32, device=dev)
             he.count(rb, re_, fc)
             if world > 1:
                 lu.assemble_counts(fc)
+            mark("count")
             rp_lu, nz = he.scan(fc)
             ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)
+            mark("scan+alloc")
             he.emit(rp_lu, ci_lu, rb, re_)
             if world > 1:
                 lu.assemble_pattern(ci_lu, rp_lu, bounds)
+            mark("emit")
             level, _ = he.levelize(rp_lu, ci_lu, args.rule)
+            mark("levelize")
             if rank == 0:
                 out_rp.copy_(rp_lu, non_blocking=True)
                 out_ci.copy_(ci_lu, non_blocking=True)
@@ -354,6 +368,10 @@ def run_ours(args, rank, world, local_rank):
             he.close()
             if k > 0:
                 e_ms.append(a.elapsed_time(b))
+                prev = a
+                for tag, ev_ in marks + [("d2h", b)]:
+                    e_phase.setdefault(tag, []).append(prev.elapsed_time(ev_))
+                    prev = ev_
         t = torch.tensor([float(np.mean(e_ms))], dtype=torch.float64, device=dev)
         if world > 1:
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -361,6 +379,7 @@ def run_ours(args, rank, world, local_rank):
                "h2d_bytes_per_step": int(rp_np.nbytes + ci_np.nbytes),
                "d2h_bytes_per_step": int((n + 1) * 8 + nnz * 4 + n * 4) if rank == 0 else 0,
                "ms_per_step": float(t.item()),
+               "phases_ms": {k: float(np.mean(v)) for k, v in e_phase.items()},
                "includes": "H2D of A, create (validate+adjacency+plan), count, scan, alloc, "
                            "emit, levelize, D2H of row_ptr/col_idx/level"}
 

@@ -57,6 +57,12 @@ enum Fill2Mode { kCount = 0, kEmit = 1, kStage = 2 };
 //   kVisGlobal : visited bitmap in an HBM slot per CTA (n too large for shared memory)
 enum Fill2Vis { kVisSmem = 0, kVisGlobal = 1 };
 
+// Stream-ordered device allocations from the current device's default memory pool, whose
+// release threshold is raised once so that memory freed by one handle stays reserved for the
+// next (creating and destroying handles then costs no cudaMalloc/cudaFree).  lu_sym_api.cu.
+cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s);
+void dev_free(void *p, cudaStream_t s);
+
 // fill2_kernels.cu (host dispatch; kernels instantiated in fill2_nt*.cu)
 size_t fill2_smem_bytes(int n, int q, int vis);
 cudaError_t fill2_configure(int nt, int w, int vis, size_t smem);
@@ -112,6 +118,6 @@ struct LevelizeInfo {
 cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, int rule,
                          bool prune, bool contract, bool wide_only, LevelizeScratch &scr,
                          int32_t *level, LevelizeInfo *info, cudaStream_t s, const char **err);
-void levelize_free(LevelizeScratch &scr);
+void levelize_free(LevelizeScratch &scr, cudaStream_t s);
 
 }  // namespace lusym

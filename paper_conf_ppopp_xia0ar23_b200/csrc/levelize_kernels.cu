@@ -397,11 +397,11 @@ int aux_grid(int64_t warps)
 
 }  // namespace
 
-void levelize_free(LevelizeScratch &s)
+void levelize_free(LevelizeScratch &s, cudaStream_t st)
 {
-    cudaFree(s.ustart); cudaFree(s.uend); cudaFree(s.indeg); cudaFree(s.queue);
-    cudaFree(s.lt_ptr); cudaFree(s.lt_idx); cudaFree(s.lt_fill); cudaFree(s.scan_blk);
-    cudaFree(s.ctrl); cudaFree(s.chain);
+    dev_free(s.ustart, st); dev_free(s.uend, st); dev_free(s.indeg, st); dev_free(s.queue, st);
+    dev_free(s.lt_ptr, st); dev_free(s.lt_idx, st); dev_free(s.lt_fill, st);
+    dev_free(s.scan_blk, st); dev_free(s.ctrl, st); dev_free(s.chain, st);
     s = LevelizeScratch();
 }
 
@@ -421,20 +421,20 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
     *info = LevelizeInfo();
     if (n == 0) return cudaSuccess;
     if (s.n_cap < n) {
-        cudaFree(s.ustart); cudaFree(s.uend); cudaFree(s.indeg); cudaFree(s.queue);
-        cudaFree(s.lt_ptr); cudaFree(s.lt_fill); cudaFree(s.scan_blk); cudaFree(s.ctrl);
-        cudaFree(s.chain);
+        dev_free(s.ustart, st); dev_free(s.uend, st); dev_free(s.indeg, st);
+        dev_free(s.queue, st); dev_free(s.lt_ptr, st); dev_free(s.lt_fill, st);
+        dev_free(s.scan_blk, st); dev_free(s.ctrl, st); dev_free(s.chain, st);
         s.ustart = s.uend = s.lt_ptr = s.lt_fill = s.scan_blk = nullptr;
         s.indeg = s.queue = s.ctrl = s.chain = nullptr;
-        LV_CK(cudaMalloc(&s.ustart, sizeof(int64_t) * n));
-        LV_CK(cudaMalloc(&s.uend, sizeof(int64_t) * n));
-        LV_CK(cudaMalloc(&s.indeg, sizeof(int32_t) * n));
-        LV_CK(cudaMalloc(&s.queue, sizeof(int32_t) * 2 * (size_t)n));
-        LV_CK(cudaMalloc(&s.lt_ptr, sizeof(int64_t) * ((size_t)n + 1)));
-        LV_CK(cudaMalloc(&s.lt_fill, sizeof(int64_t) * n));
-        LV_CK(cudaMalloc(&s.scan_blk, sizeof(int64_t) * scan_scratch_elems(n)));
-        LV_CK(cudaMalloc(&s.ctrl, sizeof(int32_t) * kCtrlInts));
-        LV_CK(cudaMalloc(&s.chain, sizeof(int32_t) * 8 * (size_t)n));
+        LV_CK(dev_alloc((void **)&s.ustart, sizeof(int64_t) * n, st));
+        LV_CK(dev_alloc((void **)&s.uend, sizeof(int64_t) * n, st));
+        LV_CK(dev_alloc((void **)&s.indeg, sizeof(int32_t) * n, st));
+        LV_CK(dev_alloc((void **)&s.queue, sizeof(int32_t) * 2 * (size_t)n, st));
+        LV_CK(dev_alloc((void **)&s.lt_ptr, sizeof(int64_t) * ((size_t)n + 1), st));
+        LV_CK(dev_alloc((void **)&s.lt_fill, sizeof(int64_t) * n, st));
+        LV_CK(dev_alloc((void **)&s.scan_blk, sizeof(int64_t) * scan_scratch_elems(n), st));
+        LV_CK(dev_alloc((void **)&s.ctrl, sizeof(int32_t) * kCtrlInts, st));
+        LV_CK(dev_alloc((void **)&s.chain, sizeof(int32_t) * 8 * (size_t)n, st));
         s.n_cap = n;
     }
     int32_t *J0 = s.chain, *D0 = J0 + n, *J1 = D0 + n, *D1 = J1 + n, *nxt = D1 + n;
@@ -458,9 +458,9 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
         LV_CK(cudaMemcpyAsync(&nl, s.lt_ptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, st));
         LV_CK(cudaStreamSynchronize(st));
         if (s.lt_cap < nl || s.lt_idx == nullptr) {
-            cudaFree(s.lt_idx);
+            dev_free(s.lt_idx, st);
             s.lt_idx = nullptr;
-            LV_CK(cudaMalloc(&s.lt_idx, sizeof(int32_t) * (size_t)(nl > 0 ? nl : 1)));
+            LV_CK(dev_alloc((void **)&s.lt_idx, sizeof(int32_t) * (size_t)(nl > 0 ? nl : 1), st));
             s.lt_cap = nl;
         }
         LV_CK(cudaMemcpyAsync(s.lt_fill, s.lt_ptr, sizeof(int64_t) * n, cudaMemcpyDeviceToDevice,

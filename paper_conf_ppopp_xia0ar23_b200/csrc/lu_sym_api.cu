@@ -11,6 +11,32 @@
 
 using namespace lusym;
 
+namespace lusym {
+
+cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s)
+{
+    static bool configured[64] = {};
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    if (dev >= 0 && dev < 64 && !configured[dev]) {
+        cudaMemPool_t pool;
+        if (cudaDeviceGetDefaultMemPool(&pool, dev) == cudaSuccess) {
+            uint64_t thr = UINT64_MAX;
+            cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &thr);
+        }
+        configured[dev] = true;
+    }
+    return cudaMallocAsync(p, bytes, s);
+}
+
+void dev_free(void *p, cudaStream_t s)
+{
+    if (p) cudaFreeAsync(p, s);
+}
+
+}  // namespace lusym
+
 namespace {
 
 thread_local std::string g_err;
@@ -82,6 +108,7 @@ struct lu_sym {
     int64_t scratch_bytes = 0;
     int64_t launches = 0;
     int64_t *row_prof = nullptr;  // borrowed, set by lu_sym_set_row_profile
+    cudaStream_t stream = nullptr;  // stream of the last call (scratch is freed on it)
 };
 
 namespace {
@@ -101,7 +128,7 @@ lu_status dalloc(lu_sym *h, T **p, size_t elems)
 {
     size_t bytes = elems * sizeof(T);
     if (bytes == 0) bytes = 16;
-    cudaError_t e = cudaMalloc(reinterpret_cast<void **>(p), bytes);
+    cudaError_t e = dev_alloc(reinterpret_cast<void **>(p), bytes, h->stream);
     if (e != cudaSuccess)
         return fail(LU_ERR_NOMEM, "cudaMalloc(%zu bytes): %s", bytes, cudaGetErrorString(e));
     h->scratch_bytes += (int64_t)bytes;
@@ -110,18 +137,11 @@ lu_status dalloc(lu_sym *h, T **p, size_t elems)
 
 void free_handle(lu_sym *h)
 {
-    cudaFree(h->ell);
-    cudaFree(h->gbitmap);
-    cudaFree(h->dbitmap);
-    cudaFree(h->gspill);
-    cudaFree(h->dstats);
-    cudaFree(h->scan_blk);
-    cudaFree(h->dbad);
-    cudaFree(h->stg);
-    cudaFree(h->pool);
-    cudaFree(h->row_off);
-    cudaFree(h->unstaged);
-    levelize_free(h->lev);
+    cudaStream_t s = h->stream;
+    void *bufs[] = {h->ell, h->gbitmap, h->dbitmap, h->gspill, h->dstats, h->scan_blk, h->dbad,
+                    h->stg, h->pool, h->row_off, h->unstaged};
+    for (void *b : bufs) dev_free(b, s);
+    levelize_free(h->lev, s);
     for (int k = 0; k < kEvN; ++k)
         for (int j = 0; j < 2; ++j)
             if (h->ev[k][j]) cudaEventDestroy(h->ev[k][j]);
@@ -324,7 +344,8 @@ lu_status ensure_pool(lu_sym *h)
         h->pool_cap = -1;  // no room: every row is re-traversed by emit
         return LU_OK;
     }
-    cudaError_t e = cudaMalloc(&h->pool, (size_t)cap * sizeof(int32_t));
+    cudaError_t e = dev_alloc(reinterpret_cast<void **>(&h->pool), (size_t)cap * sizeof(int32_t),
+                              h->stream);
     if (e != cudaSuccess) {
         cudaGetLastError();
         h->pool = nullptr;
@@ -380,6 +401,7 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
                     sizeof(lu_sym_opts));
     cudaStream_t s = (cudaStream_t)stream;
     lu_sym *h = new lu_sym();
+    h->stream = s;
     if (opts) h->opts = *opts; else lu_sym_default_opts(&h->opts);
     memset(&h->stats, 0, sizeof(h->stats));
     h->n = n;
@@ -467,6 +489,7 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
     lu_status st = check_device(h);
     if (st != LU_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
+    h->stream = s;
     ev_begin(h, kEvCount, s);
     int mode = kCount;
     if (h->staging) {
@@ -501,6 +524,7 @@ lu_status lu_sym_scan(lu_sym *h, const int32_t *d_fill_count, int64_t *d_row_ptr
     lu_status st = check_device(h);
     if (st != LU_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
+    h->stream = s;
     ev_begin(h, kEvScan, s);
     CK(scan_counts(h->n, d_fill_count, d_row_ptr_lu, h->scan_blk, s));
     h->launches += h->n > 0 ? 3 : 1;
@@ -528,6 +552,7 @@ lu_status lu_sym_emit(lu_sym *h, int32_t row_begin, int32_t row_end, const int64
     lu_status st = check_device(h);
     if (st != LU_OK) return st;
     cudaStream_t s = (cudaStream_t)stream;
+    h->stream = s;
     int64_t need = 0;
     CK(cudaMemcpyAsync(&need, d_row_ptr_lu + row_end, sizeof(int64_t), cudaMemcpyDeviceToHost,
                        s));
@@ -603,6 +628,7 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
         if (st != LU_OK) return st;
     }
     cudaStream_t s = (cudaStream_t)stream;
+    if (h) h->stream = s;
     LevelizeScratch tmp;
     LevelizeScratch &scr = h ? h->lev : tmp;
     const int flags = h ? h->opts.flags : 0;
@@ -614,7 +640,7 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
                                  (flags & LU_F_KAHN_WIDE_ONLY) != 0, scr, d_level, &info, s,
                                  &where);
     if (h) ev_end(h, kEvLev, s);
-    if (!h) levelize_free(tmp);
+    if (!h) levelize_free(tmp, s);
     if (e != cudaSuccess)
         return fail(e == cudaErrorMemoryAllocation ? LU_ERR_NOMEM : LU_ERR_CUDA,
                     "levelize: %s: %s", where, cudaGetErrorString(e));
@@ -676,8 +702,7 @@ lu_status lu_sym_set_row_profile(lu_sym *h, int64_t *d_prof)
 void lu_sym_destroy(lu_sym *h)
 {
     if (!h) return;
-    cudaDeviceSynchronize();
-    free_handle(h);
+    free_handle(h);  // stream-ordered frees on the handle's last stream
 }
 
 }  // extern "C"
