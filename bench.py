@@ -238,6 +238,7 @@ def run_ours(args, rank, world, local_rank):
     state = {}
 
     def step():
+        state.clear()  # let the allocator reuse the previous step's output blocks
         fc = torch.zeros(n, dtype=torch.int32, device=dev)
         h.count(rb, re_, fc)                                     # S3 (symbolic_1)
         if world > 1:

@@ -68,8 +68,12 @@ enum {
     LU_F_NO_PRUNE = 1 << 3,      /* levelize over every U edge (no transitive pruning)       */
     LU_F_KAHN_WIDE_ONLY = 1 << 4,/* levelize: never use the single-CTA narrow phase          */
     LU_F_NO_CONTRACT = 1 << 5,   /* levelize: Kahn over every column (no chain contraction)  */
-    LU_F_TWO_PASS = 1 << 6       /* no staging pool: emit re-runs the traversal (Alg. 3 as
+    LU_F_TWO_PASS = 1 << 6,      /* no staging pool: emit re-runs the traversal (Alg. 3 as
                                     printed, symbolic_2 repeats symbolic_1's work)           */
+    LU_F_ONE_CLASS = 1 << 7,     /* one row class (Alg. 3's single chunk size) instead of
+                                    Alg. 4's row classes by scratch need (L272-277)          */
+    LU_F_FORCE_CLASSES = 1 << 8  /* test knob: split row classes down to 64 shared words even
+                                    when that does not add rows in flight                     */
 };
 
 typedef struct {
@@ -104,7 +108,8 @@ typedef struct {
     int32_t num_levels;           /* after lu_levelize with this handle                      */
     int32_t levelize_wide_levels, levelize_narrow_levels; /* Kahn rounds by mode            */
     int32_t levelize_rank_rounds; /* pointer-jumping rounds of the chain contraction        */
-    int32_t reserved[2];
+    int32_t row_classes;          /* Alg. 4 row classes planned (1 = a single class)         */
+    int32_t reserved[1];
     int64_t pool_bytes;           /* staging pool size (0: two-pass mode)                    */
     int64_t rows_retraversed;     /* rows of the last emit that were not staged              */
     int64_t kernel_launches;      /* kernels this handle launched since create (all calls)  */

@@ -38,7 +38,7 @@ LU_OK, LU_ERR_ARG, LU_ERR_INPUT, LU_ERR_NOMEM, LU_ERR_CAPACITY = 0, 1, 2, 3, 4
 LU_ERR_CUDA, LU_ERR_STATE, LU_ERR_INTERNAL = 5, 7, 8
 DEP_U, DEP_GLU3 = 0, 1
 F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4, 8, 16
-F_NO_CONTRACT, F_TWO_PASS = 32, 64
+F_NO_CONTRACT, F_TWO_PASS, F_ONE_CLASS, F_FORCE_CLASSES = 32, 64, 128, 256
 
 
 class LuSymError(RuntimeError):
@@ -68,7 +68,8 @@ class _Stats(ctypes.Structure):
                 ("queue_capacity", ctypes.c_int32), ("num_levels", ctypes.c_int32),
                 ("levelize_wide_levels", ctypes.c_int32),
                 ("levelize_narrow_levels", ctypes.c_int32),
-                ("levelize_rank_rounds", ctypes.c_int32), ("reserved", ctypes.c_int32 * 2),
+                ("levelize_rank_rounds", ctypes.c_int32), ("row_classes", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 1),
                 ("pool_bytes", ctypes.c_int64), ("rows_retraversed", ctypes.c_int64),
                 ("kernel_launches", ctypes.c_int64)]
 

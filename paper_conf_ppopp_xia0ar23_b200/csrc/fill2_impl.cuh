@@ -30,14 +30,8 @@
 namespace lusym {
 namespace f2 {
 
-#ifndef LUSYM_LAYOUT_CONST
-#define LUSYM_LAYOUT_CONST 1
-#endif
 #ifndef LUSYM_SWZ
 #define LUSYM_SWZ 1
-#endif
-#ifndef LUSYM_SHPTX
-#define LUSYM_SHPTX 0
 #endif
 #ifndef LUSYM_THREADS_PER_SM  // register budget: 65536 / this
 #define LUSYM_THREADS_PER_SM 2048
@@ -84,37 +78,67 @@ __device__ __forceinline__ int block_scan_excl(int x, int *s, int &total)
     return r;
 }
 
-// Shared-memory bitmaps are stored with the word index XOR-swizzled inside each group of 32
-// words, so that words 32 (or a multiple of 32) apart — grid neighbours at +-k for k a
-// multiple of 1024 — fall into different banks.
-template <bool GB>
+// Visited bitmap of the row in flight.
+//   kVisSmem   : every word in shared memory
+//   kVisSplit  : words [0, lbw) in shared memory, the rest in the CTA's HBM slot — row classes
+//                (Alg. 4): rows below lbw*32 keep their whole BFS region
+//                (all vertices < src) in shared memory, only pattern marks above it go to HBM
+//   kVisGlobal : every word in the CTA's HBM slot
+// Shared words are XOR-swizzled inside each group of 32, so words 32 (or a multiple of 32)
+// apart — grid neighbours at +-k for k a multiple of 1024 — fall into different banks.
+template <int VIS>
+struct VisMap {
+    uint32_t *s;  // shared part
+    uint32_t *g;  // HBM slot (word index = vertex >> 5)
+    int lbw;      // words held in shared memory (kVisSplit)
+};
+
+template <int VIS>
 __device__ __forceinline__ int phys(int w)
 {
-    if (GB || !LUSYM_SWZ) return w;
+    if (!LUSYM_SWZ) return w;
     return w ^ ((w >> 5) & 31);
 }
 
-template <bool GB>
-__device__ __forceinline__ uint32_t bm_word(const uint32_t *bm, int w)
+template <int VIS>
+__device__ __forceinline__ bool in_smem(const VisMap<VIS> &m, int w)
 {
-    if (GB) return __ldcg(bm + w);
-    return bm[phys<GB>(w)];
+    if (VIS == kVisGlobal) return false;
+    if (VIS == kVisSmem) return true;
+    return w < m.lbw;
 }
 
-template <bool GB>
-__device__ __forceinline__ bool visited(const uint32_t *bm, int v)
+template <int VIS>
+__device__ __forceinline__ uint32_t bm_word(const VisMap<VIS> &m, int w)
 {
-    return (bm_word<GB>(bm, v >> 5) >> (v & 31)) & 1u;
+    if (in_smem(m, w)) return m.s[phys<VIS>(w)];
+    return __ldcg(m.g + w);
+}
+
+template <int VIS>
+__device__ __forceinline__ void bm_zero(const VisMap<VIS> &m, int w)
+{
+    if (in_smem(m, w))
+        m.s[phys<VIS>(w)] = 0;
+    else
+        m.g[w] = 0;
+}
+
+template <int VIS>
+__device__ __forceinline__ bool visited(const VisMap<VIS> &m, int v)
+{
+    return (bm_word(m, v >> 5) >> (v & 31)) & 1u;
 }
 
 // test-and-set (reading R26): true iff this call set the bit.  The level-1 summary sm gets bit
 // w when visited word w first becomes non-zero, so scans and clears skip empty stretches.
-template <bool GB>
-__device__ __forceinline__ bool mark(uint32_t *bm, uint32_t *sm, int v)
+template <int VIS>
+__device__ __forceinline__ bool mark(const VisMap<VIS> &m, uint32_t *sm, int v)
 {
     const uint32_t b = 1u << (v & 31);
-    const uint32_t old = atomicOr(bm + phys<GB>(v >> 5), b);
-    if (old == 0) atomicOr(sm + (v >> 10), 1u << ((v >> 5) & 31));
+    const int w = v >> 5;
+    const uint32_t old = in_smem(m, w) ? atomicOr(m.s + phys<VIS>(w), b) : atomicOr(m.g + w, b);
+    if (old == 0) atomicOr(sm + (v >> 10), 1u << (w & 31));
     return !(old & b);
 }
 
@@ -131,34 +155,6 @@ __device__ __forceinline__ void load_nb(const int32_t *ell, int f, int (&nb)[W])
         const int4 a = __ldg(reinterpret_cast<const int4 *>(ell + (size_t)f * W));
         nb[0] = a.x; nb[1] = a.y; nb[2] = a.z; nb[3] = a.w;
     }
-}
-
-// Shared-memory bitmap access through 32-bit shared-window addresses (computed once per BFS
-// level), so the hot neighbour test is LDS + shift + test without re-deriving the CTA's shared
-// base for every neighbour.
-__device__ __forceinline__ uint32_t lds_u32(uint32_t addr)
-{
-    uint32_t v;
-    asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(addr));
-    return v;
-}
-
-__device__ __forceinline__ uint32_t atoms_or(uint32_t addr, uint32_t b)
-{
-    uint32_t old;
-    asm volatile("atom.shared.or.b32 %0, [%1], %2;" : "=r"(old) : "r"(addr), "r"(b) : "memory");
-    return old;
-}
-
-// test-and-set of v in a shared bitmap at window address bmw (summary at smw); see mark()
-__device__ __forceinline__ bool visit_s(uint32_t bmw, uint32_t smw, int v)
-{
-    const uint32_t wa = bmw + 4u * (uint32_t)phys<false>(v >> 5);
-    const uint32_t b = 1u << (v & 31);
-    if (lds_u32(wa) & b) return false;
-    const uint32_t old = atoms_or(wa, b);
-    if (old == 0) atoms_or(smw + 4u * (uint32_t)(v >> 10), 1u << ((v >> 5) & 31));
-    return !(old & b);
 }
 
 __device__ __forceinline__ int64_t heavy_off(int lo, int hi)
@@ -218,8 +214,8 @@ __device__ int next_word(const uint32_t *sm, int w0, int whi, int *sred)
 // there are (at most cap when CAPPED).  WRITE: stores them at dst[base + k] for base + k < dcap.
 // One visited word per thread per chunk; on ranges wider than a chunk the level-1 summary sm
 // skips empty stretches before each chunk.  Block-uniform.
-template <int NT, bool GB, bool WRITE, bool CAPPED>
-__device__ int scan_bits(const uint32_t *bm, const uint32_t *sm, const uint32_t *dm, int lo,
+template <int NT, int VIS, bool WRITE, bool CAPPED>
+__device__ int scan_bits(const VisMap<VIS> &bm, const uint32_t *sm, const uint32_t *dm, int lo,
                          int hi, int32_t *dst, int64_t base, int64_t dcap, int cap, int *sscan)
 {
     if (lo >= hi) return 0;
@@ -234,7 +230,7 @@ __device__ int scan_bits(const uint32_t *bm, const uint32_t *sm, const uint32_t 
         const int w = w0 + (int)threadIdx.x;
         uint32_t word = 0;
         if (w <= whi) {
-            word = bm_word<GB>(bm, w);
+            word = bm_word(bm, w);
             if (w == wlo) word &= kFull << (lo & 31);
             if (w == whi) {
                 const int hb = (hi - 1) & 31;
@@ -257,32 +253,32 @@ __device__ int scan_bits(const uint32_t *bm, const uint32_t *sm, const uint32_t 
 }
 
 // Pending thresholds not yet finished: the first cap set bits of bm & ~dm in [lo, hi), sorted.
-template <int NT, bool GB>
-__device__ __forceinline__ int collect(const uint32_t *bm, const uint32_t *sm, const uint32_t *dm,
+template <int NT, int VIS>
+__device__ __forceinline__ int collect(const VisMap<VIS> &bm, const uint32_t *sm, const uint32_t *dm,
                                        int lo, int hi, int32_t *out, int cap, int *sscan)
 {
-    return scan_bits<NT, GB, true, true>(bm, sm, dm, lo, hi, out, 0, cap, cap, sscan);
+    return scan_bits<NT, VIS, true, true>(bm, sm, dm, lo, hi, out, 0, cap, cap, sscan);
 }
 
 // Count the set bits in [lo, hi) and, if WRITE, store them in increasing order at dst[base ..]
 // (bounded by cap).  Returns the count.
-template <int NT, bool GB, bool WRITE>
-__device__ __forceinline__ int emit_range(const uint32_t *bm, const uint32_t *sm, int lo, int hi,
+template <int NT, int VIS, bool WRITE>
+__device__ __forceinline__ int emit_range(const VisMap<VIS> &bm, const uint32_t *sm, int lo, int hi,
                                           int32_t *dst, int base, int64_t cap, int *sscan)
 {
-    return scan_bits<NT, GB, WRITE, false>(bm, sm, nullptr, lo, hi, dst, base, cap, 0, sscan);
+    return scan_bits<NT, VIS, WRITE, false>(bm, sm, nullptr, lo, hi, dst, base, cap, 0, sscan);
 }
 
 // Zero the visited words [wlo, whi] and their summary bits (walk the summary if wide).
-template <int NT, bool GB>
-__device__ void clear_words(uint32_t *bm, uint32_t *sm, int wlo, int whi)
+template <int NT, int VIS>
+__device__ void clear_words(const VisMap<VIS> &bm, uint32_t *sm, int wlo, int whi)
 {
     if (whi < wlo) return;
     if (whi - wlo < 4 * NT) {
-        for (int w = wlo + (int)threadIdx.x; w <= whi; w += NT) bm[phys<GB>(w)] = 0;
+        for (int w = wlo + (int)threadIdx.x; w <= whi; w += NT) bm_zero(bm, w);
     } else {
         for (int sidx = (wlo >> 5) + (int)threadIdx.x; sidx <= (whi >> 5); sidx += NT)
-            for (uint32_t t = sm[sidx]; t; t &= t - 1) bm[phys<GB>((sidx << 5) + __ffs(t) - 1)] = 0;
+            for (uint32_t t = sm[sidx]; t; t &= t - 1) bm_zero(bm, (sidx << 5) + __ffs(t) - 1);
     }
     __syncthreads();
     for (int sidx = (wlo >> 5) + (int)threadIdx.x; sidx <= (whi >> 5); sidx += NT) sm[sidx] = 0;
@@ -296,18 +292,14 @@ struct RowAcc {
 // Scan the vertices L[0..cnt) (smem, HBM past q) of one BFS level below t0: test-and-set every
 // neighbour; new ones below t0 form the next level (appended to NF), new ones above t0 are
 // pattern entries (L130-147).
-template <int NT, int W, bool GB>
-__device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, uint32_t *sm,
+template <int NT, int W, int VIS>
+__device__ __forceinline__ void scan_level(const Fill2Params &p, const VisMap<VIS> &bm, uint32_t *sm,
                                            const int32_t *L,
                                            const int32_t *gL, int cnt, int *ncnt, int32_t *NF,
                                            int32_t *gNF, const int i, const int t0, int &nmin,
                                            RowAcc &a)
 {
     const int tid = threadIdx.x, lane = tid & 31;
-#if LUSYM_SHPTX
-    const uint32_t bmw = GB ? 0u : (uint32_t)__cvta_generic_to_shared(bm);
-    const uint32_t smw = (uint32_t)__cvta_generic_to_shared(sm);
-#endif
     for (int base = 0; base < cnt; base += NT) {
         const int k = base + tid;
         const bool valid = k < cnt;
@@ -326,16 +318,7 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, u
 #pragma unroll
             for (int s = 0; s < W; ++s) {
                 const int w = nb[s];
-#if LUSYM_SHPTX
-                bool nw;
-                if constexpr (GB)
-                    nw = w >= 0 && !visited<GB>(bm, w) && mark<GB>(bm, sm, w);
-                else
-                    nw = w >= 0 && visit_s(bmw, smw, w);
-                if (nw) {
-#else
-                if (w >= 0 && !visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
-#endif
+                if (w >= 0 && !visited(bm, w) && mark(bm, sm, w)) {
                     if (w < t0) {
                         frm |= 1u << s;
                     } else if (w > i) {
@@ -394,7 +377,7 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, u
                 int w = -1;
                 if (e < len) {
                     w = __ldg(p.ci + off + e);
-                    if (!visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
+                    if (!visited(bm, w) && mark(bm, sm, w)) {
                         if (w < t0) {
                             fr = true;
                             nmin = min(nmin, w);
@@ -411,8 +394,8 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, uint32_t *bm, u
 }
 
 // Level-synchronous BFS from threshold t0 over unvisited vertices < t0 (Alg. 1).
-template <int NT, int W, bool GB>
-__device__ void bfs(const Fill2Params &p, Hdr &h, uint32_t *bm, uint32_t *sm, int32_t *qA,
+template <int NT, int W, int VIS>
+__device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_t *sm, int32_t *qA,
                     int32_t *qB,
                     int32_t *gA, int32_t *gB, const int i, const int t0, RowAcc &a)
 {
@@ -428,7 +411,7 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, uint32_t *bm, uint32_t *sm, in
         int *ncnt = &h.cnt[(lev + 1) % 3];
         if (tid == 0) h.cnt[(lev + 2) % 3] = 0;
         int nmin = INT_MAX;
-        scan_level<NT, W, GB>(p, bm, sm, F, gF, fsize, ncnt, NF, gNF, i, t0, nmin, a);
+        scan_level<NT, W, VIS>(p, bm, sm, F, gF, fsize, ncnt, NF, gNF, i, t0, nmin, a);
         a.lmin = min(a.lmin, nmin);
         __syncthreads();
         fsize = *ncnt;
@@ -448,34 +431,26 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
     Hdr &h = *reinterpret_cast<Hdr *>(smem);
     // shared layout: header | visited bitmap (at a constant offset, so the hot bit tests need
     // no address arithmetic beyond the word index) | summary | two frontier queues
-    uint32_t *bm;
+    VisMap<VIS> bm;
+    bm.g = p.gbitmap ? p.gbitmap + (size_t)blockIdx.x * p.gbitmap_stride : nullptr;
+    bm.lbw = p.lbw;
     uint32_t *sm;
     int32_t *qA, *qB;
-#if LUSYM_LAYOUT_CONST
     if constexpr (GB) {
-        bm = p.gbitmap + (size_t)blockIdx.x * p.gbitmap_stride;
+        bm.s = nullptr;
         sm = reinterpret_cast<uint32_t *>(smem + kHdrBytes);
     } else {
-        bm = reinterpret_cast<uint32_t *>(smem + kHdrBytes);
-        sm = bm + p.nw;
+        bm.s = reinterpret_cast<uint32_t *>(smem + kHdrBytes);
+        sm = bm.s + p.nw;  // p.nw = shared visited words (whole swizzle groups)
     }
     qA = reinterpret_cast<int32_t *>(sm + p.sw);
     qB = qA + p.q;
-#else
-    qA = reinterpret_cast<int32_t *>(smem + kHdrBytes);
-    qB = qA + p.q;
-    sm = reinterpret_cast<uint32_t *>(qB + p.q);
-    if constexpr (GB)
-        bm = p.gbitmap + (size_t)blockIdx.x * p.gbitmap_stride;
-    else
-        bm = sm + p.sw;
-#endif
     int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
     int32_t *gB = gA + p.spill_cap;
     const int tid = threadIdx.x, lane = tid & 31;
     for (int w = tid; w < p.sw; w += NT) sm[w] = 0;
     if constexpr (!GB)
-        for (int w = tid; w < p.nw; w += NT) bm[w] = 0;
+        for (int w = tid; w < p.nw; w += NT) bm.s[w] = 0;
 
     RowAcc a;
     a.te = a.sv = a.spills = 0;
@@ -511,7 +486,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
         for (int64_t k = rb + tid; k < re; k += NT) {
             const int v = __ldg(p.ci + k);
             ++a.te;
-            mark<GB>(bm, sm, v);
+            mark(bm, sm, v);
             if (v < i) {
                 atomicMin(&h.minseed, v);
                 a.lmin = min(a.lmin, v);
@@ -522,7 +497,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                 h.diag = 1;
             }
         }
-        if (tid == 0) mark<GB>(bm, sm, i);
+        if (tid == 0) mark(bm, sm, i);
         __syncthreads();
 
         int ptr = h.minseed - 1;  // every unprocessed threshold is > ptr
@@ -546,7 +521,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
         int cap = p.wcap;
         // ---- thresholds in increasing order (L130)
         for (;;) {
-            const int wc = collect<NT, GB>(bm, sm, dused ? dm : nullptr, ptr + 1, i, qA, cap,
+            const int wc = collect<NT, VIS>(bm, sm, dused ? dm : nullptr, ptr + 1, i, qA, cap,
                                            h.scan);
             if (wc == 0) break;
             ++n_win;
@@ -574,7 +549,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
 #pragma unroll
                     for (int s = 0; s < W; ++s) {
                         const int w = nb[s];
-                        if (w >= 0 && w < t && !visited<GB>(bm, w)) simple = false;
+                        if (w >= 0 && w < t && !visited(bm, w)) simple = false;
                     }
                     if (!simple) {
                         atomicMin(&h.tns, t);
@@ -583,7 +558,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
 #pragma unroll
                         for (int s = 0; s < W; ++s) {
                             const int w = nb[s];
-                            if (w > t && !visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
+                            if (w > t && !visited(bm, w) && mark(bm, sm, w)) {
                                 if (w < i) {
                                     nm = min(nm, w);
                                 } else {
@@ -605,7 +580,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                     bool ok = true;
                     for (int e = lane; e < len; e += 32) {
                         const int w = __ldg(p.ci + off + e);
-                        if (w < tt && !visited<GB>(bm, w)) ok = false;
+                        if (w < tt && !visited(bm, w)) ok = false;
                     }
                     ok = __all_sync(kFull, ok);
                     if (lane == 0) {
@@ -618,7 +593,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                     } else {
                         for (int e = lane; e < len; e += 32) {
                             const int w = __ldg(p.ci + off + e);
-                            if (w > tt && !visited<GB>(bm, w) && mark<GB>(bm, sm, w)) {
+                            if (w > tt && !visited(bm, w) && mark(bm, sm, w)) {
                                 if (w < i) {
                                     nm = min(nm, w);
                                 } else {
@@ -641,7 +616,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
             const int nptr = m > last ? last : (m == tns ? m : m - 1);
             // every visited bit in (ptr, nptr] is an L entry now (no BFS has marked below m yet):
             // emit / count them in increasing order as the pointer passes (L122-143)
-            Lcnt += emit_range<NT, GB, MODE != kCount>(bm, sm, ptr + 1, nptr + 1, ldst, Lcnt, lcap,
+            Lcnt += emit_range<NT, VIS, MODE != kCount>(bm, sm, ptr + 1, nptr + 1, ldst, Lcnt, lcap,
                                                        h.scan);
             if (nptr < last) {  // simple candidates beyond the pointer are finished: mark them
                 for (int k = tid; k < wc; k += NT) {
@@ -652,14 +627,14 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
             }
             __syncthreads();
             if (m <= last && m == tns) {  // smallest pending threshold: below-exploration
-                bfs<NT, W, GB>(p, h, bm, sm, qA, qB, gA, gB, i, m, a);
+                bfs<NT, W, VIS>(p, h, bm, sm, qA, qB, gA, gB, i, m, a);
                 ++n_bfs;
             }
             cap = m <= last ? min(cap, kSmallWin) : min(2 * cap, p.wcap);
             ptr = nptr;
         }
         // thresholds finished ahead of the pointer and never re-collected: the rest of (ptr, i)
-        Lcnt += emit_range<NT, GB, MODE != kCount>(bm, sm, ptr + 1, i, ldst, Lcnt, lcap, h.scan);
+        Lcnt += emit_range<NT, VIS, MODE != kCount>(bm, sm, ptr + 1, i, ldst, Lcnt, lcap, h.scan);
         if (dused)  // leave the done map zero for the next row
             for (int w = (h.minseed >> 5) + tid; w <= ((i - 1) >> 5); w += NT) dm[w] = 0;
 
@@ -688,7 +663,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                 int32_t *dst = p.pool + off;
                 for (int k = tid; k < Lcnt; k += NT) dst[k] = ldst[k];
                 if (diag && tid == 0) dst[Lcnt] = i;
-                emit_range<NT, GB, true>(bm, sm, i + 1, gmax + 1, dst + Lcnt + diag, 0, INT64_MAX,
+                emit_range<NT, VIS, true>(bm, sm, i + 1, gmax + 1, dst + Lcnt + diag, 0, INT64_MAX,
                                          h.scan);
             }
         } else {
@@ -696,7 +671,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                 if (tid == 0) atomicAdd(p.stats + kStatErr, 1ull);
             } else {
                 if (diag && tid == 0) ldst[Lcnt] = i;
-                emit_range<NT, GB, true>(bm, sm, i + 1, gmax + 1, ldst + Lcnt + diag, 0, INT64_MAX,
+                emit_range<NT, VIS, true>(bm, sm, i + 1, gmax + 1, ldst + Lcnt + diag, 0, INT64_MAX,
                                          h.scan);
             }
         }
@@ -713,7 +688,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
             }
         }
         // ---- clear the dirty word range (fill(:) = 0 for the next row, L115)
-        clear_words<NT, GB>(bm, sm, gmin >> 5, gmax >> 5);
+        clear_words<NT, VIS>(bm, sm, gmin >> 5, gmax >> 5);
         __syncthreads();
     }
 
@@ -781,8 +756,10 @@ cudaError_t dispatch_w_vis(int w, int vis, Args... args)
 {
     if (w == 4 && vis == kVisSmem) return Op<NT, 4, kVisSmem>::run(args...);
     if (w == 4 && vis == kVisGlobal) return Op<NT, 4, kVisGlobal>::run(args...);
+    if (w == 4 && vis == kVisSplit) return Op<NT, 4, kVisSplit>::run(args...);
     if (w == 8 && vis == kVisSmem) return Op<NT, 8, kVisSmem>::run(args...);
     if (w == 8 && vis == kVisGlobal) return Op<NT, 8, kVisGlobal>::run(args...);
+    if (w == 8 && vis == kVisSplit) return Op<NT, 8, kVisSplit>::run(args...);
     return cudaErrorInvalidValue;
 }
 

@@ -4,13 +4,14 @@
 
 namespace lusym {
 
-size_t fill2_smem_bytes(int n, int q, int vis)
+// header | visited words held in shared memory (smem_words, whole swizzle groups) | level-1
+// summary (one bit per visited word, all n) | two frontier queues of q entries
+size_t fill2_smem_bytes(int n, int smem_words, int q)
 {
-    // header | visited bitmap (kVisSmem) | level-1 summary | two frontier queues
-    size_t b = kHdrBytes + 2 * (size_t)q * sizeof(int32_t);
     const size_t words = (size_t)((n + 31) / 32);
+    size_t b = kHdrBytes + 2 * (size_t)q * sizeof(int32_t);
     b += (words + 31) / 32 * sizeof(uint32_t);
-    if (vis == kVisSmem) b += (words + 31) / 32 * 32 * sizeof(uint32_t);  // whole swizzle groups
+    b += (size_t)smem_words * sizeof(uint32_t);
     return (b + 15) & ~(size_t)15;
 }
 

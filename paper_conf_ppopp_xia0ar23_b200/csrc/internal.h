@@ -30,7 +30,8 @@ struct Fill2Params {
     int64_t gbitmap_stride;   // words per slot
     int32_t *gspill;          // frontier spill, 2 x spill_cap per CTA
     int64_t spill_cap;
-    int32_t nw;               // visited bitmap words = ceil(n/32)
+    int32_t nw;               // visited words held in shared memory (whole swizzle groups)
+    int32_t lbw;              // kVisSplit: words [0, lbw) are in shared memory
     int32_t sw;               // summary words = ceil(nw/32) (shared memory)
     int32_t q;                // shared frontier capacity per buffer (entries)
     int32_t wcap;             // window capacity (<= q); 1 = one threshold at a time
@@ -55,7 +56,8 @@ enum Fill2Mode { kCount = 0, kEmit = 1, kStage = 2 };
 // Visited storage of a row in flight (frontiers are lists in shared memory, spilling to HBM).
 //   kVisSmem   : visited bitmap in shared memory
 //   kVisGlobal : visited bitmap in an HBM slot per CTA (n too large for shared memory)
-enum Fill2Vis { kVisSmem = 0, kVisGlobal = 1 };
+//   kVisSplit  : words [0, lbw) in shared memory, the rest in the HBM slot (row classes)
+enum Fill2Vis { kVisSmem = 0, kVisGlobal = 1, kVisSplit = 2 };
 
 // Stream-ordered device allocations from the current device's default memory pool, whose
 // release threshold is raised once so that memory freed by one handle stays reserved for the
@@ -64,7 +66,7 @@ cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s);
 void dev_free(void *p, cudaStream_t s);
 
 // fill2_kernels.cu (host dispatch; kernels instantiated in fill2_nt*.cu)
-size_t fill2_smem_bytes(int n, int q, int vis);
+size_t fill2_smem_bytes(int n, int smem_words, int q);
 cudaError_t fill2_configure(int nt, int w, int vis, size_t smem);
 cudaError_t fill2_occupancy(int nt, int w, int vis, size_t smem, int *occ);
 cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, int mode, int vis, int grid,

@@ -4,6 +4,7 @@
 
 #include <cstdarg>
 #include <cstdio>
+#include <algorithm>
 #include <cstring>
 #include <string>
 #include <utility>
@@ -61,9 +62,24 @@ lu_status fail(lu_status s, const char *fmt, ...)
     } while (0)
 
 enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvN = 4 };
-enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11 };
+enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11, kSlotClassCounter = 16 };
 
 }  // namespace
+
+struct RowClass {
+    int32_t lo, hi;   // rows [lo, hi)
+    int vis;          // kVisSmem / kVisGlobal / kVisSplit
+    int smem_words;   // visited words held in shared memory
+    int lbw;          // kVisSplit: words [0, lbw) in shared memory
+    int nt, q, occ;
+    size_t smem;
+    int64_t cap = 0;  // per-CTA spill / staging capacity (entries)
+    int grid = 0;
+    // this class's disjoint scratch regions (classes run concurrently)
+    int64_t spill_off = 0, stg_off = 0, map_off = 0;
+    cudaStream_t stream = nullptr;  // classes after the first run on their own stream
+    cudaEvent_t done = nullptr;
+};
 
 struct lu_sym {
     int32_t n = 0;
@@ -83,6 +99,7 @@ struct lu_sym {
     uint32_t *gbitmap = nullptr;
     uint32_t *dbitmap = nullptr;
     int64_t gb_stride = 0;
+    int64_t map_words = 0;  // words of the HBM visited / done maps (all classes)
     int32_t *gspill = nullptr;
     int64_t spill_cap = 0;
     unsigned long long *dstats = nullptr;  // [0] row counter, [1..4] count pass, [5..8] emit,
@@ -97,6 +114,7 @@ struct lu_sym {
     int64_t pool_cap = 0;        // entries; -1 = no pool could be allocated
     int64_t *row_off = nullptr;  // [n] pool offset of each staged row, -1 = not staged
     int32_t *unstaged = nullptr; // [n] rows that overflowed the pool / row list for re-traversal
+    std::vector<RowClass> classes;  // Alg. 4 row classes, top (heaviest) first
     std::vector<std::pair<int32_t, int32_t>> staged;  // row ranges staged since the last reset
     // state
     bool scanned = false;
@@ -142,118 +160,174 @@ void free_handle(lu_sym *h)
                     h->stg, h->pool, h->row_off, h->unstaged};
     for (void *b : bufs) dev_free(b, s);
     levelize_free(h->lev, s);
+    for (auto &c : h->classes) {
+        if (c.stream) cudaStreamDestroy(c.stream);
+        if (c.done) cudaEventDestroy(c.done);
+    }
     for (int k = 0; k < kEvN; ++k)
         for (int j = 0; j < 2; ++j)
             if (h->ev[k][j]) cudaEventDestroy(h->ev[k][j]);
     delete h;
 }
 
-int pow2_floor(int x)
-{
-    int p = 1;
-    while (p * 2 <= x) p *= 2;
-    return p;
-}
-
 // ---------------------------------------------------------------- out-of-core planner
-// Paper (L239-243): chunk_size = L / (c n), c = 6 words per vertex per row in flight.
-// Here a row in flight owns: a visited bitmap of n bits (shared memory when it fits, else an
-// HBM slot), two frontier queues (shared memory, spilling to 2 x n int32 in HBM).  The number
-// of rows in flight is the smaller of (resident CTAs) and (scratch budget / HBM bytes per row).
-lu_status plan(lu_sym *h)
+// Paper (L239-243): chunk_size = L / (c n), c = 6 words per vertex per row in flight, and
+// Alg. 4 (L272-277): the scratch a row needs grows with its id, so rows are split into ranges
+// with different chunk sizes.  Here a row in flight is a CTA owning: a visited bitmap (shared
+// memory when it fits, else an HBM slot), a level-1 summary, two shared frontier queues
+// spilling to HBM.  Row classes: rows i < 32*lbw only need words [0, lbw) of the visited map in
+// shared memory (their whole BFS region lies below i; marks above go to the HBM slot), so lower
+// classes fit more rows per SM.  Within a class the CTA size and queue capacity maximise
+// resident threads, then rows in flight; the HBM budget caps rows in flight.
+struct Cfg {
+    int nt, q, occ;
+    size_t smem;
+    long key;
+};
+
+lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out)
 {
-    int sms = 0, smem_sm = 0, smem_optin = 0, smem_res = 0;
-    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device));
-    CK(cudaDeviceGetAttribute(&smem_sm, cudaDevAttrMaxSharedMemoryPerMultiprocessor, h->device));
-    CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->device));
-    CK(cudaDeviceGetAttribute(&smem_res, cudaDevAttrReservedSharedMemoryPerBlock, h->device));
-    const int n = h->n;
-    // visited bitmap in shared memory when it fits next to minimal queues, else HBM slots
-    if (h->opts.flags & LU_F_GLOBAL_BITMAP)
-        h->vis = kVisGlobal;
-    else if (fill2_smem_bytes(n, h->opts.queue_capacity > 0 ? h->opts.queue_capacity : 256,
-                              kVisSmem) <= (size_t)smem_optin)
-        h->vis = kVisSmem;
-    else
-        h->vis = kVisGlobal;
-    h->gb = h->vis == kVisGlobal;
-    // CTA size and shared queue capacity: the traversal is latency-bound, so maximise resident
-    // threads first, then rows in flight (CTAs), then queue capacity (fewer spills).
-    // Frontier levels larger than the queue spill to the CTA's HBM region.
     const int nts[4] = {128, 256, 512, 1024};
     const int qs[4] = {512, 1024, 2048, 4096};
-    int best_nt = 0, best_q = 0, best_occ = 0;
-    long best_key = -1;
+    Cfg best = {0, 0, 0, 0, -1};
     for (int a = 0; a < 4; ++a) {
         const int nt = nts[a];
         if (h->opts.threads_per_row > 0 && nt != h->opts.threads_per_row) continue;
         for (int b = 0; b < 4; ++b) {
-            const int q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : qs[b];
+            int q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : qs[b];
             if (h->opts.queue_capacity > 0 && b > 0) break;
-            const size_t smem = fill2_smem_bytes(n, q < 32 ? 32 : q, h->vis);
+            if (q < 32) q = 32;
+            const size_t smem = fill2_smem_bytes(h->n, smem_words, q);
             if (smem > (size_t)smem_optin) continue;
-            CK(fill2_configure(nt, h->w, h->vis, smem));
+            // the attribute is a cap: set it to the device maximum so that every class sharing
+            // this kernel can launch with its own dynamic shared memory size
+            CK(fill2_configure(nt, h->w, vis, (size_t)smem_optin));
             int occ = 0;
-            CK(fill2_occupancy(nt, h->w, h->vis, smem, &occ));
+            CK(fill2_occupancy(nt, h->w, vis, smem, &occ));
             if (occ < 1) continue;
-            // small matrices: rows are short, prefer small CTAs; large rows want big levels
             const long key = ((long)occ * nt << 24) | ((long)occ << 14) | q;
-            if (key > best_key) {
-                best_key = key;
-                best_nt = nt;
-                best_q = q < 32 ? 32 : q;
-                best_occ = occ;
-            }
+            if (key > best.key) best = Cfg{nt, q, occ, smem, key};
         }
     }
-    if (best_key < 0) {
-        if (h->opts.threads_per_row > 0 && h->opts.threads_per_row != 128 &&
-            h->opts.threads_per_row != 256 && h->opts.threads_per_row != 512 &&
-            h->opts.threads_per_row != 1024)
-            return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512 or 1024 (got %d)",
-                        h->opts.threads_per_row);
-        return fail(LU_ERR_NOMEM, "no resident fill2 configuration (queue_capacity %d)",
-                    h->opts.queue_capacity);
+    *out = best;
+    return LU_OK;
+}
+
+lu_status plan(lu_sym *h)
+{
+    int sms = 0, smem_optin = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device));
+    CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->device));
+    const int n = h->n;
+    const int nw = (int)(((int64_t)n + 31) / 32);
+    const int nw32 = (nw + 31) / 32 * 32;  // whole swizzle groups
+    if (h->opts.threads_per_row > 0 && h->opts.threads_per_row != 128 &&
+        h->opts.threads_per_row != 256 && h->opts.threads_per_row != 512 &&
+        h->opts.threads_per_row != 1024)
+        return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512 or 1024 (got %d)",
+                    h->opts.threads_per_row);
+    // top class: the whole visited map in shared memory, else in HBM
+    Cfg cur;
+    int vis = kVisGlobal, lbw = 0;
+    lu_status st;
+    if (!(h->opts.flags & LU_F_GLOBAL_BITMAP)) {
+        if ((st = best_cfg(h, nw32, kVisSmem, smem_optin, &cur)) != LU_OK) return st;
+        if (cur.key >= 0) {
+            vis = kVisSmem;
+            lbw = nw32;
+        }
     }
-    h->nt = best_nt;
-    h->q = best_q;
-    h->smem = fill2_smem_bytes(n, h->q, h->vis);
-    const int occ = best_occ;
-    (void)smem_res;
-    (void)pow2_floor;
-    int64_t grid = (int64_t)sms * occ;
-    if (h->opts.rows_in_flight > 0 && h->opts.rows_in_flight < grid) grid = h->opts.rows_in_flight;
-    // HBM budget
+    if (vis == kVisGlobal) {
+        if ((st = best_cfg(h, 0, kVisGlobal, smem_optin, &cur)) != LU_OK) return st;
+        if (cur.key < 0)
+            return fail(LU_ERR_NOMEM, "no resident fill2 configuration (queue_capacity %d)",
+                        h->opts.queue_capacity);
+        lbw = nw32;  // for splitting below: start from the full map
+    }
+    // lower row classes (Alg. 4): halve the shared part while that adds rows in flight
+    h->classes.clear();
+    int hi = n;
+    const bool one_class = (h->opts.flags & LU_F_ONE_CLASS) != 0;
+    while (!one_class) {
+        int nl = (lbw / 2 + 31) / 32 * 32;
+        if (nl < 64 || nl >= lbw) break;
+        Cfg c;
+        if ((st = best_cfg(h, nl, kVisSplit, smem_optin, &c)) != LU_OK) return st;
+        if (c.key < 0) {
+            if (vis != kVisGlobal) break;
+            lbw = nl;  // an HBM-resident top class: keep halving until a split map fits
+            continue;
+        }
+        if (c.occ <= cur.occ && !(h->opts.flags & LU_F_FORCE_CLASSES)) break;
+        const int lo = nl * 32 < hi ? nl * 32 : hi;  // rows i < 32*nl fit the smaller map
+        const int sw_words = vis == kVisSmem ? nw32 : (vis == kVisSplit ? lbw : 0);
+        h->classes.push_back(RowClass{lo, hi, vis, sw_words, vis == kVisGlobal ? 0 : sw_words,
+                                      cur.nt, cur.q, cur.occ, cur.smem});
+        hi = lo;
+        vis = kVisSplit;
+        lbw = nl;
+        cur = c;
+    }
+    {
+        const int sw_words = vis == kVisSmem ? nw32 : (vis == kVisSplit ? lbw : 0);
+        h->classes.push_back(RowClass{0, hi, vis, sw_words, vis == kVisGlobal ? 0 : sw_words,
+                                      cur.nt, cur.q, cur.occ, cur.smem});
+    }
+    // HBM budget: per row in flight, frontier spill (2 x cap) + L staging (cap) + done map
+    // (+ the HBM visited slot); cap = rows of the class (a row's frontier and L part lie below i)
     size_t free_b = 0, total_b = 0;
     CK(cudaMemGetInfo(&free_b, &total_b));
-    uint64_t budget = h->opts.scratch_budget_bytes ? h->opts.scratch_budget_bytes
-                                                   : (uint64_t)(0.85 * (double)free_b);
-    const int64_t nw = ((int64_t)n + 31) / 32;
-    h->gb_stride = (nw + 31) & ~(int64_t)31;  // 128 B aligned slots
-    h->spill_cap = n > 0 ? n : 1;
-    h->staging = !(h->opts.flags & LU_F_TWO_PASS);
+    const uint64_t budget = h->opts.scratch_budget_bytes ? h->opts.scratch_budget_bytes
+                                                         : (uint64_t)(0.85 * (double)free_b);
     h->budget = budget;
-    const uint64_t per_row = (uint64_t)(h->staging ? 3 : 2) * h->spill_cap * 4 +
-                             (uint64_t)(h->gb ? 2 : 1) * h->gb_stride * 4;
-    const uint64_t fit = budget / per_row;
-    if (fit < 1)
-        return fail(LU_ERR_NOMEM, "scratch budget %llu B < one row's scratch %llu B",
-                    (unsigned long long)budget, (unsigned long long)per_row);
-    if ((uint64_t)grid > fit) grid = (int64_t)fit;
-    if (grid < 1) grid = 1;
-    h->grid = (int)grid;
-    lu_status st = dalloc(h, &h->gspill, (size_t)2 * h->spill_cap * h->grid);
-    if (st != LU_OK) return st;
-    if (h->gb) {
-        st = dalloc(h, &h->gbitmap, (size_t)h->gb_stride * h->grid);
-        if (st != LU_OK) return st;
+    h->staging = !(h->opts.flags & LU_F_TWO_PASS);
+    h->gb_stride = nw32;
+    const bool need_hbm_map = h->classes.front().vis != kVisSmem || h->classes.size() > 1;
+    uint64_t need_spill = 0, need_stg = 0, need_map = 0;
+    int max_grid = 0;
+    for (auto &c : h->classes) {
+        const int64_t cap = c.hi > 0 ? c.hi : 1;
+        c.cap = cap;
+        const uint64_t per_row = (uint64_t)(h->staging ? 3 : 2) * cap * 4 +
+                                 (uint64_t)(need_hbm_map ? 2 : 1) * h->gb_stride * 4;
+        const uint64_t fit = budget / per_row;
+        if (fit < 1)
+            return fail(LU_ERR_NOMEM, "scratch budget %llu B < one row's scratch %llu B",
+                        (unsigned long long)budget, (unsigned long long)per_row);
+        int64_t grid = (int64_t)sms * c.occ;
+        if (h->opts.rows_in_flight > 0 && h->opts.rows_in_flight < grid)
+            grid = h->opts.rows_in_flight;
+        if ((uint64_t)grid > fit) grid = (int64_t)fit;
+        c.grid = (int)(grid < 1 ? 1 : grid);
+        c.spill_off = (int64_t)need_spill;
+        c.stg_off = (int64_t)need_stg;
+        c.map_off = (int64_t)need_map;
+        need_spill += (uint64_t)2 * cap * c.grid;
+        need_stg += (uint64_t)cap * c.grid;
+        need_map += (uint64_t)h->gb_stride * c.grid;
+        max_grid = std::max(max_grid, c.grid);
     }
-    if ((st = dalloc(h, &h->dbitmap, (size_t)h->gb_stride * h->grid)) != LU_OK) return st;
+    h->grid = max_grid;
+    h->map_words = (int64_t)need_map;
+    if ((st = dalloc(h, &h->gspill, need_spill)) != LU_OK) return st;
+    if (need_hbm_map && (st = dalloc(h, &h->gbitmap, need_map)) != LU_OK) return st;
+    if ((st = dalloc(h, &h->dbitmap, need_map)) != LU_OK) return st;
+    for (size_t k = 0; k < h->classes.size(); ++k) {
+        CK(cudaEventCreateWithFlags(&h->classes[k].done, cudaEventDisableTiming));
+        if (k > 0) CK(cudaStreamCreateWithFlags(&h->classes[k].stream, cudaStreamNonBlocking));
+    }
     if ((st = dalloc(h, &h->unstaged, (size_t)n)) != LU_OK) return st;
     if (h->staging) {
-        if ((st = dalloc(h, &h->stg, (size_t)h->spill_cap * h->grid)) != LU_OK) return st;
+        if ((st = dalloc(h, &h->stg, need_stg)) != LU_OK) return st;
         if ((st = dalloc(h, &h->row_off, (size_t)n)) != LU_OK) return st;
     }
+    // summary fields (the top class)
+    const RowClass &top = h->classes.front();
+    h->vis = top.vis;
+    h->gb = top.vis == kVisGlobal;
+    h->nt = top.nt;
+    h->q = top.q;
+    h->smem = top.smem;
     return LU_OK;
 }
 
@@ -272,42 +346,34 @@ void ev_end(lu_sym *h, int k, cudaStream_t s)
     h->ev_used[k] = true;
 }
 
+// One traversal pass over rows [rb, re) (or row_list): one launch per row class, top class
+// (heaviest rows) first, as Alg. 4 launches each part in turn.
 lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_count,
                    const int64_t *rp_lu, int32_t *ci_lu, cudaStream_t s,
                    const int32_t *row_list = nullptr, int32_t list_len = 0)
 {
     const bool emit = mode == kEmit;
     unsigned long long *st = h->dstats + (emit ? 5 : 1);
-    CK(cudaMemsetAsync(h->dstats, 0, sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(st, 0, sizeof(unsigned long long) * kStatCount, s));
-    if (h->gb)
-        CK(cudaMemsetAsync(h->gbitmap, 0, sizeof(uint32_t) * (size_t)h->gb_stride * h->grid, s));
-    CK(cudaMemsetAsync(h->dbitmap, 0, sizeof(uint32_t) * (size_t)h->gb_stride * h->grid, s));
+    if (h->gbitmap) CK(cudaMemsetAsync(h->gbitmap, 0, sizeof(uint32_t) * h->map_words, s));
+    CK(cudaMemsetAsync(h->dbitmap, 0, sizeof(uint32_t) * h->map_words, s));
+    CK(cudaMemsetAsync(h->dstats + kSlotClassCounter, 0,
+                       sizeof(unsigned long long) * h->classes.size(), s));
+    if (h->row_prof && mode != kEmit && !row_list)
+        CK(cudaMemsetAsync(h->row_prof + 4 * (size_t)rb, 0,
+                           sizeof(int64_t) * 4 * (size_t)(re - rb), s));
     Fill2Params p;
     p.n = h->n;
     p.rp = h->rp;
     p.ci = h->ci;
     p.ell = h->ell;
-    p.row_begin = rb;
-    p.row_end = re;
     p.descending = (h->opts.flags & LU_F_ASCENDING) ? 0 : 1;
     p.fill_count = fill_count;
     p.rp_lu = rp_lu;
     p.ci_lu = ci_lu;
-    p.gbitmap = h->gbitmap;
-    p.dbitmap = h->dbitmap;
     p.gbitmap_stride = h->gb_stride;
-    p.gspill = h->gspill;
-    p.spill_cap = h->spill_cap;
-    p.nw = (int32_t)((((int64_t)h->n + 31) / 32 + 31) / 32 * 32);  // whole swizzle groups
-    p.sw = (p.nw + 31) / 32;
-    p.q = h->q;
-    p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : h->q;
-    p.row_counter = h->dstats;
+    p.sw = (int32_t)((((int64_t)h->n + 31) / 32 + 31) / 32);
     p.stats = st;
-    p.row_list = row_list;
-    p.list_len = list_len;
-    p.stg = h->stg;
     p.pool = h->pool;
     p.pool_cap = h->pool_cap;
     p.row_off = h->row_off;
@@ -315,14 +381,48 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     p.unstaged = h->unstaged;
     p.unstaged_cnt = h->dstats + kSlotUnstaged;
     p.row_prof = h->row_prof;
-    if (h->row_prof && mode != kEmit)
-        CK(cudaMemsetAsync(h->row_prof + 4 * (size_t)rb, 0, sizeof(int64_t) * 4 * (size_t)(re - rb), s));
-    int rows = row_list ? list_len : re - rb;
-    int grid = h->grid;
-    if (grid > rows) grid = rows;
-    if (grid < 1) return LU_OK;
-    CK(fill2_launch(p, h->nt, h->w, mode, h->vis, grid, h->smem, s));
-    h->launches += 1;
+    // classes run concurrently: the top class on s, the others on their own streams forked
+    // from s, so lower-class CTAs take over SMs as soon as top-class CTAs drain
+    bool forked = false;
+    for (size_t k = 0; k < h->classes.size(); ++k) {
+        const RowClass &c = h->classes[k];
+        // a row list (rows that did not fit the staging pool) runs in the top class only
+        if (row_list && k > 0) break;
+        const int32_t lo = row_list ? 0 : std::max(rb, c.lo), hi = row_list ? 0 : std::min(re, c.hi);
+        const int rows = row_list ? list_len : hi - lo;
+        if (rows <= 0) continue;
+        cudaStream_t cs = s;
+        if (k > 0) {
+            if (!forked) {
+                CK(cudaEventRecord(h->classes[0].done, s));
+                forked = true;
+            }
+            cs = c.stream;
+            CK(cudaStreamWaitEvent(cs, h->classes[0].done, 0));
+        }
+        p.row_begin = lo;
+        p.row_end = hi;
+        p.row_list = row_list;
+        p.list_len = list_len;
+        p.spill_cap = c.cap;
+        p.gspill = h->gspill + c.spill_off;
+        p.stg = h->stg ? h->stg + c.stg_off : nullptr;
+        p.gbitmap = h->gbitmap ? h->gbitmap + c.map_off : nullptr;
+        p.dbitmap = h->dbitmap + c.map_off;
+        p.row_counter = h->dstats + kSlotClassCounter + k;
+        p.nw = c.smem_words;
+        p.lbw = c.lbw;
+        p.q = c.q;
+        p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : c.q;
+        const int grid = c.grid < rows ? c.grid : rows;
+        CK(fill2_launch(p, c.nt, h->w, mode, c.vis, grid, c.smem, cs));
+        h->launches += 1;
+    }
+    if (forked)  // join
+        for (size_t k = 1; k < h->classes.size(); ++k) {
+            CK(cudaEventRecord(h->classes[k].done, h->classes[k].stream));
+            CK(cudaStreamWaitEvent(s, h->classes[k].done, 0));
+        }
     return LU_OK;
 }
 
@@ -418,10 +518,10 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
     if (cudaEventCreate(&t0) != cudaSuccess || cudaEventCreate(&t1) != cudaSuccess)
         return bail(fail(LU_ERR_CUDA, "cudaEventCreate failed"));
     cudaEventRecord(t0, s);
-    if ((st = dalloc(h, &h->dstats, 16)) != LU_OK) return bail(st);
+    if ((st = dalloc(h, &h->dstats, 32)) != LU_OK) return bail(st);
     if ((st = dalloc(h, &h->dbad, 2)) != LU_OK) return bail(st);
     if ((st = dalloc(h, &h->scan_blk, scan_scratch_elems(n))) != LU_OK) return bail(st);
-    cudaMemsetAsync(h->dstats, 0, 16 * sizeof(unsigned long long), s);
+    cudaMemsetAsync(h->dstats, 0, 32 * sizeof(unsigned long long), s);
     // S1: validate A
     {
         cudaError_t e = validate_csr(n, nnz_a, d_row_ptr, d_col_idx, h->dbad, s);
@@ -683,6 +783,7 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
     h->stats.threads_per_row = h->nt;
     h->stats.smem_bytes_per_row = (int32_t)h->smem;
     h->stats.visited_in_smem = h->gb ? 0 : 1;
+    h->stats.row_classes = (int32_t)h->classes.size();
     h->stats.ell_width = h->w;
     h->stats.queue_capacity = h->q;
     h->stats.kernel_launches = h->launches;

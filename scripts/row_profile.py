@@ -35,3 +35,5 @@ for q in (10, 100, 1000):
     print(f"top {q} rows: {cyc[order[:q]].sum() / cyc.sum() * 100:.1f}% of cycles")
 for r in order[:10]:
     print("row", r, "cycles %.3e sv %d bfs %d windows %d count %d" % (P[r, 0], P[r, 1], P[r, 2], P[r, 3], fc[r]))
+print("sum(row cycles)/SMs = %.3e cycles (%.0f ms at 1.9 GHz); max row %.3e cycles (%.0f ms)" % (
+    cyc.sum() / 148, cyc.sum() / 148 / 1.9e6, cyc.max(), cyc.max() / 1.9e6))

@@ -143,6 +143,9 @@ KNOBS = [
     dict(flags=lu.F_NO_CONTRACT | lu.F_NO_PRUNE | lu.F_KAHN_WIDE_ONLY),
     dict(flags=lu.F_TWO_PASS),                       # Alg. 3 as printed: emit re-traverses
     dict(flags=lu.F_TWO_PASS, queue_capacity=64),
+    dict(flags=lu.F_ONE_CLASS), dict(flags=lu.F_ONE_CLASS | lu.F_GLOBAL_BITMAP),
+    dict(flags=lu.F_FORCE_CLASSES), dict(flags=lu.F_FORCE_CLASSES | lu.F_GLOBAL_BITMAP),
+    dict(flags=lu.F_FORCE_CLASSES, queue_capacity=32, rows_in_flight=7),
     dict(pool_bytes=4096),                           # pool overflow: most rows re-traversed
     dict(pool_bytes=200_000),                        # partial staging
 ]
@@ -160,6 +163,15 @@ def test_pool_overflow_falls_back_to_traversal():
     assert 0 < g["stats"]["rows_retraversed"] < 4096
     g = check(*gen.circuit(64, 5), tag="pool-full")
     assert g["stats"]["rows_retraversed"] == 0 and g["stats"]["pool_bytes"] > 0
+
+
+def test_row_classes():
+    """Alg. 4 row classes (split visited map: low words shared, high words in HBM) on inputs
+    large enough for several classes; bit-exact against the oracle."""
+    for rp, ci in (gen.circuit(128, 3), gen.lap3d(20), gen.random_pattern(30000, 2.0, seed=11)):
+        g = check(rp, ci, tag="classes", flags=lu.F_FORCE_CLASSES)
+        assert g["stats"]["row_classes"] >= 3
+        g = check(rp, ci, tag="classes+two-pass", flags=lu.F_FORCE_CLASSES | lu.F_TWO_PASS)
 
 
 def test_spills_are_exercised():
