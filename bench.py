@@ -57,15 +57,21 @@ def parse():
 
 
 # --------------------------------------------------------------------------- work units
-def work_units(rp):
-    """Method work of one traversal (reading R24).
-
-    TE = sum_i row_ptr[i+1] and SV = n(n-1)/2 are exact on connected natural-order grids
-    (pinned in tests/test_oracle_pins.py); for other inputs they are upper bounds."""
+def work_units(rp, cfg=None):
+    """Method work of one traversal (reading R24): TE traversed edges, SV
+    scanned vertices.  Exact values per config come from tests/golden/work_units.json
+    (scripts/work_units.py: oracle counts, or the pinned grid closed forms TE = sum
+    row_ptr[i+1], SV = n(n-1)/2); without an entry the grid closed forms are used (upper
+    bounds for other inputs)."""
     n = len(rp) - 1
-    te = int(rp[1:].sum())
-    sv = n * (n - 1) // 2
-    return te, sv
+    try:
+        wu = json.load(open(os.path.join(ROOT, "tests", "golden", "work_units.json")))
+        e = wu.get(f"cfg{cfg}")
+        if e and e["n"] == n and e["nnz_a"] == int(rp[-1]):
+            return int(e["te"]), int(e["sv"])
+    except Exception:
+        pass
+    return int(rp[1:].sum()), n * (n - 1) // 2
 
 
 def alg_bytes_per_pass(te, sv, n, nnz_lu, emit):
@@ -180,7 +186,7 @@ def run_reference(args, rank, world):
         return
     name, rp, ci = gen.config(args.config)
     n = len(rp) - 1
-    te, _ = work_units(rp)
+    te, _ = work_units(rp, args.config)
     stride = args.cpu_sample_stride or auto_stride(n, te)
     times, entries = [], None
     for k in range(args.warmup + args.steps):
@@ -220,7 +226,7 @@ def run_ours(args, rank, world, local_rank):
     stream = torch.cuda.current_stream()
     name, rp_np, ci_np = gen.config(args.config)
     n = len(rp_np) - 1
-    te, sv = work_units(rp_np)
+    te, sv = work_units(rp_np, args.config)
     rp = torch.from_numpy(rp_np).to(dev)
     ci = torch.from_numpy(ci_np).to(dev)
     sym_opts = dict(flags=args.flags, threads_per_row=args.threads_per_row,

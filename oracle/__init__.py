@@ -41,7 +41,7 @@ def _load():
     if _lib is None:
         lib = ctypes.CDLL(build())
         P = ctypes.c_void_p
-        lib.oracle_fill2.argtypes = [ctypes.c_int32, P, P, P, ctypes.c_int64, P, P, P, P,
+        lib.oracle_fill2.argtypes = [ctypes.c_int32, P, P, P, ctypes.c_int64, P, P, P, P, P,
                                      ctypes.c_int]
         lib.oracle_fill2.restype = ctypes.c_int
         lib.oracle_kahn.argtypes = [ctypes.c_int32, P, P, ctypes.c_int, P]
@@ -58,7 +58,8 @@ def fill2(row_ptr, col_idx, rows=None, emit: bool = True, threads: int = 0):
     """Symbolic factorization by Algorithm 1, rows independent.
 
     rows=None computes every row; otherwise only the listed rows (sampled parity).
-    Returns dict(counts=int32[m], te=int64[m], row_ptr=int64[m+1], col_idx=int32[nnz] | None)
+    Returns dict(counts=int32[m], te=int64[m], sv=int64[m], row_ptr=int64[m+1],
+    col_idx=int32[nnz] | None); te / sv = traversed edges / scanned vertices per row.
     where m = number of computed rows and row_ptr/col_idx is the CSR of those rows (Alg. 3:
     count, prefix sum, allocate, emit).
     """
@@ -74,7 +75,8 @@ def fill2(row_ptr, col_idx, rows=None, emit: bool = True, threads: int = 0):
         m = r.size
     counts = np.zeros(m, dtype=np.int32)
     te = np.zeros(m, dtype=np.int64)
-    rc = lib.oracle_fill2(n, _ptr(rp), _ptr(ci), _ptr(r), m, _ptr(counts), _ptr(te),
+    sv = np.zeros(m, dtype=np.int64)
+    rc = lib.oracle_fill2(n, _ptr(rp), _ptr(ci), _ptr(r), m, _ptr(counts), _ptr(te), _ptr(sv),
                           None, None, threads)
     if rc != 0:
         raise MemoryError("oracle_fill2 allocation failed")
@@ -83,11 +85,11 @@ def fill2(row_ptr, col_idx, rows=None, emit: bool = True, threads: int = 0):
     cols = None
     if emit:
         cols = np.empty(int(out_ptr[-1]), dtype=np.int32)  # line 8: allocate
-        rc = lib.oracle_fill2(n, _ptr(rp), _ptr(ci), _ptr(r), m, None, None,
+        rc = lib.oracle_fill2(n, _ptr(rp), _ptr(ci), _ptr(r), m, None, None, None,
                               _ptr(out_ptr), _ptr(cols), threads)
         if rc != 0:
             raise MemoryError("oracle_fill2 allocation failed")
-    return {"counts": counts, "te": te, "row_ptr": out_ptr, "col_idx": cols}
+    return {"counts": counts, "te": te, "sv": sv, "row_ptr": out_ptr, "col_idx": cols}
 
 
 def levels(row_ptr_lu, col_idx_lu, rule: str = "u"):

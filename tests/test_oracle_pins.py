@@ -117,8 +117,9 @@ def test_closed_form_2d(k):
     r = oracle.fill2(rp, ci)
     assert int(r["row_ptr"][-1]) == pins.nnz_2d(k)
     assert pins.csr_rows(r["row_ptr"], r["col_idx"]) == pins.closed_form_2d(k)
-    # TE (R24): every vertex below row i is scanned once -> TE(i) = row_ptr_A[i+1]
+    # TE (R24): every vertex below row i is scanned once -> TE(i) = row_ptr_A[i+1], SV(i) = i
     assert np.array_equal(r["te"], rp[1:])
+    assert np.array_equal(r["sv"], np.arange(len(rp) - 1))
 
 
 @pytest.mark.parametrize("k", [2, 3, 4, 5, 6, 7, 8])
@@ -128,6 +129,7 @@ def test_closed_form_3d(k):
     assert int(r["row_ptr"][-1]) == pins.nnz_3d(k)
     assert pins.csr_rows(r["row_ptr"], r["col_idx"]) == pins.closed_form_3d(k)
     assert np.array_equal(r["te"], rp[1:])
+    assert np.array_equal(r["sv"], np.arange(len(rp) - 1))
 
 
 def test_closed_form_counts_cfg2():
