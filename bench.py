@@ -428,6 +428,7 @@ def run_ours(args, rank, world, local_rank):
         "clocks": clk.summary(),
         "plan": {k: stats[k] for k in ("rows_in_flight", "threads_per_row", "smem_bytes_per_row",
                                         "visited_in_smem", "ell_width", "queue_capacity",
+                                        "row_classes", "pool_bytes", "rows_retraversed",
                                         "levelize_wide_levels", "levelize_narrow_levels",
                                         "spills")},
     }

@@ -181,6 +181,16 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
                       const int32_t *d_col_idx_lu, int32_t dep_rule, int32_t *d_level,
                       int32_t *num_levels, void *stream);
 
+/*
+ * Level-grouped column schedule (the form of Fig. 1(d), L72-80, consumed level by level by the
+ * numeric phase, L206-208): from d_level[n] (levels in [0, num_levels), e.g. lu_levelize's
+ * output) write d_level_ptr[num_levels+1] (int64) and d_level_cols[n] (int32) such that the
+ * columns of level l are d_level_cols[d_level_ptr[l] .. d_level_ptr[l+1]), ascending (R15).
+ * Synchronises.  LU_ERR_ARG on null pointers or num_levels < 1 with n > 0.
+ */
+lu_status lu_level_schedule(int32_t n, const int32_t *d_level, int32_t num_levels,
+                            int64_t *d_level_ptr, int32_t *d_level_cols, void *stream);
+
 /* Copy the handle's statistics to *out (host). */
 lu_status lu_sym_get_stats(const lu_sym *h, lu_sym_stats *out);
 

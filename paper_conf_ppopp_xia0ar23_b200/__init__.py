@@ -26,7 +26,7 @@ import torch
 from .parallel import (assemble_counts, assemble_pattern, partition_rows,  # noqa: F401
                        row_cost_upper_bound)
 
-__all__ = ["Symbolic", "LuSymError", "levelize", "load_library", "library_path",
+__all__ = ["Symbolic", "LuSymError", "levelize", "level_schedule", "load_library", "library_path",
            "partition_rows", "assemble_counts", "assemble_pattern", "symbolic_distributed",
            "row_cost_upper_bound", "DEP_U", "DEP_GLU3"]
 
@@ -78,7 +78,8 @@ _lib = None
 
 EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sym_count",
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
-            "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile"]
+            "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile",
+            "lu_level_schedule"]
 
 
 def library_path() -> str:
@@ -106,6 +107,8 @@ def load_library():
     lib.lu_sym_get_stats.argtypes = [P, P]
     lib.lu_sym_destroy.argtypes = [P]
     lib.lu_sym_set_row_profile.argtypes = [P, P]
+    lib.lu_level_schedule.argtypes = [I32, P, I32, P, P, P]
+    lib.lu_level_schedule.restype = I32
     lib.lu_sym_set_row_profile.restype = I32
     lib.lu_status_str.argtypes = [I32]
     lib.lu_status_str.restype = ctypes.c_char_p
@@ -286,6 +289,20 @@ def levelize(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, rule: str = "u"
                            _dev(level, torch.int32, "level") if n else None, ctypes.byref(nl),
                            _stream_ptr(stream)))
     return level, int(nl.value)
+
+
+def level_schedule(level: torch.Tensor, num_levels: int, stream=None):
+    """Columns grouped by level (Fig. 1(d)): (level_ptr int64[num_levels+1], level_cols int32[n])
+    on the device; the columns of level l are level_cols[level_ptr[l]:level_ptr[l+1]], ascending."""
+    n = int(level.numel())
+    dev = level.device
+    level_ptr = torch.empty(num_levels + 1, dtype=torch.int64, device=dev)
+    level_cols = torch.empty(max(n, 1), dtype=torch.int32, device=dev)[:n]
+    _check(load_library().lu_level_schedule(
+        n, _dev(level, torch.int32, "level") if n else None, num_levels,
+        _dev(level_ptr, torch.int64, "level_ptr"),
+        ctypes.c_void_p(level_cols.data_ptr()) if n else None, _stream_ptr(stream)))
+    return level_ptr, level_cols
 
 
 def symbolic_distributed(row_ptr: torch.Tensor, col_idx: torch.Tensor, group=None,

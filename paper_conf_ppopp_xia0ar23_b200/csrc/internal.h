@@ -89,6 +89,8 @@ cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, in
 cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,
                         cudaStream_t s);
 size_t scan_scratch_elems(int32_t n);
+cudaError_t count_far_rows(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
+                           unsigned long long *d_cnt, cudaStream_t s);
 
 // place_kernels.cu — symbolic_2 for staged rows: copy pool rows to their CSR slots
 cudaError_t place_rows(int32_t row_begin, int32_t row_end, const int64_t *rp_lu,
@@ -97,6 +99,10 @@ cudaError_t place_rows(int32_t row_begin, int32_t row_end, const int64_t *rp_lu,
 // rows of [row_begin, row_end) with row_off < 0 -> list[0..*cnt)
 cudaError_t collect_unstaged(int32_t row_begin, int32_t row_end, const int64_t *row_off,
                              int32_t *list, unsigned long long *cnt, cudaStream_t s);
+
+// schedule_kernels.cu — columns grouped by level (Fig. 1(d) form)
+cudaError_t level_schedule(int32_t n, const int32_t *level, int32_t num_levels,
+                           int64_t *level_ptr, int32_t *level_cols, cudaStream_t s);
 
 // levelize_kernels.cu
 struct LevelizeScratch {

@@ -259,6 +259,17 @@ lu_status plan(lu_sym *h)
             continue;
         }
         if (c.occ <= cur.occ && !(h->opts.flags & LU_F_FORCE_CLASSES)) break;
+        if (!(h->opts.flags & LU_F_FORCE_CLASSES)) {
+            // rows of the new class with neighbours above its shared part would send their
+            // pattern marks to HBM; split only when that is rare (grids: rows within k of the
+            // boundary; circuits with hubs at the end: most rows)
+            unsigned long long far = 0;
+            CK(count_far_rows(n, h->rp, h->ci, nl * 32, h->dstats + 14, h->stream));
+            CK(cudaMemcpyAsync(&far, h->dstats + 14, 8, cudaMemcpyDeviceToHost, h->stream));
+            CK(cudaStreamSynchronize(h->stream));
+            const int rows = nl * 32 < n ? nl * 32 : n;
+            if (far * 20 > (unsigned long long)rows) break;
+        }
         const int lo = nl * 32 < hi ? nl * 32 : hi;  // rows i < 32*nl fit the smaller map
         const int sw_words = vis == kVisSmem ? nw32 : (vis == kVisSplit ? lbw : 0);
         h->classes.push_back(RowClass{lo, hi, vis, sw_words, vis == kVisGlobal ? 0 : sw_words,
@@ -752,6 +763,20 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
         h->stats.levelize_narrow_levels = info.narrow_rounds;
         h->stats.levelize_rank_rounds = info.rank_rounds;
     }
+    return LU_OK;
+}
+
+lu_status lu_level_schedule(int32_t n, const int32_t *d_level, int32_t num_levels,
+                            int64_t *d_level_ptr, int32_t *d_level_cols, void *stream)
+{
+    g_err.clear();
+    if (n < 0 || num_levels < 0) return fail(LU_ERR_ARG, "negative size");
+    if (!d_level_ptr || (n > 0 && (!d_level || !d_level_cols)))
+        return fail(LU_ERR_ARG, "null pointer");
+    if (n > 0 && num_levels < 1) return fail(LU_ERR_ARG, "num_levels must be >= 1 when n > 0");
+    cudaStream_t s = (cudaStream_t)stream;
+    CK(level_schedule(n, d_level, num_levels, d_level_ptr, d_level_cols, s));
+    CK(cudaStreamSynchronize(s));
     return LU_OK;
 }
 

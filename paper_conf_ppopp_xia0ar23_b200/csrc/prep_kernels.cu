@@ -106,6 +106,20 @@ __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int
     if constexpr (W == 8) dst[1] = make_int4(out[4], out[5], out[6], out[7]);
 }
 
+// rows i < bound whose largest column is >= bound (their marks would leave a split map)
+__global__ void k_count_far(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
+                            unsigned long long *cnt)
+{
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    bool far = false;
+    if (i < n && i < bound) {
+        const int64_t b = rp[i + 1];
+        far = b > rp[i] && ci[b - 1] >= bound;
+    }
+    const unsigned m = __ballot_sync(kFull, far);
+    if ((threadIdx.x & 31) == 0 && m) atomicAdd(cnt, (unsigned long long)__popc(m));
+}
+
 // ---------------------------------------------------------------- scan (int32 -> int64)
 constexpr int kScanNT = 1024;
 constexpr int kScanItems = 4;
@@ -220,6 +234,16 @@ cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, in
         k_build_ell<4><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
     else
         k_build_ell<8><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
+    return cudaGetLastError();
+}
+
+cudaError_t count_far_rows(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
+                           unsigned long long *d_cnt, cudaStream_t s)
+{
+    cudaError_t e = cudaMemsetAsync(d_cnt, 0, sizeof(unsigned long long), s);
+    const int rows = bound < n ? bound : n;
+    if (e != cudaSuccess || rows <= 0) return e;
+    k_count_far<<<(rows + 255) / 256, 256, 0, s>>>(n, rp, ci, bound, d_cnt);
     return cudaGetLastError();
 }
 

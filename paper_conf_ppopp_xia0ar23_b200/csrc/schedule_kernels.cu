@@ -1,0 +1,62 @@
+// Level-grouped column schedule: the columns of each level, the form of
+// PAPER.md Fig. 1(d) (L72-80, "Column ids for different levels") that the numeric phase's
+// level-by-level launches consume (L206-208).  level_ptr[l] .. level_ptr[l+1] delimit the
+// columns of level l in level_cols, ascending within a level (reading R15).  Not on the hot
+// path: a stable radix sort of (level, column) pairs from CUB does the grouping.
+#include "internal.h"
+
+#include <cub/device/device_radix_sort.cuh>
+
+namespace lusym {
+namespace {
+
+__global__ void k_iota(int32_t n, int32_t *v)
+{
+    const int j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < n) v[j] = j;
+}
+
+// level_ptr[l] = first position of level l in the sorted keys (keys sorted ascending)
+__global__ void k_level_ptr(int32_t n, const int32_t *sorted_level, int32_t num_levels,
+                            int64_t *level_ptr)
+{
+    const int j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j >= n) return;
+    const int l = sorted_level[j];
+    const int prev = j ? sorted_level[j - 1] : -1;
+    for (int k = prev + 1; k <= l; ++k) level_ptr[k] = j;  // levels prev+1..l start here
+    if (j == n - 1)
+        for (int k = l + 1; k <= num_levels; ++k) level_ptr[k] = n;
+}
+
+}  // namespace
+
+cudaError_t level_schedule(int32_t n, const int32_t *level, int32_t num_levels,
+                           int64_t *level_ptr, int32_t *level_cols, cudaStream_t s)
+{
+    if (n <= 0) return cudaMemsetAsync(level_ptr, 0, sizeof(int64_t) * (num_levels + 1), s);
+    int32_t *keys_out = nullptr, *vals_in = nullptr;
+    void *tmp = nullptr;
+    size_t tmp_bytes = 0;
+    int bits = 1;
+    while ((1ll << bits) <= num_levels) ++bits;
+    cudaError_t e = cub::DeviceRadixSort::SortPairs(nullptr, tmp_bytes, level, keys_out, vals_in,
+                                                    level_cols, n, 0, bits, s);
+    if (e != cudaSuccess) return e;
+    if ((e = dev_alloc((void **)&keys_out, sizeof(int32_t) * n, s)) != cudaSuccess) return e;
+    if ((e = dev_alloc((void **)&vals_in, sizeof(int32_t) * n, s)) != cudaSuccess) goto out;
+    if ((e = dev_alloc(&tmp, tmp_bytes, s)) != cudaSuccess) goto out;
+    k_iota<<<(n + 255) / 256, 256, 0, s>>>(n, vals_in);
+    e = cub::DeviceRadixSort::SortPairs(tmp, tmp_bytes, level, keys_out, vals_in, level_cols, n, 0,
+                                        bits, s);
+    if (e != cudaSuccess) goto out;
+    k_level_ptr<<<(n + 255) / 256, 256, 0, s>>>(n, keys_out, num_levels, level_ptr);
+    e = cudaGetLastError();
+out:
+    dev_free(keys_out, s);
+    dev_free(vals_in, s);
+    dev_free(tmp, s);
+    return e;
+}
+
+}  // namespace lusym

@@ -174,6 +174,32 @@ def test_row_classes():
         g = check(rp, ci, tag="classes+two-pass", flags=lu.F_FORCE_CLASSES | lu.F_TWO_PASS)
 
 
+def test_level_schedule():
+    """Fig. 1(d) form: columns grouped by level, ascending within each level."""
+    import os
+    A, fills, table = pins.read_fig1_golden(
+        os.path.join(os.path.dirname(__file__), "golden", "fig1_fixture.txt"))
+    R = [r for r, cs in A.items() for _ in cs]
+    C = [c for r, cs in A.items() for c in cs]
+    cases = [gen.csr_from_edges(10, R, C), gen.circuit(48, 2), gen.lap2d(12),
+             gen.random_pattern(500, 2.0, seed=3)]
+    d = dev()
+    for k, (rp, ci) in enumerate(cases):
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+        fc, rp_lu, ci_lu = h.run()
+        lv, nl = h.levelize(rp_lu, ci_lu, "u")
+        ptr, cols = lu.level_schedule(lv, nl)
+        ptr, cols, lvh = ptr.cpu().numpy(), cols.cpu().numpy(), lv.cpu().numpy()
+        assert ptr[0] == 0 and ptr[-1] == len(rp) - 1 and np.all(np.diff(ptr) > 0)
+        for l in range(nl):
+            seg = cols[ptr[l]:ptr[l + 1]]
+            assert np.array_equal(seg, np.sort(np.nonzero(lvh == l)[0]))
+        if k == 0:   # the printed table, 1-based in the paper
+            got = {l: (cols[ptr[l]:ptr[l + 1]] + 1).tolist() for l in range(nl)}
+            assert got == {0: [1, 2, 3, 6, 7], 1: [4, 5], 2: [8], 3: [9], 4: [10]}
+        h.close()
+
+
 def test_spills_are_exercised():
     g = check(*gen.lap3d(12), tag="spill", queue_capacity=32)
     assert g["stats"]["spills"] > 0
