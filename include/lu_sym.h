@@ -83,7 +83,7 @@ typedef struct {
     int32_t threads_per_row;       /* CTA size per row in flight; 0 => planner (128..1024)   */
     int32_t rows_in_flight;        /* 0 => planner (all resident CTAs); > 0 caps it          */
     int32_t queue_capacity;        /* shared-memory frontier entries per buffer; 0 => planner */
-    int32_t ell_width;             /* traversal adjacency width 4 or 8; 0 => planner         */
+    int32_t ell_width;             /* traversal adjacency slots 4, 6 or 8; 0 => planner     */
     uint64_t pool_bytes;           /* HBM staging pool for the rows found by lu_sym_count, so
                                       lu_sym_emit places them instead of re-traversing;
                                       0 => min(32 GiB, what the budget leaves)              */

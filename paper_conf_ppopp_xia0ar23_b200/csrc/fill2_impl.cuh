@@ -45,6 +45,7 @@ struct Hdr {
     int cnt[3];
     int pad;
     long long stage_off;
+    unsigned long long te, sv, spills;  // statistics of this CTA (thread 0 / shared atomics)
     int scan[40];
 };
 static_assert(sizeof(Hdr) <= kHdrBytes, "header too large");
@@ -108,10 +109,40 @@ __device__ __forceinline__ bool in_smem(const VisMap<VIS> &m, int w)
     return w < m.lbw;
 }
 
+// The shared visited words sit at a constant offset of the CTA's shared window: dynamic shared
+// memory starts right after the 1 KB system reservation (checked at kernel start, see
+// check_smem_base), then the header.  Addressing them as [4*word + immediate] keeps the window
+// base out of the registers of the slot loop (at 32 registers/thread the compiler would
+// otherwise rematerialise it for every neighbour).
+constexpr uint32_t kDynSmemBase = 0x400;
+constexpr uint32_t kBmShared = kDynSmemBase + kHdrBytes;
+
+__device__ __forceinline__ uint32_t lds_bm(int pw)
+{
+    uint32_t v;
+    asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(v) : "r"(pw * 4), "n"(kBmShared) : "memory");
+    return v;
+}
+
+__device__ __forceinline__ uint32_t atom_or_bm(int pw, uint32_t b)
+{
+    uint32_t old;
+    asm volatile("atom.shared.or.b32 %0, [%1+%2], %3;"
+                 : "=r"(old)
+                 : "r"(pw * 4), "n"(kBmShared), "r"(b)
+                 : "memory");
+    return old;
+}
+
+__device__ __forceinline__ void check_smem_base(const unsigned char *smem)
+{
+    if (threadIdx.x == 0 && (uint32_t)__cvta_generic_to_shared(smem) != kDynSmemBase) __trap();
+}
+
 template <int VIS>
 __device__ __forceinline__ uint32_t bm_word(const VisMap<VIS> &m, int w)
 {
-    if (in_smem(m, w)) return m.s[phys<VIS>(w)];
+    if (in_smem(m, w)) return lds_bm(phys<VIS>(w));
     return __ldcg(m.g + w);
 }
 
@@ -137,24 +168,42 @@ __device__ __forceinline__ bool mark(const VisMap<VIS> &m, uint32_t *sm, int v)
 {
     const uint32_t b = 1u << (v & 31);
     const int w = v >> 5;
-    const uint32_t old = in_smem(m, w) ? atomicOr(m.s + phys<VIS>(w), b) : atomicOr(m.g + w, b);
+    const uint32_t old = in_smem(m, w) ? atom_or_bm(phys<VIS>(w), b) : atomicOr(m.g + w, b);
     if (old == 0) atomicOr(sm + (v >> 10), 1u << (w & 31));
     return !(old & b);
 }
 
+// ELL slots W in {4, 6, 8}; rows are stored 4 (W = 4) or 8 (W = 6, 8) entries wide.  A light
+// row of degree < W is padded with the vertex itself, which is always visited when its row is
+// read, so the slot loop needs no sentinel test.
 template <int W>
-__device__ __forceinline__ void load_nb(const int32_t *ell, int f, int (&nb)[W])
+__host__ __device__ constexpr int ell_stride()
 {
-    if constexpr (W == 8) {
+    return W <= 4 ? 4 : 8;
+}
+
+template <int W>
+__device__ __forceinline__ void load_nb(const int32_t *ell, int f, int (&nb)[ell_stride<W>()])
+{
+    if constexpr (ell_stride<W>() == 8) {
         // one 256-bit load per adjacency row (LDG.E.256 on sm_100a)
         asm("ld.global.nc.v8.b32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
             : "=r"(nb[0]), "=r"(nb[1]), "=r"(nb[2]), "=r"(nb[3]), "=r"(nb[4]), "=r"(nb[5]),
               "=r"(nb[6]), "=r"(nb[7])
-            : "l"(ell + (size_t)f * W));
+            : "l"(ell + (size_t)f * 8));
     } else {
-        const int4 a = __ldg(reinterpret_cast<const int4 *>(ell + (size_t)f * W));
+        const int4 a = __ldg(reinterpret_cast<const int4 *>(ell + (size_t)f * 4));
         nb[0] = a.x; nb[1] = a.y; nb[2] = a.z; nb[3] = a.w;
     }
+}
+
+// store a frontier entry (shared memory, HBM past q)
+__device__ __forceinline__ void put(int pos, int w, int32_t *NF, int32_t *gNF, int q)
+{
+    if (pos < q)
+        NF[pos] = w;
+    else
+        gNF[pos] = w;
 }
 
 __device__ __forceinline__ int64_t heavy_off(int lo, int hi)
@@ -163,8 +212,7 @@ __device__ __forceinline__ int64_t heavy_off(int lo, int hi)
 }
 
 // warp-aggregated append to a list (smem, spilling to HBM past q entries)
-__device__ __forceinline__ void push(bool pred, int w, int *cnt, int32_t *NF, int32_t *gNF, int q,
-                                     unsigned long long &spills)
+__device__ __forceinline__ void push(bool pred, int w, int *cnt, int32_t *NF, int32_t *gNF, int q)
 {
     const unsigned b = __ballot_sync(kFull, pred);
     if (b == 0) return;
@@ -173,15 +221,7 @@ __device__ __forceinline__ void push(bool pred, int w, int *cnt, int32_t *NF, in
     int base = 0;
     if (lane == leader) base = atomicAdd(cnt, __popc(b));
     base = __shfl_sync(kFull, base, leader);
-    if (pred) {
-        const int pos = base + __popc(b & ((1u << lane) - 1u));
-        if (pos < q) {
-            NF[pos] = w;
-        } else {
-            gNF[pos] = w;
-            ++spills;
-        }
-    }
+    if (pred) put(base + __popc(b & ((1u << lane) - 1u)), w, NF, gNF, q);
 }
 
 // Smallest visited word index >= w0 whose summary bit is set (may exceed whi within the last
@@ -286,78 +326,63 @@ __device__ void clear_words(const VisMap<VIS> &bm, uint32_t *sm, int wlo, int wh
 
 struct RowAcc {
     int ucnt, lmin, lmax;
-    unsigned long long te, sv, spills;
 };
 
 // Scan the vertices L[0..cnt) (smem, HBM past q) of one BFS level below t0: test-and-set every
 // neighbour; new ones below t0 form the next level (appended to NF), new ones above t0 are
 // pattern entries (L130-147).
 template <int NT, int W, int VIS>
-__device__ __forceinline__ void scan_level(const Fill2Params &p, const VisMap<VIS> &bm, uint32_t *sm,
-                                           const int32_t *L,
-                                           const int32_t *gL, int cnt, int *ncnt, int32_t *NF,
-                                           int32_t *gNF, const int i, const int t0, int &nmin,
-                                           RowAcc &a)
+__device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm,
+                                           uint32_t *sm, const int32_t *L, const int32_t *gL,
+                                           int cnt, int *ncnt, int32_t *NF, int32_t *gNF,
+                                           const int i, const int t0, RowAcc &a)
 {
     const int tid = threadIdx.x, lane = tid & 31;
+    const unsigned lt = (1u << lane) - 1u;
     for (int base = 0; base < cnt; base += NT) {
         const int k = base + tid;
         const bool valid = k < cnt;
-        int nb[W];
+        int nb[ell_stride<W>()];
 #pragma unroll
-        for (int s = 0; s < W; ++s) nb[s] = -1;
+        for (int s = 0; s < ell_stride<W>(); ++s) nb[s] = 0;
         bool heavy = false;
+        // new frontier vertices of this thread: the first two stay in registers (f0, f1) for
+        // one warp-aggregated append; further ones (rare: a vertex with 3+ new neighbours below
+        // t0) are appended one by one
+        int c = 0, f0 = 0, f1 = 0;
         if (valid) {
             const int f = k < p.q ? L[k] : __ldcg(gL + k);
             load_nb<W>(p.ell, f, nb);
             heavy = nb[0] == kHeavy;
-        }
-        uint32_t frm = 0;
-        if (valid && !heavy) {
-            ++a.sv;
-#pragma unroll
-            for (int s = 0; s < W; ++s) {
-                const int w = nb[s];
-                if (w >= 0 && !visited(bm, w) && mark(bm, sm, w)) {
-                    if (w < t0) {
-                        frm |= 1u << s;
-                    } else if (w > i) {
-                        ++a.ucnt;
-                        a.lmax = max(a.lmax, w);
-                    }
-                }
-            }
-        }
-        {
-            // one warp-aggregated append for all new frontier vertices of the warp
-            const int c = __popc(frm);
-            int inc = c;
-#pragma unroll
-            for (int o = 1; o < 32; o <<= 1) {
-                const int y = __shfl_up_sync(kFull, inc, o);
-                if (lane >= o) inc += y;
-            }
-            const int total = __shfl_sync(kFull, inc, 31);
-            if (total) {
-                int wbase = 0;
-                if (lane == 31) wbase = atomicAdd(ncnt, total);
-                wbase = __shfl_sync(kFull, wbase, 31);
-                int pos = wbase + inc - c;
+            if (!heavy) {
 #pragma unroll
                 for (int s = 0; s < W; ++s) {
-                    if (frm & (1u << s)) {
-                        const int w = nb[s];
-                        nmin = min(nmin, w);
-                        if (pos < p.q) {
-                            NF[pos] = w;
-                        } else {
-                            gNF[pos] = w;
-                            ++a.spills;
+                    const int w = nb[s];
+                    if (!visited(bm, w) && mark(bm, sm, w)) {
+                        if (w < t0) {
+                            if (c == 2) {
+                                put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
+                            } else {
+                                f1 = f0;
+                                f0 = w;
+                                ++c;
+                            }
+                        } else if (w > i) {
+                            ++a.ucnt;
+                            a.lmax = max(a.lmax, w);
                         }
-                        ++pos;
                     }
                 }
             }
+        }
+        const unsigned b1 = __ballot_sync(kFull, c & 1), b2 = __ballot_sync(kFull, c & 2);
+        if (b1 | b2) {
+            int wbase = 0;
+            if (lane == 0) wbase = atomicAdd(ncnt, __popc(b1) + 2 * __popc(b2));
+            wbase = __shfl_sync(kFull, wbase, 0);
+            const int pos = wbase + __popc(b1 & lt) + 2 * __popc(b2 & lt);
+            if (c) put(pos, f0, NF, gNF, p.q);
+            if (c == 2) put(pos + 1, f1, NF, gNF, p.q);
         }
         // heavy vertices (degree > W): one warp each, over A's CSR row
         unsigned hm = __ballot_sync(kFull, valid && heavy);
@@ -367,10 +392,7 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, const VisMap<VI
             const int len = __shfl_sync(kFull, nb[1], src);
             const int64_t off =
                 heavy_off(__shfl_sync(kFull, nb[2], src), __shfl_sync(kFull, nb[3], src));
-            if (lane == 0) {
-                a.te += len;
-                ++a.sv;
-            }
+            if (lane == 0) atomicAdd(&h.te, (unsigned long long)len);
             for (int eb = 0; eb < len; eb += 32) {
                 const int e = eb + lane;
                 bool fr = false;
@@ -380,14 +402,13 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, const VisMap<VI
                     if (!visited(bm, w) && mark(bm, sm, w)) {
                         if (w < t0) {
                             fr = true;
-                            nmin = min(nmin, w);
                         } else if (w > i) {
                             ++a.ucnt;
                             a.lmax = max(a.lmax, w);
                         }
                     }
                 }
-                push(fr, w, ncnt, NF, gNF, p.q, a.spills);
+                push(fr, w, ncnt, NF, gNF, p.q);
             }
         }
     }
@@ -409,16 +430,19 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_
     int fsize = 1;
     for (int lev = 0;; ++lev) {
         int *ncnt = &h.cnt[(lev + 1) % 3];
-        if (tid == 0) h.cnt[(lev + 2) % 3] = 0;
-        int nmin = INT_MAX;
-        scan_level<NT, W, VIS>(p, bm, sm, F, gF, fsize, ncnt, NF, gNF, i, t0, nmin, a);
-        a.lmin = min(a.lmin, nmin);
+        if (tid == 0) {
+            h.cnt[(lev + 2) % 3] = 0;
+            h.sv += fsize;
+        }
+        scan_level<NT, W, VIS>(p, h, bm, sm, F, gF, fsize, ncnt, NF, gNF, i, t0, a);
         __syncthreads();
         fsize = *ncnt;
         if (fsize == 0) break;
+        if (tid == 0 && fsize > p.q) h.spills += fsize - p.q;
         int32_t *t = F; F = NF; NF = t;
         t = gF; gF = gNF; gNF = t;
     }
+    a.lmin = 0;  // the BFS marked vertices somewhere below t0: clear from word 0 (summary walk)
 }
 
 // MODE: kCount (symbolic_1, counts only), kStage (counts + rows staged into the HBM pool, so
@@ -448,12 +472,14 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
     int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
     int32_t *gB = gA + p.spill_cap;
     const int tid = threadIdx.x, lane = tid & 31;
+    (void)lane;
+    if constexpr (!GB) check_smem_base(smem);
     for (int w = tid; w < p.sw; w += NT) sm[w] = 0;
     if constexpr (!GB)
         for (int w = tid; w < p.nw; w += NT) bm.s[w] = 0;
 
     RowAcc a;
-    a.te = a.sv = a.spills = 0;
+    if (tid == 0) h.te = h.sv = h.spills = 0;
     const int nrows = p.row_end - p.row_begin;
     for (;;) {
         if (tid == 0) {
@@ -475,7 +501,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
         const int i = h.row;
         if (i < 0) break;
         const long long t_row = p.row_prof ? clock64() : 0;
-        const unsigned long long sv_row = a.sv;
+        const unsigned long long sv_row = h.sv;  // read and written by thread 0 only
         int n_bfs = 0, n_win = 0;
         a.ucnt = 0;
         a.lmin = i;
@@ -485,7 +511,6 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
         const int64_t rb = p.rp[i], re = p.rp[i + 1];
         for (int64_t k = rb + tid; k < re; k += NT) {
             const int v = __ldg(p.ci + k);
-            ++a.te;
             mark(bm, sm, v);
             if (v < i) {
                 atomicMin(&h.minseed, v);
@@ -497,7 +522,10 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                 h.diag = 1;
             }
         }
-        if (tid == 0) mark(bm, sm, i);
+        if (tid == 0) {
+            mark(bm, sm, i);
+            h.te += (unsigned long long)(re - rb);
+        }
         __syncthreads();
 
         int ptr = h.minseed - 1;  // every unprocessed threshold is > ptr
@@ -528,6 +556,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
             if (tid == 0) {
                 h.tns = INT_MAX;
                 h.newmin = INT_MAX;
+                h.sv += wc;
             }
             __syncthreads();
             int nm = INT_MAX;
@@ -535,21 +564,20 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                 const int k = base + tid;
                 const bool valid = k < wc;
                 const int t = valid ? qA[k] : 0;
-                int nb[W];
+                int nb[ell_stride<W>()];
 #pragma unroll
-                for (int s = 0; s < W; ++s) nb[s] = -1;
+                for (int s = 0; s < ell_stride<W>(); ++s) nb[s] = 0;
                 bool heavy = false, done = false;
                 if (valid) {
                     load_nb<W>(p.ell, t, nb);
                     heavy = nb[0] == kHeavy;
                 }
                 if (valid && !heavy) {
-                    ++a.sv;
                     bool simple = true;
 #pragma unroll
                     for (int s = 0; s < W; ++s) {
                         const int w = nb[s];
-                        if (w >= 0 && w < t && !visited(bm, w)) simple = false;
+                        if (w < t && !visited(bm, w)) simple = false;
                     }
                     if (!simple) {
                         atomicMin(&h.tns, t);
@@ -583,10 +611,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                         if (w < tt && !visited(bm, w)) ok = false;
                     }
                     ok = __all_sync(kFull, ok);
-                    if (lane == 0) {
-                        a.te += len;
-                        ++a.sv;
-                    }
+                    if (lane == 0) atomicAdd(&h.te, (unsigned long long)len);
                     if (lane == src) done = ok;
                     if (!ok) {
                         if (lane == 0) atomicMin(&h.tns, tt);
@@ -675,35 +700,22 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                                          h.scan);
             }
         }
-        if (p.row_prof) {
-            unsigned long long dsv = a.sv - sv_row;
-#pragma unroll
-            for (int o = 16; o > 0; o >>= 1) dsv += __shfl_xor_sync(kFull, dsv, o);
-            if (lane == 0 && dsv) atomicAdd(reinterpret_cast<unsigned long long *>(p.row_prof) +
-                                                4 * (size_t)i + 1, dsv);
-            if (tid == 0) {
-                p.row_prof[4 * (size_t)i + 0] = clock64() - t_row;
-                p.row_prof[4 * (size_t)i + 2] = n_bfs;
-                p.row_prof[4 * (size_t)i + 3] = n_win;
-            }
+        if (p.row_prof && tid == 0) {
+            p.row_prof[4 * (size_t)i + 0] = clock64() - t_row;
+            p.row_prof[4 * (size_t)i + 1] = (long long)(h.sv - sv_row);
+            p.row_prof[4 * (size_t)i + 2] = n_bfs;
+            p.row_prof[4 * (size_t)i + 3] = n_win;
         }
         // ---- clear the dirty word range (fill(:) = 0 for the next row, L115)
         clear_words<NT, VIS>(bm, sm, gmin >> 5, gmax >> 5);
         __syncthreads();
     }
 
-    // flush statistics
-    unsigned long long te = a.te, sv = a.sv, sp = a.spills;
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) {
-        te += __shfl_xor_sync(kFull, te, o);
-        sv += __shfl_xor_sync(kFull, sv, o);
-        sp += __shfl_xor_sync(kFull, sp, o);
-    }
-    if (lane == 0) {
-        atomicAdd(p.stats + kStatEdges, te);
-        atomicAdd(p.stats + kStatVerts, sv);
-        if (sp) atomicAdd(p.stats + kStatSpills, sp);
+    // flush statistics (every heavy-vertex atomic finished before the last barrier)
+    if (tid == 0) {
+        atomicAdd(p.stats + kStatEdges, h.te);
+        atomicAdd(p.stats + kStatVerts, h.sv);
+        if (h.spills) atomicAdd(p.stats + kStatSpills, h.spills);
     }
 }
 
@@ -757,6 +769,9 @@ cudaError_t dispatch_w_vis(int w, int vis, Args... args)
     if (w == 4 && vis == kVisSmem) return Op<NT, 4, kVisSmem>::run(args...);
     if (w == 4 && vis == kVisGlobal) return Op<NT, 4, kVisGlobal>::run(args...);
     if (w == 4 && vis == kVisSplit) return Op<NT, 4, kVisSplit>::run(args...);
+    if (w == 6 && vis == kVisSmem) return Op<NT, 6, kVisSmem>::run(args...);
+    if (w == 6 && vis == kVisGlobal) return Op<NT, 6, kVisGlobal>::run(args...);
+    if (w == 6 && vis == kVisSplit) return Op<NT, 6, kVisSplit>::run(args...);
     if (w == 8 && vis == kVisSmem) return Op<NT, 8, kVisSmem>::run(args...);
     if (w == 8 && vis == kVisGlobal) return Op<NT, 8, kVisGlobal>::run(args...);
     if (w == 8 && vis == kVisSplit) return Op<NT, 8, kVisSplit>::run(args...);

@@ -556,22 +556,23 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
         *out = h;
         return LU_OK;
     }
-    // traversal adjacency width: 4 when nearly every vertex has <= 4 off-diagonal entries
+    // traversal adjacency slots W: the smallest of 4 / 6 / 8 that holds nearly every vertex's
+    // off-diagonal entries (rows are stored 4 or 8 wide; larger rows are heavy records)
     {
         int w = h->opts.ell_width;
-        if (w != 0 && w != 4 && w != 8)
-            return bail(fail(LU_ERR_ARG, "ell_width must be 0, 4 or 8 (got %d)", w));
-        if (w == 0) {
-            unsigned long long light4 = 0;
-            cudaError_t e = count_light(n, d_row_ptr, d_col_idx, 4, h->dstats + 15, s);
+        if (w != 0 && w != 4 && w != 6 && w != 8)
+            return bail(fail(LU_ERR_ARG, "ell_width must be 0, 4, 6 or 8 (got %d)", w));
+        for (int cand = 4; w == 0 && cand <= 8; cand += 2) {
+            unsigned long long light = 0;
+            cudaError_t e = count_light(n, d_row_ptr, d_col_idx, cand, h->dstats + 15, s);
             if (e == cudaSuccess)
-                e = cudaMemcpyAsync(&light4, h->dstats + 15, 8, cudaMemcpyDeviceToHost, s);
+                e = cudaMemcpyAsync(&light, h->dstats + 15, 8, cudaMemcpyDeviceToHost, s);
             if (e == cudaSuccess) e = cudaStreamSynchronize(s);
             if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
-            w = (light4 >= (unsigned long long)(0.995 * n)) ? 4 : 8;
+            if (cand == 8 || light >= (unsigned long long)(0.995 * n)) w = cand;
         }
         h->w = w;
-        if ((st = dalloc(h, &h->ell, (size_t)n * w)) != LU_OK) return bail(st);
+        if ((st = dalloc(h, &h->ell, (size_t)n * (w <= 4 ? 4 : 8))) != LU_OK) return bail(st);
         cudaError_t e = build_ell(n, d_row_ptr, d_col_idx, w, h->ell, s);
         if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
     }

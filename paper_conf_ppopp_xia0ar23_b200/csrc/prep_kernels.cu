@@ -67,19 +67,21 @@ __global__ void k_count_light(int32_t n, const int64_t *rp, const int32_t *ci, i
     if ((threadIdx.x & 31) == 0 && m) atomicAdd(cnt, (unsigned long long)__popc(m));
 }
 
-// ell[i*W .. i*W+W) = off-diagonal neighbours of i padded with -1, or the heavy record
-// {kHeavy, len, off_lo, off_hi} pointing at A's own row (diagonal included: it is always
-// visited when i is scanned, so the traversal skips it).
+// ell[i*S .. i*S+S), S = 4 (W = 4) or 8 (W = 6, 8): the off-diagonal neighbours of i padded
+// with i itself up to W slots (i is always visited when its row is read, so a padded slot is a
+// no-op test), or, for degree > W, the heavy record {kHeavy, len, off_lo, off_hi} pointing at
+// A's own row (diagonal included: it is always visited when i is scanned, so it is skipped).
 template <int W>
 __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int32_t *ell)
 {
+    constexpr int S = W <= 4 ? 4 : 8;
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
     if (i >= n) return;
     const int64_t a = rp[i], b = rp[i + 1];
     const int64_t len = b - a;
-    int out[W];
+    int out[S];
 #pragma unroll
-    for (int s = 0; s < W; ++s) out[s] = -1;
+    for (int s = 0; s < S; ++s) out[s] = s < W ? i : -1;
     bool heavy = len > W + 1;
     if (!heavy) {
         int m = 0;
@@ -90,7 +92,10 @@ __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int
                 heavy = true;
                 break;
             }
-            out[m++] = c;
+#pragma unroll
+            for (int s = 0; s < W; ++s)
+                if (s == m) out[s] = c;
+            ++m;
         }
     }
     if (heavy) {
@@ -99,11 +104,11 @@ __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int
         out[2] = (int)(uint32_t)(a & 0xffffffffll);
         out[3] = (int)(a >> 32);
 #pragma unroll
-        for (int s = 4; s < W; ++s) out[s] = -1;
+        for (int s = 4; s < S; ++s) out[s] = -1;
     }
-    int4 *dst = reinterpret_cast<int4 *>(ell + (size_t)i * W);
+    int4 *dst = reinterpret_cast<int4 *>(ell + (size_t)i * S);
     dst[0] = make_int4(out[0], out[1], out[2], out[3]);
-    if constexpr (W == 8) dst[1] = make_int4(out[4], out[5], out[6], out[7]);
+    if constexpr (S == 8) dst[1] = make_int4(out[4], out[5], out[6], out[7]);
 }
 
 // rows i < bound whose largest column is >= bound (their marks would leave a split map)
@@ -232,6 +237,8 @@ cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, in
     if (n == 0) return cudaSuccess;
     if (w == 4)
         k_build_ell<4><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
+    else if (w == 6)
+        k_build_ell<6><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
     else
         k_build_ell<8><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
     return cudaGetLastError();
