@@ -415,32 +415,38 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
 }
 
 // Level-synchronous BFS from threshold t0 over unvisited vertices < t0 (Alg. 1).
+// Level lev reads queue lev&1 and writes queue (lev+1)&1 (shared, spilling to the CTA's two
+// HBM halves); the level counters rotate through h.cnt[0..2] so one barrier per level suffices.
+// Queue and spill addresses are recomputed from the launch parameters each level rather than
+// carried in registers (at 32 registers per thread they would otherwise spill).
 template <int NT, int W, int VIS>
 __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_t *sm, int32_t *qA,
-                    int32_t *qB,
-                    int32_t *gA, int32_t *gB, const int i, const int t0, RowAcc &a)
+                    const int i, const int t0, RowAcc &a)
 {
     const int tid = threadIdx.x;
-    int32_t *F = qA, *NF = qB, *gF = gA, *gNF = gB;
     if (tid == 0) {
-        F[0] = t0;
+        qA[0] = t0;
         h.cnt[1] = h.cnt[2] = 0;
+        h.sv += 1;
     }
     __syncthreads();
-    int fsize = 1;
+    int fsize = 1, cur = 0;  // cur: counter index of the level being read
     for (int lev = 0;; ++lev) {
-        int *ncnt = &h.cnt[(lev + 1) % 3];
-        if (tid == 0) {
-            h.cnt[(lev + 2) % 3] = 0;
-            h.sv += fsize;
-        }
-        scan_level<NT, W, VIS>(p, h, bm, sm, F, gF, fsize, ncnt, NF, gNF, i, t0, a);
+        const int par = lev & 1;
+        const int nxt = cur == 2 ? 0 : cur + 1;
+        int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
+        scan_level<NT, W, VIS>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap, fsize,
+                               &h.cnt[nxt], qA + (par ^ 1) * p.q, gA + (par ^ 1) * p.spill_cap,
+                               i, t0, a);
         __syncthreads();
-        fsize = *ncnt;
+        fsize = h.cnt[nxt];
         if (fsize == 0) break;
-        if (tid == 0 && fsize > p.q) h.spills += fsize - p.q;
-        int32_t *t = F; F = NF; NF = t;
-        t = gF; gF = gNF; gNF = t;
+        if (tid == 0) {
+            h.cnt[cur] = 0;  // becomes the write counter two levels from now
+            h.sv += fsize;
+            if (fsize > p.q) h.spills += fsize - p.q;
+        }
+        cur = nxt;
     }
     a.lmin = 0;  // the BFS marked vertices somewhere below t0: clear from word 0 (summary walk)
 }
@@ -469,8 +475,6 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
     }
     qA = reinterpret_cast<int32_t *>(sm + p.sw);
     qB = qA + p.q;
-    int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
-    int32_t *gB = gA + p.spill_cap;
     const int tid = threadIdx.x, lane = tid & 31;
     (void)lane;
     if constexpr (!GB) check_smem_base(smem);
@@ -652,7 +656,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
             }
             __syncthreads();
             if (m <= last && m == tns) {  // smallest pending threshold: below-exploration
-                bfs<NT, W, VIS>(p, h, bm, sm, qA, qB, gA, gB, i, m, a);
+                bfs<NT, W, VIS>(p, h, bm, sm, qA, i, m, a);
                 ++n_bfs;
             }
             cap = m <= last ? min(cap, kSmallWin) : min(2 * cap, p.wcap);
