@@ -92,7 +92,9 @@ struct VisMap {
     uint32_t *s;  // shared part
     uint32_t *g;  // HBM slot (word index = vertex >> 5)
     int lbw;      // words held in shared memory (kVisSplit)
+    int nw;       // shared visited words (the level-1 summary follows them)
 };
+
 
 template <int VIS>
 __device__ __forceinline__ int phys(int w)
@@ -139,6 +141,13 @@ __device__ __forceinline__ void check_smem_base(const unsigned char *smem)
     if (threadIdx.x == 0 && (uint32_t)__cvta_generic_to_shared(smem) != kDynSmemBase) __trap();
 }
 
+// shared byte address of the level-1 summary (right after the shared visited words)
+template <int VIS>
+__device__ __forceinline__ uint32_t summary_saddr(const VisMap<VIS> &m)
+{
+    return VIS == kVisGlobal ? kBmShared : kBmShared + 4u * (uint32_t)m.nw;
+}
+
 template <int VIS>
 __device__ __forceinline__ uint32_t bm_word(const VisMap<VIS> &m, int w)
 {
@@ -169,7 +178,11 @@ __device__ __forceinline__ bool mark(const VisMap<VIS> &m, uint32_t *sm, int v)
     const uint32_t b = 1u << (v & 31);
     const int w = v >> 5;
     const uint32_t old = in_smem(m, w) ? atom_or_bm(phys<VIS>(w), b) : atomicOr(m.g + w, b);
-    if (old == 0) atomicOr(sm + (v >> 10), 1u << (w & 31));
+    if (old == 0)
+        asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(summary_saddr(m) + (uint32_t)(v >> 10) * 4u),
+                     "r"(1u << (w & 31))
+                     : "memory");
+    (void)sm;
     return !(old & b);
 }
 
@@ -346,10 +359,10 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
 #pragma unroll
         for (int s = 0; s < ell_stride<W>(); ++s) nb[s] = 0;
         bool heavy = false;
-        // new frontier vertices of this thread: the first two stay in registers (f0, f1) for
-        // one warp-aggregated append; further ones (rare: a vertex with 3+ new neighbours below
-        // t0) are appended one by one
-        int c = 0, f0 = 0, f1 = 0;
+        // new frontier vertices of this thread: the first three stay in registers (f0..f2) for
+        // one warp-aggregated append (a grid vertex has up to three neighbours further from
+        // the BFS source); further ones (rare) are appended one by one
+        int c = 0, f0 = 0, f1 = 0, f2 = 0;
         if (valid) {
             const int f = k < p.q ? L[k] : __ldcg(gL + k);
             load_nb<W>(p.ell, f, nb);
@@ -360,9 +373,10 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                     const int w = nb[s];
                     if (!visited(bm, w) && mark(bm, sm, w)) {
                         if (w < t0) {
-                            if (c == 2) {
+                            if (c == 3) {
                                 put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
                             } else {
+                                f2 = f1;
                                 f1 = f0;
                                 f0 = w;
                                 ++c;
@@ -382,7 +396,8 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
             wbase = __shfl_sync(kFull, wbase, 0);
             const int pos = wbase + __popc(b1 & lt) + 2 * __popc(b2 & lt);
             if (c) put(pos, f0, NF, gNF, p.q);
-            if (c == 2) put(pos + 1, f1, NF, gNF, p.q);
+            if (c >= 2) put(pos + 1, f1, NF, gNF, p.q);
+            if (c == 3) put(pos + 2, f2, NF, gNF, p.q);
         }
         // heavy vertices (degree > W): one warp each, over A's CSR row
         unsigned hm = __ballot_sync(kFull, valid && heavy);
@@ -464,6 +479,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
     VisMap<VIS> bm;
     bm.g = p.gbitmap ? p.gbitmap + (size_t)blockIdx.x * p.gbitmap_stride : nullptr;
     bm.lbw = p.lbw;
+    bm.nw = GB ? 0 : p.nw;
     uint32_t *sm;
     int32_t *qA, *qB;
     if constexpr (GB) {
