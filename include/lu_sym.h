@@ -72,8 +72,14 @@ enum {
                                     printed, symbolic_2 repeats symbolic_1's work)           */
     LU_F_ONE_CLASS = 1 << 7,     /* one row class (Alg. 3's single chunk size) instead of
                                     Alg. 4's row classes by scratch need (L272-277)          */
-    LU_F_FORCE_CLASSES = 1 << 8  /* test knob: split row classes down to 64 shared words even
+    LU_F_FORCE_CLASSES = 1 << 8, /* test knob: split row classes down to 64 shared words even
                                     when that does not add rows in flight                     */
+    LU_F_SELF_CONT = 1 << 9,     /* BFS self-continuation (a lane expands its own first new
+                                    vertex in the next round; the order below a threshold is
+                                    free, reading R5) in every row class, not only in classes
+                                    with one row per SM                                       */
+    LU_F_NO_SELF_CONT = 1 << 10  /* no self-continuation anywhere (plain level-synchronous
+                                    BFS)                                                      */
 };
 
 typedef struct {

@@ -343,7 +343,12 @@ struct RowAcc {
 
 // Scan the vertices L[0..cnt) (smem, HBM past q) of one BFS level below t0: test-and-set every
 // neighbour; new ones below t0 form the next level (appended to NF), new ones above t0 are
-// pattern entries (L130-147).
+// pattern entries (L130-147).  Self-continuation (reading R5, the order below a threshold is
+// free): a lane that discovered new vertices expands the first of them itself in the next
+// round, up to p.kloc rounds, so a BFS front advances more than one step per level barrier;
+// only the other discoveries go through the next-level queue.  Worth it only where a row has
+// an SM to itself and waits on each level's latency (the planner sets kloc per row class):
+// with many rows per SM the extra rounds, in which lanes drop out, cost issue slots.
 template <int NT, int W, int VIS>
 __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm,
                                            uint32_t *sm, const int32_t *L, const int32_t *gL,
@@ -352,9 +357,12 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
 {
     const int tid = threadIdx.x, lane = tid & 31;
     const unsigned lt = (1u << lane) - 1u;
+    unsigned nloc = 0;  // vertices expanded by self-continuation (statistics, lane 0)
     for (int base = 0; base < cnt; base += NT) {
         const int k = base + tid;
-        const bool valid = k < cnt;
+        bool valid = k < cnt;
+        int f = valid ? (k < p.q ? L[k] : __ldcg(gL + k)) : 0;
+      for (int r = 0;; ++r) {
         int nb[ell_stride<W>()];
 #pragma unroll
         for (int s = 0; s < ell_stride<W>(); ++s) nb[s] = 0;
@@ -364,7 +372,6 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
         // the BFS source); further ones (rare) are appended one by one
         int c = 0, f0 = 0, f1 = 0, f2 = 0;
         if (valid) {
-            const int f = k < p.q ? L[k] : __ldcg(gL + k);
             load_nb<W>(p.ell, f, nb);
             heavy = nb[0] == kHeavy;
             if (!heavy) {
@@ -388,6 +395,15 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                     }
                 }
             }
+        }
+        // keep f0 for the next round, append the rest
+        const bool keep = r < p.kloc && c > 0;
+        if (keep) {
+            --c;
+            const int t = f0;
+            f0 = f1;
+            f1 = f2;
+            f2 = t;
         }
         const unsigned b1 = __ballot_sync(kFull, c & 1), b2 = __ballot_sync(kFull, c & 2);
         if (b1 | b2) {
@@ -426,7 +442,14 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                 push(fr, w, ncnt, NF, gNF, p.q);
             }
         }
+        const unsigned kb = __ballot_sync(kFull, keep);
+        if (!kb) break;
+        nloc += __popc(kb);
+        valid = keep;
+        f = f2;
+      }
     }
+    if (lane == 0 && nloc) atomicAdd(&h.sv, (unsigned long long)nloc);
 }
 
 // Level-synchronous BFS from threshold t0 over unvisited vertices < t0 (Alg. 1).

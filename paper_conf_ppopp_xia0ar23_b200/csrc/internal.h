@@ -50,6 +50,8 @@ struct Fill2Params {
     unsigned long long *unstaged_cnt;
     // optional per-row profile (4 x int64 per row: cycles, vertices scanned, BFS runs, windows)
     int64_t *row_prof;
+    // self-continuation rounds per BFS level (scan_level); 0 = plain level-synchronous BFS
+    int32_t kloc;
 };
 enum Fill2Mode { kCount = 0, kEmit = 1, kStage = 2 };
 

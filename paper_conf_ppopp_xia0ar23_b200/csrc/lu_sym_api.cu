@@ -179,6 +179,13 @@ void free_handle(lu_sym *h)
 // shared memory (their whole BFS region lies below i; marks above go to the HBM slot), so lower
 // classes fit more rows per SM.  Within a class the CTA size and queue capacity maximise
 // resident threads, then rows in flight; the HBM budget caps rows in flight.
+#ifndef LUSYM_KLOC  // self-continuation rounds in latency-bound classes (scan_level)
+#define LUSYM_KLOC 2
+#endif
+#ifndef LUSYM_KLOC_OCC  // ... those with at most this many rows per SM
+#define LUSYM_KLOC_OCC 2
+#endif
+
 struct Cfg {
     int nt, q, occ;
     size_t smem;
@@ -425,6 +432,11 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
         p.lbw = c.lbw;
         p.q = c.q;
         p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : c.q;
+        // one row per SM: a BFS level is latency-bound, let lanes run ahead a little
+        p.kloc = ((c.occ <= LUSYM_KLOC_OCC || (h->opts.flags & LU_F_SELF_CONT)) &&
+                  !(h->opts.flags & LU_F_NO_SELF_CONT))
+                     ? LUSYM_KLOC
+                     : 0;
         const int grid = c.grid < rows ? c.grid : rows;
         CK(fill2_launch(p, c.nt, h->w, mode, c.vis, grid, c.smem, cs));
         h->launches += 1;

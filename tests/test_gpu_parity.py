@@ -148,6 +148,11 @@ KNOBS = [
     dict(flags=lu.F_FORCE_CLASSES, queue_capacity=32, rows_in_flight=7),
     dict(pool_bytes=4096),                           # pool overflow: most rows re-traversed
     dict(pool_bytes=200_000),                        # partial staging
+    dict(flags=lu.F_SELF_CONT),                      # BFS self-continuation in every class
+    dict(flags=lu.F_SELF_CONT, queue_capacity=32),   # ... with frontier spills
+    dict(flags=lu.F_SELF_CONT | lu.F_GLOBAL_BITMAP | lu.F_FORCE_CLASSES),
+    dict(flags=lu.F_SELF_CONT | lu.F_TWO_PASS, threads_per_row=1024),
+    dict(flags=lu.F_NO_SELF_CONT, threads_per_row=1024, rows_in_flight=148),
 ]
 
 
