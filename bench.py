@@ -93,17 +93,34 @@ REASONS = ["gpu_idle", "applications_clocks_setting", "sw_power_cap", "hw_slowdo
 
 
 class ClockSampler:
+    """SM clock + clock-event reasons sampled DURING the timed region: NVML in a thread every
+    10 ms (nvidia-smi -lms as the fallback), so even a ~0.2 s region gets a dozen samples.
+    Reason bits follow nvmlClocksEventReason* (the same bits nvidia-smi reports)."""
+
+    PERIOD_S = 0.01
+
     def __init__(self, index):
         self.index = index
-        self.samples = []
+        self.samples = []  # (sm_mhz, max_mhz, reasons_bitmask, busy)
         self.proc = None
+        self.stop = threading.Event()
+        self.thread = None
 
     def __enter__(self):
+        try:
+            import pynvml
+            pynvml.nvmlInit()
+            hd = pynvml.nvmlDeviceGetHandleByIndex(self._nvml_index())
+            self.thread = threading.Thread(target=self._nvml, args=(pynvml, hd), daemon=True)
+            self.thread.start()
+            return self
+        except Exception:
+            pass
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.index),
                  "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
-                 "utilization.gpu", "--format=csv,noheader,nounits", "-lms", "200"],
+                 "utilization.gpu", "--format=csv,noheader,nounits", "-lms", "100"],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.thread = threading.Thread(target=self._read, daemon=True)
             self.thread.start()
@@ -111,37 +128,60 @@ class ClockSampler:
             self.proc = None
         return self
 
+    def _nvml_index(self):
+        # CUDA_VISIBLE_DEVICES may remap: take the physical index of the visible device
+        ids = [v.strip() for v in os.environ.get("CUDA_VISIBLE_DEVICES", "").split(",")
+               if v.strip()]
+        if ids and self.index < len(ids) and ids[self.index].isdigit():
+            return int(ids[self.index])
+        return self.index
+
+    def _nvml(self, pynvml, hd):
+        mx = pynvml.nvmlDeviceGetMaxClockInfo(hd, pynvml.NVML_CLOCK_SM)
+        while not self.stop.is_set():
+            try:
+                c = pynvml.nvmlDeviceGetClockInfo(hd, pynvml.NVML_CLOCK_SM)
+                r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(hd)
+                self.samples.append((float(c), float(mx), int(r), not (r & 1)))
+            except Exception:
+                pass
+            self.stop.wait(self.PERIOD_S)
+
     def _read(self):
         for line in self.proc.stdout:
             parts = [p.strip() for p in line.split(",")]
-            if len(parts) >= 4:
-                self.samples.append(parts)
+            try:
+                r = int(parts[2], 16)
+                self.samples.append((float(parts[0]), float(parts[1]), r,
+                                     float(parts[3]) > 0 or not (r & 1)))
+            except (ValueError, IndexError):
+                continue
 
     def __exit__(self, *a):
+        self.stop.set()
         if self.proc is not None:
             self.proc.terminate()
             try:
                 self.proc.wait(timeout=5)
             except Exception:
                 self.proc.kill()
+        if self.thread is not None:
+            self.thread.join(timeout=5)
 
     def summary(self):
         if not self.samples:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"]}
         sm, mx, reasons = [], None, set()
-        for s in self.samples:
-            try:
-                c, m, r, u = float(s[0]), float(s[1]), int(s[2], 16), float(s[3])
-            except ValueError:
-                continue
+        for c, m, r, busy in self.samples:
             mx = m
-            if u > 0:
+            if busy:
                 sm.append(c)
             for b, name in enumerate(REASONS):
                 if r & (1 << b) and name != "gpu_idle":
                     reasons.add(name)
         return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx,
-                "reasons": sorted(reasons), "samples": len(self.samples)}
+                "reasons": sorted(reasons), "samples": len(self.samples),
+                "source": "nvml" if self.proc is None else "nvidia-smi"}
 
 
 # --------------------------------------------------------------------------- CPU oracle

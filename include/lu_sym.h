@@ -78,8 +78,16 @@ enum {
                                     vertex in the next round; the order below a threshold is
                                     free, reading R5) in every row class, not only in classes
                                     with one row per SM                                       */
-    LU_F_NO_SELF_CONT = 1 << 10  /* no self-continuation anywhere (plain level-synchronous
+    LU_F_NO_SELF_CONT = 1 << 10, /* no self-continuation anywhere (plain level-synchronous
                                     BFS)                                                      */
+    LU_F_PAPER_CHUNKS = 1 << 11  /* Alg. 3's launch scheme (L239-243, L253-267): each pass is
+                                    num_iter = ceil(rows / chunk_size) launches issued one
+                                    after another, chunk_size = L / (c n) rows with c = 6
+                                    4-byte words per vertex and L = the scratch budget (reading
+                                    R16), chunks in increasing row order; with LU_F_ONE_CLASS
+                                    this is Alg. 3, without it Alg. 4 (one chunk size per row
+                                    class).  Ablation of the persistent heaviest-first launch
+                                                                                */
 };
 
 typedef struct {

@@ -437,6 +437,23 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
                   !(h->opts.flags & LU_F_NO_SELF_CONT))
                      ? LUSYM_KLOC
                      : 0;
+        if ((h->opts.flags & LU_F_PAPER_CHUNKS) && !row_list) {
+            // Alg. 3 / Alg. 4 as printed: chunk_size = L / (c n) rows per launch (c = 6 words of
+            // 4 B per vertex, L = scratch budget, reading R16), launches in increasing row order
+            const uint64_t per_row = (uint64_t)6 * 4 * (uint64_t)h->n;
+            int64_t chunk = (int64_t)(h->budget / (per_row ? per_row : 1));
+            if (chunk < 1) chunk = 1;
+            for (int64_t c0 = lo; c0 < hi; c0 += chunk) {
+                const int64_t c1 = std::min<int64_t>(hi, c0 + chunk);
+                CK(cudaMemsetAsync(p.row_counter, 0, sizeof(unsigned long long), cs));
+                p.row_begin = (int32_t)c0;
+                p.row_end = (int32_t)c1;
+                const int64_t g = std::min<int64_t>(c.grid, c1 - c0);
+                CK(fill2_launch(p, c.nt, h->w, mode, c.vis, (int)g, c.smem, cs));
+                h->launches += 1;
+            }
+            continue;
+        }
         const int grid = c.grid < rows ? c.grid : rows;
         CK(fill2_launch(p, c.nt, h->w, mode, c.vis, grid, c.smem, cs));
         h->launches += 1;

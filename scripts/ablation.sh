@@ -20,8 +20,10 @@ for c in ${CFGS:-2 5 3}; do
   run $c 0   "B200 design (default)"
   run $c 64  "TWO_PASS (symbolic_2 re-traverses)"
   run $c 128 "ONE_CLASS (Alg.3 single chunk size)"
+  run $c 2048 "PAPER_CHUNKS (Alg.4: L/(6n)-row launches)"
+  run $c 2176 "PAPER_CHUNKS|ONE_CLASS (Alg.3 launches)"
   run $c 2   "NO_BATCH (one threshold at a time)"
   run $c 40  "NO_CONTRACT|NO_PRUNE (plain Alg.5 Kahn)"
   run $c 1   "GLOBAL_BITMAP (visited state in HBM)"
-  run $c 235 "paper as printed (all of the above)"
+  run $c 2283 "paper as printed (all of the above)"
 done

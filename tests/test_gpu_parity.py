@@ -153,6 +153,10 @@ KNOBS = [
     dict(flags=lu.F_SELF_CONT | lu.F_GLOBAL_BITMAP | lu.F_FORCE_CLASSES),
     dict(flags=lu.F_SELF_CONT | lu.F_TWO_PASS, threads_per_row=1024),
     dict(flags=lu.F_NO_SELF_CONT, threads_per_row=1024, rows_in_flight=148),
+    # Alg. 3 / Alg. 4 launch scheme: chunk_size = L/(6n) rows per launch (several chunks here)
+    dict(flags=lu.F_PAPER_CHUNKS, scratch_budget_bytes=2_000_000),
+    dict(flags=lu.F_PAPER_CHUNKS | lu.F_ONE_CLASS, scratch_budget_bytes=1_000_000),
+    dict(flags=lu.F_PAPER_CHUNKS | lu.F_FORCE_CLASSES | lu.F_TWO_PASS, scratch_budget_bytes=3_000_000),
 ]
 
 
