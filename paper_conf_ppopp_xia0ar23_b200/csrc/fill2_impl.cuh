@@ -33,6 +33,9 @@ namespace f2 {
 #ifndef LUSYM_SWZ
 #define LUSYM_SWZ 1
 #endif
+#ifndef LUSYM_BATCH_TEST  // scan_level: load every neighbour's visited word before any atomic
+#define LUSYM_BATCH_TEST 0    // (A/B on B200: 3.7% slower on cfg2, 5% on cfg5 — kept as a knob)
+#endif
 #ifndef LUSYM_THREADS_PER_SM  // register budget: 65536 / this
 #define LUSYM_THREADS_PER_SM 2048
 #endif
@@ -349,7 +352,7 @@ struct RowAcc {
 // only the other discoveries go through the next-level queue.  Worth it only where a row has
 // an SM to itself and waits on each level's latency (the planner sets kloc per row class):
 // with many rows per SM the extra rounds, in which lanes drop out, cost issue slots.
-template <int NT, int W, int VIS>
+template <int NT, int W, int VIS, bool SC>
 __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm,
                                            uint32_t *sm, const int32_t *L, const int32_t *gL,
                                            int cnt, int *ncnt, int32_t *NF, int32_t *gNF,
@@ -357,6 +360,7 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
 {
     const int tid = threadIdx.x, lane = tid & 31;
     const unsigned lt = (1u << lane) - 1u;
+    const uint32_t ncnt_s = (uint32_t)__cvta_generic_to_shared(ncnt);
     unsigned nloc = 0;  // vertices expanded by self-continuation (statistics, lane 0)
     for (int base = 0; base < cnt; base += NT) {
         const int k = base + tid;
@@ -375,10 +379,22 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
             load_nb<W>(p.ell, f, nb);
             heavy = nb[0] == kHeavy;
             if (!heavy) {
+                // all W visited words first (independent loads in flight together), then the
+                // test-and-set only on the slots that looked unvisited (the atomic decides)
+                uint32_t um = 0;
+#pragma unroll
+                for (int s = 0; s < W; ++s) {
+#if LUSYM_BATCH_TEST
+                    const uint32_t wd = bm_word(bm, nb[s] >> 5);
+                    um |= ((~wd >> (nb[s] & 31)) & 1u) << s;
+#else
+                    um |= 1u << s;
+#endif
+                }
 #pragma unroll
                 for (int s = 0; s < W; ++s) {
                     const int w = nb[s];
-                    if (!visited(bm, w) && mark(bm, sm, w)) {
+                    if ((um >> s & 1u) && (LUSYM_BATCH_TEST || !visited(bm, w)) && mark(bm, sm, w)) {
                         if (w < t0) {
                             if (c == 3) {
                                 put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
@@ -396,24 +412,37 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                 }
             }
         }
-        // keep f0 for the next round, append the rest
-        const bool keep = r < p.kloc && c > 0;
-        if (keep) {
-            --c;
-            const int t = f0;
-            f0 = f1;
-            f1 = f2;
-            f2 = t;
+        // SC: keep f0 for the next round, append the rest
+        bool keep = false;
+        if constexpr (SC) {
+            keep = r < p.kloc && c > 0;
+            if (keep) {
+                --c;
+                const int t = f0;
+                f0 = f1;
+                f1 = f2;
+                f2 = t;
+            }
         }
         const unsigned b1 = __ballot_sync(kFull, c & 1), b2 = __ballot_sync(kFull, c & 2);
         if (b1 | b2) {
+            const int tot = __popc(b1) + 2 * __popc(b2);
             int wbase = 0;
-            if (lane == 0) wbase = atomicAdd(ncnt, __popc(b1) + 2 * __popc(b2));
+            // one shared atomic by lane 0 (inline PTX: no compiler re-aggregation around it)
+            if (lane == 0)
+                asm volatile("atom.shared.add.u32 %0, [%1], %2;"
+                             : "=r"(wbase) : "r"(ncnt_s), "r"(tot) : "memory");
             wbase = __shfl_sync(kFull, wbase, 0);
             const int pos = wbase + __popc(b1 & lt) + 2 * __popc(b2 & lt);
-            if (c) put(pos, f0, NF, gNF, p.q);
-            if (c >= 2) put(pos + 1, f1, NF, gNF, p.q);
-            if (c == 3) put(pos + 2, f2, NF, gNF, p.q);
+            if (wbase + tot <= p.q) {  // warp-uniform: the whole append lands in shared memory
+                if (c) NF[pos] = f0;
+                if (c >= 2) NF[pos + 1] = f1;
+                if (c == 3) NF[pos + 2] = f2;
+            } else {
+                if (c) put(pos, f0, NF, gNF, p.q);
+                if (c >= 2) put(pos + 1, f1, NF, gNF, p.q);
+                if (c == 3) put(pos + 2, f2, NF, gNF, p.q);
+            }
         }
         // heavy vertices (degree > W): one warp each, over A's CSR row
         unsigned hm = __ballot_sync(kFull, valid && heavy);
@@ -442,14 +471,18 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                 push(fr, w, ncnt, NF, gNF, p.q);
             }
         }
-        const unsigned kb = __ballot_sync(kFull, keep);
-        if (!kb) break;
-        nloc += __popc(kb);
-        valid = keep;
-        f = f2;
+        if constexpr (!SC) {
+            break;
+        } else {
+            const unsigned kb = __ballot_sync(kFull, keep);
+            if (!kb) break;
+            nloc += __popc(kb);
+            valid = keep;
+            f = f2;
+        }
       }
     }
-    if (lane == 0 && nloc) atomicAdd(&h.sv, (unsigned long long)nloc);
+    if (SC && lane == 0 && nloc) atomicAdd(&h.sv, (unsigned long long)nloc);
 }
 
 // Level-synchronous BFS from threshold t0 over unvisited vertices < t0 (Alg. 1).
@@ -473,9 +506,14 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_
         const int par = lev & 1;
         const int nxt = cur == 2 ? 0 : cur + 1;
         int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
-        scan_level<NT, W, VIS>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap, fsize,
-                               &h.cnt[nxt], qA + (par ^ 1) * p.q, gA + (par ^ 1) * p.spill_cap,
-                               i, t0, a);
+        if (p.kloc)
+            scan_level<NT, W, VIS, true>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
+                                         fsize, &h.cnt[nxt], qA + (par ^ 1) * p.q,
+                                         gA + (par ^ 1) * p.spill_cap, i, t0, a);
+        else
+            scan_level<NT, W, VIS, false>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
+                                          fsize, &h.cnt[nxt], qA + (par ^ 1) * p.q,
+                                          gA + (par ^ 1) * p.spill_cap, i, t0, a);
         __syncthreads();
         fsize = h.cnt[nxt];
         if (fsize == 0) break;
