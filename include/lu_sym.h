@@ -80,7 +80,7 @@ enum {
                                     with one row per SM                                       */
     LU_F_NO_SELF_CONT = 1 << 10, /* no self-continuation anywhere (plain level-synchronous
                                     BFS)                                                      */
-    LU_F_PAPER_CHUNKS = 1 << 11  /* Alg. 3's launch scheme (L239-243, L253-267): each pass is
+    LU_F_PAPER_CHUNKS = 1 << 11, /* Alg. 3's launch scheme (L239-243, L253-267): each pass is
                                     num_iter = ceil(rows / chunk_size) launches issued one
                                     after another, chunk_size = L / (c n) rows with c = 6
                                     4-byte words per vertex and L = the scratch budget (reading
@@ -88,6 +88,13 @@ enum {
                                     this is Alg. 3, without it Alg. 4 (one chunk size per row
                                     class).  Ablation of the persistent heaviest-first launch
                                                                                 */
+    LU_F_MANAGED = 1 << 12,      /* unified-memory variant (Figs 5-6,
+                                    Table 3): the traversal scratch (visited /
+                                    done maps, frontier spill, L staging, staging pool, row
+                                    offsets) comes from cudaMallocManaged and migrates to the
+                                    GPU on first touch (page faults)                         */
+    LU_F_MANAGED_PREFETCH = 1 << 13 /* with LU_F_MANAGED: cudaMemAdvise(preferred location =
+                                    this GPU) + cudaMemPrefetchAsync after each allocation    */
 };
 
 typedef struct {

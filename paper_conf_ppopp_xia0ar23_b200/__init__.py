@@ -40,6 +40,7 @@ DEP_U, DEP_GLU3 = 0, 1
 F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4, 8, 16
 F_NO_CONTRACT, F_TWO_PASS, F_ONE_CLASS, F_FORCE_CLASSES = 32, 64, 128, 256
 F_SELF_CONT, F_NO_SELF_CONT, F_PAPER_CHUNKS = 512, 1024, 2048
+F_MANAGED, F_MANAGED_PREFETCH = 4096, 8192
 
 
 class LuSymError(RuntimeError):

@@ -127,6 +127,7 @@ struct lu_sym {
     int64_t launches = 0;
     int64_t *row_prof = nullptr;  // borrowed, set by lu_sym_set_row_profile
     cudaStream_t stream = nullptr;  // stream of the last call (scratch is freed on it)
+    std::vector<void *> managed;    // LU_F_MANAGED scratch (freed with cudaFree)
 };
 
 namespace {
@@ -153,12 +154,54 @@ lu_status dalloc(lu_sym *h, T **p, size_t elems)
     return LU_OK;
 }
 
+bool is_managed(const lu_sym *h) { return (h->opts.flags & (LU_F_MANAGED | LU_F_MANAGED_PREFETCH)) != 0; }
+
+// Traversal scratch: device memory from the stream-ordered pool, or (LU_F_MANAGED, the
+// unified-memory variant of PAPER.md L237-239) cudaMallocManaged pages that migrate on first
+// touch, optionally advised to and prefetched onto this GPU (LU_F_MANAGED_PREFETCH).
+cudaError_t scratch_alloc_raw(lu_sym *h, void **p, size_t bytes)
+{
+    if (!is_managed(h)) return dev_alloc(p, bytes, h->stream);
+    cudaError_t e = cudaMallocManaged(p, bytes, cudaMemAttachGlobal);
+    if (e != cudaSuccess) return e;
+    h->managed.push_back(*p);
+    if (h->opts.flags & LU_F_MANAGED_PREFETCH) {
+        cudaMemLocation loc;
+        loc.type = cudaMemLocationTypeDevice;
+        loc.id = h->device;
+        if ((e = cudaMemAdvise(*p, bytes, cudaMemAdviseSetPreferredLocation, loc)) != cudaSuccess)
+            return e;
+        if ((e = cudaMemPrefetchAsync(*p, bytes, loc, 0, h->stream)) != cudaSuccess) return e;
+    }
+    return cudaSuccess;
+}
+
+template <class T>
+lu_status salloc(lu_sym *h, T **p, size_t elems)
+{
+    if (!is_managed(h)) return dalloc(h, p, elems);
+    size_t bytes = elems * sizeof(T);
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = scratch_alloc_raw(h, reinterpret_cast<void **>(p), bytes);
+    if (e != cudaSuccess)
+        return fail(LU_ERR_NOMEM, "cudaMallocManaged(%zu bytes): %s", bytes, cudaGetErrorString(e));
+    h->scratch_bytes += (int64_t)bytes;
+    return LU_OK;
+}
+
 void free_handle(lu_sym *h)
 {
     cudaStream_t s = h->stream;
     void *bufs[] = {h->ell, h->gbitmap, h->dbitmap, h->gspill, h->dstats, h->scan_blk, h->dbad,
                     h->stg, h->pool, h->row_off, h->unstaged};
-    for (void *b : bufs) dev_free(b, s);
+    if (!h->managed.empty()) cudaStreamSynchronize(s);
+    for (void *b : bufs) {
+        if (!b) continue;
+        if (std::find(h->managed.begin(), h->managed.end(), b) != h->managed.end())
+            cudaFree(b);
+        else
+            dev_free(b, s);
+    }
     levelize_free(h->lev, s);
     for (auto &c : h->classes) {
         if (c.stream) cudaStreamDestroy(c.stream);
@@ -327,17 +370,17 @@ lu_status plan(lu_sym *h)
     }
     h->grid = max_grid;
     h->map_words = (int64_t)need_map;
-    if ((st = dalloc(h, &h->gspill, need_spill)) != LU_OK) return st;
-    if (need_hbm_map && (st = dalloc(h, &h->gbitmap, need_map)) != LU_OK) return st;
-    if ((st = dalloc(h, &h->dbitmap, need_map)) != LU_OK) return st;
+    if ((st = salloc(h, &h->gspill, need_spill)) != LU_OK) return st;
+    if (need_hbm_map && (st = salloc(h, &h->gbitmap, need_map)) != LU_OK) return st;
+    if ((st = salloc(h, &h->dbitmap, need_map)) != LU_OK) return st;
     for (size_t k = 0; k < h->classes.size(); ++k) {
         CK(cudaEventCreateWithFlags(&h->classes[k].done, cudaEventDisableTiming));
         if (k > 0) CK(cudaStreamCreateWithFlags(&h->classes[k].stream, cudaStreamNonBlocking));
     }
-    if ((st = dalloc(h, &h->unstaged, (size_t)n)) != LU_OK) return st;
+    if ((st = salloc(h, &h->unstaged, (size_t)n)) != LU_OK) return st;
     if (h->staging) {
-        if ((st = dalloc(h, &h->stg, need_stg)) != LU_OK) return st;
-        if ((st = dalloc(h, &h->row_off, (size_t)n)) != LU_OK) return st;
+        if ((st = salloc(h, &h->stg, need_stg)) != LU_OK) return st;
+        if ((st = salloc(h, &h->row_off, (size_t)n)) != LU_OK) return st;
     }
     // summary fields (the top class)
     const RowClass &top = h->classes.front();
@@ -484,8 +527,8 @@ lu_status ensure_pool(lu_sym *h)
         h->pool_cap = -1;  // no room: every row is re-traversed by emit
         return LU_OK;
     }
-    cudaError_t e = dev_alloc(reinterpret_cast<void **>(&h->pool), (size_t)cap * sizeof(int32_t),
-                              h->stream);
+    cudaError_t e = scratch_alloc_raw(h, reinterpret_cast<void **>(&h->pool),
+                                      (size_t)cap * sizeof(int32_t));
     if (e != cudaSuccess) {
         cudaGetLastError();
         h->pool = nullptr;

@@ -25,5 +25,8 @@ for c in ${CFGS:-2 5 3}; do
   run $c 2   "NO_BATCH (one threshold at a time)"
   run $c 40  "NO_CONTRACT|NO_PRUNE (plain Alg.5 Kahn)"
   run $c 1   "GLOBAL_BITMAP (visited state in HBM)"
+  run $c 4096 "MANAGED (UM scratch, first-touch faults)"
+  run $c 8192 "MANAGED_PREFETCH (UM scratch, prefetched)"
+  run $c 4097 "MANAGED|GLOBAL_BITMAP (visited state in UM)"
   run $c 2283 "paper as printed (all of the above)"
 done

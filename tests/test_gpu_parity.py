@@ -157,6 +157,10 @@ KNOBS = [
     dict(flags=lu.F_PAPER_CHUNKS, scratch_budget_bytes=2_000_000),
     dict(flags=lu.F_PAPER_CHUNKS | lu.F_ONE_CLASS, scratch_budget_bytes=1_000_000),
     dict(flags=lu.F_PAPER_CHUNKS | lu.F_FORCE_CLASSES | lu.F_TWO_PASS, scratch_budget_bytes=3_000_000),
+    # unified-memory variant: scratch from cudaMallocManaged, +- prefetch
+    dict(flags=lu.F_MANAGED), dict(flags=lu.F_MANAGED_PREFETCH),
+    dict(flags=lu.F_MANAGED | lu.F_GLOBAL_BITMAP | lu.F_FORCE_CLASSES),
+    dict(flags=lu.F_MANAGED | lu.F_TWO_PASS, pool_bytes=200_000),
 ]
 
 
