@@ -47,6 +47,10 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-mode", default="pipelined", choices=["pipelined", "plain"],
+                    help="pipelined: lu_sym_run_host (pattern copied to the host behind the "
+                         "traversal, 1 GPU); plain: count/scan/emit then copies")
+    ap.add_argument("--e2e-chunks", type=int, default=0, help="lu_sym_run_host chunks (0 = the library default, 16)")
     ap.add_argument("--cpu-sample-stride", type=int, default=0,
                     help="oracle sample: every s-th row (0 = auto, ~10-30 s of CPU work)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras)")
@@ -375,6 +379,7 @@ def run_ours(args, rank, world, local_rank):
         out_lv = torch.empty(n, dtype=torch.int32).pin_memory()
         e_ms = []
         e_phase = {}
+        pipelined = args.e2e_mode == "pipelined" and world == 1
         for k in range(args.e2e_steps + 1):
             barrier()
             torch.cuda.synchronize()
@@ -392,24 +397,32 @@ def run_ours(args, rank, world, local_rank):
             mark("h2d")
             he = lu.Symbolic(rpd, cid, **sym_opts)             # S1 + S2 (validate, plan)
             mark("create")
-            fc = torch.zeros(n, dtype=torch.int32, device=dev)
-            he.count(rb, re_, fc)
-            if world > 1:
-                lu.assemble_counts(fc)
-            mark("count")
-            rp_lu, nz = he.scan(fc)
-            ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)
-            mark("scan+alloc")
-            he.emit(rp_lu, ci_lu, rb, re_)
-            if world > 1:
-                lu.assemble_pattern(ci_lu, rp_lu, bounds)
-            mark("emit")
-            level, _ = he.levelize(rp_lu, ci_lu, args.rule)
-            mark("levelize")
-            if rank == 0:
-                out_rp.copy_(rp_lu, non_blocking=True)
-                out_ci.copy_(ci_lu, non_blocking=True)
+            if pipelined:
+                # S3-S6 with the pattern streamed to pinned host memory behind the traversal
+                fc, rp_lu, ci_lu = he.run_host(nnz, out_rp, out_ci, nchunks=args.e2e_chunks)
+                mark("count+scan+emit+d2h(pattern)")
+                level, _ = he.levelize(rp_lu, ci_lu, args.rule)
+                mark("levelize")
                 out_lv.copy_(level, non_blocking=True)
+            else:
+                fc = torch.zeros(n, dtype=torch.int32, device=dev)
+                he.count(rb, re_, fc)
+                if world > 1:
+                    lu.assemble_counts(fc)
+                mark("count")
+                rp_lu, nz = he.scan(fc)
+                ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)
+                mark("scan+alloc")
+                he.emit(rp_lu, ci_lu, rb, re_)
+                if world > 1:
+                    lu.assemble_pattern(ci_lu, rp_lu, bounds)
+                mark("emit")
+                level, _ = he.levelize(rp_lu, ci_lu, args.rule)
+                mark("levelize")
+                if rank == 0:
+                    out_rp.copy_(rp_lu, non_blocking=True)
+                    out_ci.copy_(ci_lu, non_blocking=True)
+                    out_lv.copy_(level, non_blocking=True)
             b.record(stream)
             torch.cuda.synchronize()
             he.close()
@@ -427,6 +440,8 @@ def run_ours(args, rank, world, local_rank):
                "d2h_bytes_per_step": int((n + 1) * 8 + nnz * 4 + n * 4) if rank == 0 else 0,
                "ms_per_step": float(t.item()),
                "phases_ms": {k: float(np.mean(v)) for k, v in e_phase.items()},
+               "mode": "lu_sym_run_host (chunked count/scan/place, pattern D2H behind the "
+                       "traversal)" if pipelined else "count, scan, alloc, emit, then copies",
                "includes": "H2D of A, create (validate+adjacency+plan), count, scan, alloc, "
                            "emit, levelize, D2H of row_ptr/col_idx/level"}
 

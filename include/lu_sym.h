@@ -191,6 +191,28 @@ lu_status lu_sym_run(lu_sym *h, int32_t *d_fill_count, int64_t *d_row_ptr_lu,
                      int32_t *d_col_idx_lu, int64_t cap, int64_t *nnz_lu, void *stream);
 
 /*
+ * Whole symbolic pass with the result streamed to the host while later rows are still being
+ * traversed: Alg. 3's out-of-core chunks (L239-270) taken in INCREASING row order, nchunks row
+ * ranges of equal a-priori traversal cost (0 => 16; at most 64).  Per chunk: symbolic_1 with
+ * staging (the traversal; chunk k+1 runs on a second scratch set so it fills the SMs chunk k
+ * drains), the chained prefix sum of its counts (L262), symbolic_2 as a placement of its
+ * staged rows (L264-270) and the device->host copy of its rows, the last three behind the
+ * next chunks' traversal.
+ *   d_fill_count [n], d_row_ptr_lu [n+1], d_col_idx_lu [cap]: device outputs, as lu_sym_run.
+ *   h_row_ptr_lu [n+1], h_col_idx_lu [cap]: host copies (pinned memory overlaps the copies
+ *   with the traversal; pageable works but serialises); either may be NULL.
+ *   *nnz_lu (host) = nnz(L+U).  cap must be an upper bound of nnz(L+U) given up front;
+ *   cap < nnz: LU_ERR_CAPACITY with *nnz_lu, d_fill_count and d_row_ptr_lu valid.
+ * Blocks until the host copies are complete.  The handle is left scanned (lu_sym_emit and
+ * lu_levelize may follow).  With LU_F_TWO_PASS (no staging pool) it runs lu_sym_run's two
+ * calls and copies afterwards.  Allocates a second traversal scratch set on first use.
+ */
+lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
+                          int64_t *d_row_ptr_lu, int32_t *d_col_idx_lu, int64_t cap,
+                          int64_t *h_row_ptr_lu, int32_t *h_col_idx_lu, int64_t *nnz_lu,
+                          void *stream);
+
+/*
  * S8+S9 — levelization (Algorithm 5) of the column-dependency DAG of the pattern
  * (d_row_ptr_lu int64[n+1], d_col_idx_lu int32[nnz], rows sorted as lu_sym_emit writes them):
  *   d_level[j] = 0 if column j has no predecessor, else 1 + max level of its predecessors

@@ -81,7 +81,7 @@ _lib = None
 EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sym_count",
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
             "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile",
-            "lu_level_schedule"]
+            "lu_level_schedule", "lu_sym_run_host"]
 
 
 def library_path() -> str:
@@ -105,6 +105,7 @@ def load_library():
     lib.lu_sym_scan.argtypes = [P, P, P, P, P]
     lib.lu_sym_emit.argtypes = [P, I32, I32, P, P, I64, P]
     lib.lu_sym_run.argtypes = [P, P, P, P, I64, P, P]
+    lib.lu_sym_run_host.argtypes = [P, I32, P, P, P, I64, P, P, P, P]
     lib.lu_levelize.argtypes = [P, I32, P, P, I32, P, P, P]
     lib.lu_sym_get_stats.argtypes = [P, P]
     lib.lu_sym_destroy.argtypes = [P]
@@ -116,7 +117,7 @@ def load_library():
     lib.lu_status_str.restype = ctypes.c_char_p
     lib.lu_last_error.restype = ctypes.c_char_p
     for f in ("lu_sym_create", "lu_sym_count", "lu_sym_scan", "lu_sym_emit", "lu_sym_run",
-              "lu_levelize", "lu_sym_get_stats"):
+              "lu_levelize", "lu_sym_get_stats", "lu_sym_run_host"):
         getattr(lib, f).restype = I32
     if lib.lu_sym_abi_version() != 1:
         raise ImportError("liblusym.so ABI version mismatch")
@@ -240,6 +241,31 @@ class Symbolic:
         ci_lu = torch.empty(nnz, dtype=torch.int32, device=self.device)   # Alg. 3 line 8
         self.emit(rp_lu, ci_lu, stream=stream)
         return fc, rp_lu, ci_lu
+
+    def run_host(self, cap: int, host_row_ptr=None, host_col_idx=None, nchunks: int = 0,
+                 stream=None):
+        """S3-S6 with the pattern streamed to host memory behind the traversal
+        (lu_sym_run_host): row chunks in increasing order, each scanned, placed and copied to
+        the host while later chunks are traversed.  cap = capacity (>= nnz(L+U)) of the device
+        and host column arrays; host_* are CPU tensors (pinned for overlap) or None.
+        Returns (fill_count, row_ptr_lu, col_idx_lu[:nnz]) on the device."""
+        fc = torch.zeros(self.n, dtype=torch.int32, device=self.device)
+        rp_lu = torch.empty(self.n + 1, dtype=torch.int64, device=self.device)
+        ci_lu = torch.empty(max(cap, 1), dtype=torch.int32, device=self.device)
+        for t, dt, name, size in ((host_row_ptr, torch.int64, "host_row_ptr", self.n + 1),
+                                  (host_col_idx, torch.int32, "host_col_idx", cap)):
+            if t is not None and (t.is_cuda or t.dtype != dt or not t.is_contiguous()
+                                  or t.numel() < size):
+                raise ValueError(f"{name} must be a contiguous CPU {dt} tensor of >= {size}")
+        nnz = ctypes.c_int64(0)
+        _check(load_library().lu_sym_run_host(
+            self._h, nchunks, _dev(fc, torch.int32, "fill_count") if self.n else None,
+            _dev(rp_lu, torch.int64, "row_ptr_lu"), ctypes.c_void_p(ci_lu.data_ptr()), cap,
+            ctypes.c_void_p(host_row_ptr.data_ptr()) if host_row_ptr is not None else None,
+            ctypes.c_void_p(host_col_idx.data_ptr()) if host_col_idx is not None else None,
+            ctypes.byref(nnz), _stream_ptr(stream)))
+        self.nnz_lu = int(nnz.value)
+        return fc, rp_lu, ci_lu[: self.nnz_lu]
 
     def levelize(self, row_ptr_lu, col_idx_lu, rule: str = "u", level=None, stream=None):
         return levelize(row_ptr_lu, col_idx_lu, rule, level=level, handle=self, stream=stream)

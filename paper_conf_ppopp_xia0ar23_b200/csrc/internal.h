@@ -88,8 +88,10 @@ cudaError_t count_light(int32_t n, const int64_t *rp, const int32_t *ci, int w,
                         unsigned long long *d_cnt, cudaStream_t s);
 cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, int32_t *ell,
                       cudaStream_t s);
+// row_ptr[0..n] = exclusive prefix sum of counts[0..n); chained: offsets start at the value
+// row_ptr[0] holds on entry (a row block continuing an earlier one), else at 0
 cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,
-                        cudaStream_t s);
+                        cudaStream_t s, bool chained = false);
 size_t scan_scratch_elems(int32_t n);
 cudaError_t count_far_rows(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
                            unsigned long long *d_cnt, cudaStream_t s);

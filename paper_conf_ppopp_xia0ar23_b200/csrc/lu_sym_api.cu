@@ -62,7 +62,8 @@ lu_status fail(lu_status s, const char *fmt, ...)
     } while (0)
 
 enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvN = 4 };
-enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11, kSlotClassCounter = 16 };
+enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11, kSlotClassCounter = 16,
+       kSlotSetStride = 32, kStatSlots = 80, kMaxChunks = 64 };
 
 }  // namespace
 
@@ -128,6 +129,16 @@ struct lu_sym {
     int64_t *row_prof = nullptr;  // borrowed, set by lu_sym_set_row_profile
     cudaStream_t stream = nullptr;  // stream of the last call (scratch is freed on it)
     std::vector<void *> managed;    // LU_F_MANAGED scratch (freed with cudaFree)
+    // second traversal scratch set (lu_sym_run_host: two row chunks in flight at once, so the
+    // next chunk's CTAs take over SMs while the previous chunk drains); allocated on first use
+    int32_t *gspill1 = nullptr, *stg1 = nullptr;
+    uint32_t *gbitmap1 = nullptr, *dbitmap1 = nullptr;
+    std::vector<cudaStream_t> cls_stream1;
+    std::vector<cudaEvent_t> cls_done1;
+    cudaStream_t pipe_stream[3] = {};  // lu_sym_run_host: second count stream, place, copy
+    cudaEvent_t pipe_ev[4][kMaxChunks + 1] = {};  // count done, scanned, placed, copied
+    int64_t *pin = nullptr;                       // pinned host slot (chunk end offset)
+    std::vector<int32_t> chunk_bounds;            // lu_sym_run_host row chunks (cached)
 };
 
 namespace {
@@ -192,8 +203,9 @@ lu_status salloc(lu_sym *h, T **p, size_t elems)
 void free_handle(lu_sym *h)
 {
     cudaStream_t s = h->stream;
-    void *bufs[] = {h->ell, h->gbitmap, h->dbitmap, h->gspill, h->dstats, h->scan_blk, h->dbad,
-                    h->stg, h->pool, h->row_off, h->unstaged};
+    void *bufs[] = {h->ell,      h->gbitmap,  h->dbitmap, h->gspill, h->dstats,  h->scan_blk,
+                    h->dbad,     h->stg,      h->pool,    h->row_off, h->unstaged, h->gspill1,
+                    h->gbitmap1, h->dbitmap1, h->stg1};
     if (!h->managed.empty()) cudaStreamSynchronize(s);
     for (void *b : bufs) {
         if (!b) continue;
@@ -207,6 +219,16 @@ void free_handle(lu_sym *h)
         if (c.stream) cudaStreamDestroy(c.stream);
         if (c.done) cudaEventDestroy(c.done);
     }
+    for (auto cs : h->cls_stream1)
+        if (cs) cudaStreamDestroy(cs);
+    for (auto ce : h->cls_done1)
+        if (ce) cudaEventDestroy(ce);
+    for (auto ps : h->pipe_stream)
+        if (ps) cudaStreamDestroy(ps);
+    for (auto &row : h->pipe_ev)
+        for (auto pe : row)
+            if (pe) cudaEventDestroy(pe);
+    if (h->pin) cudaFreeHost(h->pin);
     for (int k = 0; k < kEvN; ++k)
         for (int j = 0; j < 2; ++j)
             if (h->ev[k][j]) cudaEventDestroy(h->ev[k][j]);
@@ -409,17 +431,24 @@ void ev_end(lu_sym *h, int k, cudaStream_t s)
 
 // One traversal pass over rows [rb, re) (or row_list): one launch per row class, top class
 // (heaviest rows) first, as Alg. 4 launches each part in turn.
+// set: traversal scratch set (0, or 1 = the second set of lu_sym_run_host); reset_stats: zero
+// the pass statistics first (a pipelined run accumulates over its chunks).
 lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_count,
                    const int64_t *rp_lu, int32_t *ci_lu, cudaStream_t s,
-                   const int32_t *row_list = nullptr, int32_t list_len = 0)
+                   const int32_t *row_list = nullptr, int32_t list_len = 0, int set = 0,
+                   bool reset_stats = true)
 {
     const bool emit = mode == kEmit;
     unsigned long long *st = h->dstats + (emit ? 5 : 1);
-    CK(cudaMemsetAsync(st, 0, sizeof(unsigned long long) * kStatCount, s));
-    if (h->gbitmap) CK(cudaMemsetAsync(h->gbitmap, 0, sizeof(uint32_t) * h->map_words, s));
-    CK(cudaMemsetAsync(h->dbitmap, 0, sizeof(uint32_t) * h->map_words, s));
-    CK(cudaMemsetAsync(h->dstats + kSlotClassCounter, 0,
-                       sizeof(unsigned long long) * h->classes.size(), s));
+    int32_t *gspill = set ? h->gspill1 : h->gspill;
+    int32_t *stg = set ? h->stg1 : h->stg;
+    uint32_t *gbitmap = set ? h->gbitmap1 : h->gbitmap;
+    uint32_t *dbitmap = set ? h->dbitmap1 : h->dbitmap;
+    unsigned long long *counters = h->dstats + kSlotClassCounter + set * kSlotSetStride;
+    if (reset_stats) CK(cudaMemsetAsync(st, 0, sizeof(unsigned long long) * kStatCount, s));
+    if (gbitmap) CK(cudaMemsetAsync(gbitmap, 0, sizeof(uint32_t) * h->map_words, s));
+    CK(cudaMemsetAsync(dbitmap, 0, sizeof(uint32_t) * h->map_words, s));
+    CK(cudaMemsetAsync(counters, 0, sizeof(unsigned long long) * h->classes.size(), s));
     if (h->row_prof && mode != kEmit && !row_list)
         CK(cudaMemsetAsync(h->row_prof + 4 * (size_t)rb, 0,
                            sizeof(int64_t) * 4 * (size_t)(re - rb), s));
@@ -454,23 +483,24 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
         if (rows <= 0) continue;
         cudaStream_t cs = s;
         if (k > 0) {
+            cudaEvent_t fork_ev = set ? h->cls_done1[0] : h->classes[0].done;
             if (!forked) {
-                CK(cudaEventRecord(h->classes[0].done, s));
+                CK(cudaEventRecord(fork_ev, s));
                 forked = true;
             }
-            cs = c.stream;
-            CK(cudaStreamWaitEvent(cs, h->classes[0].done, 0));
+            cs = set ? h->cls_stream1[k] : c.stream;
+            CK(cudaStreamWaitEvent(cs, fork_ev, 0));
         }
         p.row_begin = lo;
         p.row_end = hi;
         p.row_list = row_list;
         p.list_len = list_len;
         p.spill_cap = c.cap;
-        p.gspill = h->gspill + c.spill_off;
-        p.stg = h->stg ? h->stg + c.stg_off : nullptr;
-        p.gbitmap = h->gbitmap ? h->gbitmap + c.map_off : nullptr;
-        p.dbitmap = h->dbitmap + c.map_off;
-        p.row_counter = h->dstats + kSlotClassCounter + k;
+        p.gspill = gspill + c.spill_off;
+        p.stg = stg ? stg + c.stg_off : nullptr;
+        p.gbitmap = gbitmap ? gbitmap + c.map_off : nullptr;
+        p.dbitmap = dbitmap + c.map_off;
+        p.row_counter = counters + k;
         p.nw = c.smem_words;
         p.lbw = c.lbw;
         p.q = c.q;
@@ -503,9 +533,42 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     }
     if (forked)  // join
         for (size_t k = 1; k < h->classes.size(); ++k) {
-            CK(cudaEventRecord(h->classes[k].done, h->classes[k].stream));
-            CK(cudaStreamWaitEvent(s, h->classes[k].done, 0));
+            cudaEvent_t je = set ? h->cls_done1[k] : h->classes[k].done;
+            CK(cudaEventRecord(je, set ? h->cls_stream1[k] : h->classes[k].stream));
+            CK(cudaStreamWaitEvent(s, je, 0));
         }
+    return LU_OK;
+}
+
+// The second traversal scratch set (same sizes as the first), its class streams and the
+// pipeline's streams/events; allocated on the first lu_sym_run_host call.
+lu_status ensure_set1(lu_sym *h)
+{
+    if (h->dbitmap1) return LU_OK;
+    int64_t need_spill = 0, need_stg = 0;
+    for (auto &c : h->classes) {
+        need_spill = std::max<int64_t>(need_spill, c.spill_off + 2 * c.cap * (int64_t)c.grid);
+        need_stg = std::max<int64_t>(need_stg, c.stg_off + c.cap * (int64_t)c.grid);
+    }
+    lu_status st;
+    if ((st = salloc(h, &h->gspill1, (size_t)need_spill)) != LU_OK) return st;
+    if (h->gbitmap && (st = salloc(h, &h->gbitmap1, (size_t)h->map_words)) != LU_OK) return st;
+    if ((st = salloc(h, &h->dbitmap1, (size_t)h->map_words)) != LU_OK) return st;
+    if (h->staging && (st = salloc(h, &h->stg1, (size_t)need_stg)) != LU_OK) return st;
+    h->cls_stream1.assign(h->classes.size(), nullptr);
+    h->cls_done1.assign(h->classes.size(), nullptr);
+    for (size_t k = 0; k < h->classes.size(); ++k) {
+        CK(cudaEventCreateWithFlags(&h->cls_done1[k], cudaEventDisableTiming));
+        if (k > 0) CK(cudaStreamCreateWithFlags(&h->cls_stream1[k], cudaStreamNonBlocking));
+    }
+    int lo = 0, hi = 0;
+    CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    // [0] second count stream (normal priority); [1] scan + place and [2] device->host copies
+    // at the highest priority, so a chunk's placement CTAs go ahead of queued traversal CTAs
+    CK(cudaStreamCreateWithPriority(&h->pipe_stream[0], cudaStreamNonBlocking, lo));
+    CK(cudaStreamCreateWithPriority(&h->pipe_stream[1], cudaStreamNonBlocking, hi));
+    CK(cudaStreamCreateWithPriority(&h->pipe_stream[2], cudaStreamNonBlocking, hi));
+    CK(cudaMallocHost(reinterpret_cast<void **>(&h->pin), 2 * sizeof(int64_t)));
     return LU_OK;
 }
 
@@ -601,10 +664,10 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
     if (cudaEventCreate(&t0) != cudaSuccess || cudaEventCreate(&t1) != cudaSuccess)
         return bail(fail(LU_ERR_CUDA, "cudaEventCreate failed"));
     cudaEventRecord(t0, s);
-    if ((st = dalloc(h, &h->dstats, 32)) != LU_OK) return bail(st);
+    if ((st = dalloc(h, &h->dstats, kStatSlots)) != LU_OK) return bail(st);
     if ((st = dalloc(h, &h->dbad, 2)) != LU_OK) return bail(st);
     if ((st = dalloc(h, &h->scan_blk, scan_scratch_elems(n))) != LU_OK) return bail(st);
-    cudaMemsetAsync(h->dstats, 0, 32 * sizeof(unsigned long long), s);
+    cudaMemsetAsync(h->dstats, 0, kStatSlots * sizeof(unsigned long long), s);
     // S1: validate A
     {
         cudaError_t e = validate_csr(n, nnz_a, d_row_ptr, d_col_idx, h->dbad, s);
@@ -795,6 +858,172 @@ lu_status lu_sym_run(lu_sym *h, int32_t *d_fill_count, int64_t *d_row_ptr_lu,
         return fail(LU_ERR_CAPACITY, "cap %lld < nnz %lld", (long long)cap,
                     (long long)h->nnz_lu);
     return lu_sym_emit(h, 0, h->n, d_row_ptr_lu, d_col_idx_lu, cap, stream);
+}
+
+lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
+                          int64_t *d_row_ptr_lu, int32_t *d_col_idx_lu, int64_t cap,
+                          int64_t *h_row_ptr_lu, int32_t *h_col_idx_lu, int64_t *nnz_lu,
+                          void *stream)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    if (nchunks < 0 || nchunks > kMaxChunks)
+        return fail(LU_ERR_ARG, "nchunks %d outside [0,%d]", nchunks, (int)kMaxChunks);
+    if (cap < 0) return fail(LU_ERR_ARG, "cap < 0");
+    if (!d_row_ptr_lu || (h->n > 0 && (!d_fill_count || (cap > 0 && !d_col_idx_lu))))
+        return fail(LU_ERR_ARG, "null pointer");
+    lu_status st = check_device(h);
+    if (st != LU_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    h->stream = s;
+    const int32_t n = h->n;
+    if (nchunks == 0) nchunks = 16;
+    if (nchunks > n) nchunks = n > 0 ? n : 1;
+    if (h->staging) {
+        if ((st = ensure_pool(h)) != LU_OK) return st;
+    }
+    if (!h->staging || !h->pool || n == 0) {
+        // two-pass mode (or no pool): the plain calls, then the copies
+        int64_t nnz = 0;
+        if ((st = lu_sym_run(h, d_fill_count, d_row_ptr_lu, nullptr, 0, &nnz, stream)) != LU_OK)
+            return st;
+        if (nnz_lu) *nnz_lu = nnz;
+        if (cap < nnz)
+            return fail(LU_ERR_CAPACITY, "cap %lld < nnz %lld", (long long)cap, (long long)nnz);
+        if (nnz > 0 && (st = lu_sym_run(h, d_fill_count, d_row_ptr_lu, d_col_idx_lu, cap, &nnz,
+                                         stream)) != LU_OK)
+            return st;
+        if (h_row_ptr_lu)
+            CK(cudaMemcpyAsync(h_row_ptr_lu, d_row_ptr_lu, sizeof(int64_t) * ((size_t)n + 1),
+                               cudaMemcpyDeviceToHost, s));
+        if (h_col_idx_lu && nnz > 0)
+            CK(cudaMemcpyAsync(h_col_idx_lu, d_col_idx_lu, sizeof(int32_t) * (size_t)nnz,
+                               cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        return LU_OK;
+    }
+    if ((st = ensure_set1(h)) != LU_OK) return st;
+    // row chunks of equal a-priori traversal cost (row_ptr[i+1]: the TE bound of row i, exact on
+    // the grids), in increasing row order so that each chunk's offsets follow its predecessor's
+    if ((int)h->chunk_bounds.size() != nchunks + 1) {
+        std::vector<int64_t> rp((size_t)n + 1);
+        CK(cudaMemcpyAsync(rp.data(), h->rp, sizeof(int64_t) * rp.size(), cudaMemcpyDeviceToHost,
+                           s));
+        CK(cudaStreamSynchronize(s));
+        double total = 0;
+        for (int32_t i = 0; i < n; ++i) total += (double)rp[(size_t)i + 1] + 1.0;
+        h->chunk_bounds.assign(1, 0);
+        double acc = 0;
+        for (int32_t i = 0; i < n && (int)h->chunk_bounds.size() < nchunks; ++i) {
+            acc += (double)rp[(size_t)i + 1] + 1.0;
+            if (acc >= total * (double)h->chunk_bounds.size() / nchunks &&
+                i + 1 > h->chunk_bounds.back())
+                h->chunk_bounds.push_back(i + 1);
+        }
+        while ((int)h->chunk_bounds.size() < nchunks + 1) h->chunk_bounds.push_back(n);
+        h->chunk_bounds.back() = n;
+    }
+    const std::vector<int32_t> &b = h->chunk_bounds;
+    for (auto &row : h->pipe_ev)  // events of chunks 0..nchunks-1 and the fork slot
+        for (int k = 0; k <= kMaxChunks; ++k)
+            if (!row[k] && (k < nchunks || k == kMaxChunks))
+                CK(cudaEventCreateWithFlags(&row[k], cudaEventDisableTiming));
+    cudaStream_t cs[2] = {s, h->pipe_stream[0]};
+    cudaStream_t sp = h->pipe_stream[1], sc = h->pipe_stream[2];
+    cudaEvent_t *ev_count = h->pipe_ev[0], *ev_scan = h->pipe_ev[1], *ev_place = h->pipe_ev[2],
+                *ev_copy = h->pipe_ev[3];
+    ev_begin(h, kEvCount, s);
+    // a fresh staging pool, statistics and row_ptr_lu[0] = 0, then fork the pipeline streams
+    h->staged.clear();
+    h->staged.emplace_back(0, n);
+    h->scanned = false;
+    CK(cudaMemsetAsync(h->row_off, 0xff, sizeof(int64_t) * (size_t)n, s));
+    CK(cudaMemsetAsync(h->dstats + kSlotPoolCursor, 0, 2 * sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(h->dstats + 1, 0, sizeof(unsigned long long) * kStatCount, s));
+    CK(cudaMemsetAsync(d_row_ptr_lu, 0, sizeof(int64_t), s));
+    CK(cudaEventRecord(ev_count[kMaxChunks], s));
+    for (cudaStream_t x : {cs[1], sp, sc}) CK(cudaStreamWaitEvent(x, ev_count[kMaxChunks], 0));
+    // symbolic_1 with staging, chunk k on scratch set k & 1: chunk k+1's CTAs fill the SMs that
+    // chunk k's CTAs leave while it drains
+    for (int k = 0; k < nchunks; ++k) {
+        if (b[k] < b[k + 1] &&
+            (st = run_pass(h, kStage, b[k], b[k + 1], d_fill_count, nullptr, nullptr, cs[k & 1],
+                           nullptr, 0, k & 1, false)) != LU_OK)
+            return st;
+        CK(cudaEventRecord(ev_count[k], cs[k & 1]));
+    }
+    if (nchunks > 1) CK(cudaStreamWaitEvent(s, ev_count[nchunks - 1 - ((nchunks - 1) & 1 ? 0 : 1)], 0));
+    CK(cudaEventRecord(h->ev[kEvCount][1], s));  // s now follows every chunk's traversal
+    h->ev_used[kEvCount] = true;
+    // per chunk, behind its traversal: chained prefix sum, placement (symbolic_2 of staged
+    // rows) and the device->host copies of its rows
+    int64_t base = 0;
+    bool overflow = false;
+    ev_begin(h, kEvEmit, sp);
+    for (int k = 0; k < nchunks; ++k) {
+        const int32_t r0 = b[k], r1 = b[k + 1];
+        CK(cudaStreamWaitEvent(sp, ev_count[k], 0));
+        CK(scan_counts(r1 - r0, d_fill_count + r0, d_row_ptr_lu + r0, h->scan_blk, sp, true));
+        h->launches += r1 > r0 ? 3 : 1;
+        CK(cudaMemcpyAsync(h->pin, d_row_ptr_lu + r1, sizeof(int64_t), cudaMemcpyDeviceToHost,
+                           sp));
+        CK(cudaEventRecord(ev_scan[k], sp));
+        CK(cudaEventSynchronize(ev_scan[k]));
+        const int64_t end = h->pin[0];
+        if (end > cap) overflow = true;
+        if (!overflow) {
+            CK(place_rows(r0, r1, d_row_ptr_lu, h->row_off, h->pool, d_col_idx_lu, base,
+                          end - base, sp));
+            h->launches += end > base ? 1 : 0;
+        }
+        CK(cudaEventRecord(ev_place[k], sp));
+        CK(cudaStreamWaitEvent(sc, ev_place[k], 0));
+        if (h_row_ptr_lu)
+            CK(cudaMemcpyAsync(h_row_ptr_lu + r0, d_row_ptr_lu + r0,
+                               sizeof(int64_t) * ((size_t)(r1 - r0) + (k == nchunks - 1)),
+                               cudaMemcpyDeviceToHost, sc));
+        if (h_col_idx_lu && !overflow && end > base)
+            CK(cudaMemcpyAsync(h_col_idx_lu + base, d_col_idx_lu + base,
+                               sizeof(int32_t) * (size_t)(end - base), cudaMemcpyDeviceToHost, sc));
+        CK(cudaEventRecord(ev_copy[k], sc));
+        base = end;
+    }
+    const int64_t nnz = base;
+    CK(cudaEventRecord(h->ev[kEvEmit][1], sp));
+    h->ev_used[kEvEmit] = true;
+    // join everything into the caller's stream
+    CK(cudaStreamWaitEvent(s, ev_place[nchunks - 1], 0));
+    CK(cudaStreamWaitEvent(s, ev_copy[nchunks - 1], 0));
+    h->nnz_lu = nnz;
+    h->stats.nnz_lu = nnz;
+    h->scanned = true;
+    if (nnz_lu) *nnz_lu = nnz;
+    if (overflow) {
+        CK(cudaStreamSynchronize(s));
+        return fail(LU_ERR_CAPACITY, "cap %lld < nnz %lld", (long long)cap, (long long)nnz);
+    }
+    // rows that did not fit the staging pool: symbolic_2 by traversal, then copy everything
+    CK(collect_unstaged(0, n, h->row_off, h->unstaged, h->dstats + kSlotList, s));
+    unsigned long long nun = 0;
+    CK(cudaMemcpyAsync(&nun, h->dstats + kSlotList, 8, cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    h->launches += 1;
+    h->stats.rows_retraversed = (int64_t)nun;
+    if (nun > 0) {
+        if ((st = run_pass(h, kEmit, 0, n, nullptr, d_row_ptr_lu, d_col_idx_lu, s, h->unstaged,
+                           (int32_t)nun)) != LU_OK)
+            return st;
+        if (h_col_idx_lu && nnz > 0)
+            CK(cudaMemcpyAsync(h_col_idx_lu, d_col_idx_lu, sizeof(int32_t) * (size_t)nnz,
+                               cudaMemcpyDeviceToHost, s));
+        unsigned long long err = 0;
+        CK(cudaMemcpyAsync(&err, h->dstats + 5 + kStatErr, 8, cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        if (err)
+            return fail(LU_ERR_INTERNAL, "%llu rows emitted a length different from their count",
+                        err);
+    }
+    return LU_OK;
 }
 
 lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,

@@ -172,10 +172,11 @@ __global__ void __launch_bounds__(kScanNT) k_scan_tiles(int32_t n, const int32_t
 }
 
 __global__ void __launch_bounds__(kScanNT) k_scan_blocks(int64_t nb, int64_t *blk,
-                                                         int64_t *row_ptr_n)
+                                                         int64_t *row_ptr_n,
+                                                         const int64_t *carry_in)
 {
     __shared__ long long s[32];
-    long long carry = 0;
+    long long carry = carry_in ? *carry_in : 0;  // chained scan: offsets continue from row_ptr[0]
     for (int64_t b0 = 0; b0 < nb; b0 += kScanNT) {
         const int64_t b = b0 + threadIdx.x;
         const long long v = b < nb ? blk[b] : 0;
@@ -260,7 +261,7 @@ size_t scan_scratch_elems(int32_t n)
 }
 
 cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,
-                        cudaStream_t s)
+                        cudaStream_t s, bool chained)
 {
     const int64_t nb = ((int64_t)n + kScanTile - 1) / kScanTile;
     if (nb > 0) {
@@ -268,7 +269,7 @@ cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int6
         cudaError_t e = cudaGetLastError();
         if (e != cudaSuccess) return e;
     }
-    k_scan_blocks<<<1, kScanNT, 0, s>>>(nb, blk, row_ptr + n);
+    k_scan_blocks<<<1, kScanNT, 0, s>>>(nb, blk, row_ptr + n, chained ? row_ptr : nullptr);
     cudaError_t e = cudaGetLastError();
     if (e != cudaSuccess || nb == 0) return e;
     k_scan_final<<<(unsigned)nb, kScanNT, 0, s>>>(n, counts, blk, row_ptr);

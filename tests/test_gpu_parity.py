@@ -390,3 +390,50 @@ def test_cfg45_closed_forms(cfg):
     assert nl == n
     assert torch.equal(lv, torch.arange(n, dtype=torch.int32, device=d))
     h.close()
+
+
+# ---------------------------------------------------------------- pipelined run to host memory
+@pytest.mark.parametrize("nchunks,knob", [(0, {}), (1, {}), (3, {}), (17, {}), (64, {}),
+                                          (5, dict(flags=lu.F_FORCE_CLASSES)),
+                                          (4, dict(flags=lu.F_TWO_PASS)),
+                                          (6, dict(pool_bytes=60_000)),
+                                          (7, dict(queue_capacity=32, rows_in_flight=9)),
+                                          (3, dict(flags=lu.F_MANAGED))])
+def test_run_host_pipelined(nchunks, knob):
+    """lu_sym_run_host: chunked count -> chained scan -> place -> D2H, bit-exact on the device
+    and host copies, repeated on the same handle (fresh pool and scratch sets each call)."""
+    d = dev()
+    for rp, ci in (gen.lap3d(11), gen.circuit(48, 7), gen.random_pattern(900, 2.0, seed=5),
+                   gen.lap2d(1), gen.random_pattern(40, 0.5, seed=1)):
+        ref = oracle.fill2(rp, ci)
+        nnz = int(ref["row_ptr"][-1])
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d), **knob)
+        for rep in range(2):
+            hr = torch.full((len(rp),), -7, dtype=torch.int64).pin_memory()
+            hc = torch.full((nnz + 5,), -7, dtype=torch.int32).pin_memory()
+            fc, rp_lu, ci_lu = h.run_host(nnz + 5, hr, hc, nchunks=nchunks)
+            torch.cuda.synchronize()
+            assert h.nnz_lu == nnz
+            assert np.array_equal(fc.cpu().numpy(), ref["counts"])
+            assert np.array_equal(rp_lu.cpu().numpy(), ref["row_ptr"])
+            assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+            assert np.array_equal(hr.numpy(), ref["row_ptr"])
+            assert np.array_equal(hc.numpy()[:nnz], ref["col_idx"])
+            lv, nl = h.levelize(rp_lu, ci_lu, "u")
+            assert np.array_equal(lv.cpu().numpy(), oracle.levels(ref["row_ptr"],
+                                                                  ref["col_idx"], "u")[0])
+        h.close()
+
+
+def test_run_host_capacity():
+    d = dev()
+    rp, ci = gen.lap3d(8)
+    ref = oracle.fill2(rp, ci)
+    nnz = int(ref["row_ptr"][-1])
+    h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+    with pytest.raises(lu.LuSymError) as e:
+        h.run_host(nnz - 1, nchunks=4)
+    assert e.value.status == lu.LU_ERR_CAPACITY
+    fc, rp_lu, ci_lu = h.run_host(nnz, nchunks=4)   # the handle stays usable
+    assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+    h.close()
