@@ -107,3 +107,39 @@ def levels(row_ptr_lu, col_idx_lu, rule: str = "u"):
     if rc == -2:
         raise ValueError("dependency graph has a cycle")
     return lvl, int(rc)
+
+
+# GLU3.0 level types, reading R28: the sub-columns of column j are
+# the columns k > j with As(j,k) != 0 — the columns Alg. 2 lines 7-14 update from column j
+# (L165-204), i.e. column j's out-edges in the U-rule dependency graph (L167).
+LEVEL_A, LEVEL_B, LEVEL_C = 0, 1, 2
+
+
+def level_types(row_ptr_lu, col_idx_lu, level, num_levels, min_cols, max_sub_a):
+    """Per level l: width[l] = number of columns, sub[l] = total sub-columns of its columns;
+    type[l] = C if width < min_cols ("a limited number of columns"), else A if
+    sub <= max_sub_a * width ("very few associated sub-columns" per column), else B ("great
+    numbers of columns ... also many sub-columns").  Plain loops; returns (type, sub, width)."""
+    rp = np.asarray(row_ptr_lu, dtype=np.int64)
+    ci = np.asarray(col_idx_lu)
+    lv = np.asarray(level)
+    n = len(rp) - 1
+    width = [0] * num_levels
+    sub = [0] * num_levels
+    for j in range(n):
+        u = 0
+        for p in range(rp[j], rp[j + 1]):
+            if ci[p] > j:
+                u += 1
+        width[lv[j]] += 1
+        sub[lv[j]] += u
+    typ = []
+    for l in range(num_levels):
+        if width[l] < min_cols:
+            typ.append(LEVEL_C)
+        elif sub[l] <= max_sub_a * width[l]:
+            typ.append(LEVEL_A)
+        else:
+            typ.append(LEVEL_B)
+    return (np.array(typ, dtype=np.int32), np.array(sub, dtype=np.int64),
+            np.array(width, dtype=np.int64))

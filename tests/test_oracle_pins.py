@@ -270,3 +270,70 @@ def test_row_subset_matches_full():
     sr = pins.csr_rows(sub["row_ptr"], sub["col_idx"])
     assert sr == [fr[i] for i in rows]
     assert np.array_equal(sub["te"], full["te"][rows])
+
+
+# ---------------------------------------------------------------- GLU3.0 level types (f3)
+def test_level_types_against_bge_dense_rows():
+    """Sub-columns per level (Alg. 2 lines 7-14: column j updates every k > j with As(j,k) != 0,
+    reading R28) from BGE's dense pattern and the index-order level DP, vs the oracle."""
+    rng = np.random.default_rng(99)
+    for case in range(150):
+        n = int(rng.integers(1, 40))
+        rp, ci = gen.random_pattern(n, float(rng.uniform(0.3, 3)), seed=77_000 + case,
+                                    sym_frac=float(rng.uniform(0, 1)))
+        P = pins.bge(pins.to_dense(rp, ci))
+        sub_col = np.triu(P, 1).sum(axis=1)                     # strict-U row counts
+        E = [(i, j) for i in range(n) for j in range(i + 1, n) if P[i, j]]
+        lv = pins.levels_dp(n, E)
+        nl = int(lv.max()) + 1 if n else 0
+        r = oracle.fill2(rp, ci)
+        lvo, nlo = oracle.levels(r["row_ptr"], r["col_idx"], "u")
+        assert nlo == nl and np.array_equal(lvo, lv)
+        mc, ms = int(rng.integers(0, 6)), int(rng.integers(0, 5))
+        typ, sub, width = oracle.level_types(r["row_ptr"], r["col_idx"], lvo, nl, mc, ms)
+        assert np.array_equal(width, np.bincount(lv, minlength=nl))
+        assert np.array_equal(sub, np.bincount(lv, weights=sub_col, minlength=nl).astype(np.int64))
+        # the three regimes of L208, at the extremes of the two thresholds
+        assert np.all(oracle.level_types(r["row_ptr"], r["col_idx"], lvo, nl, n + 1, 0)[0] == 2)
+        assert np.all(oracle.level_types(r["row_ptr"], r["col_idx"], lvo, nl, 0, n)[0] == 0)
+        tb = oracle.level_types(r["row_ptr"], r["col_idx"], lvo, nl, 0, -1)[0]
+        assert np.all(tb == 1)
+
+
+def test_level_types_2d_grid_closed_form():
+    """Natural-order 2D grid: rows of L+U in closed form (pins.closed_form_2d), levels are the
+    chain 0..n-1, so level l holds column l with its strict-U count as sub-columns (k in the
+    interior, i+2 in the first grid row, n-1-l in the last): every level is type C for
+    min_cols >= 2, and the A/B split follows max_sub_a exactly."""
+    k = 9
+    rp, ci = gen.lap2d(k)
+    n = k * k
+    r = oracle.fill2(rp, ci)
+    lv, nl = oracle.levels(r["row_ptr"], r["col_idx"], "u")
+    assert nl == n and np.array_equal(lv, np.arange(n))
+    expect_sub = np.array([sum(1 for c in row if c > l)
+                           for l, row in enumerate(pins.closed_form_2d(k))], dtype=np.int64)
+    assert expect_sub.max() == k and expect_sub[0] == 2 and expect_sub[-1] == 0
+    typ, sub, width = oracle.level_types(r["row_ptr"], r["col_idx"], lv, nl, 2, 4)
+    assert np.array_equal(sub, expect_sub) and np.all(width == 1) and np.all(typ == 2)
+    typ, _, _ = oracle.level_types(r["row_ptr"], r["col_idx"], lv, nl, 1, k - 1)
+    assert np.array_equal(typ, np.where(expect_sub <= k - 1, 0, 1))
+
+
+def test_level_types_fig1():
+    """Fig. 1 fixture: level widths are the printed table's (Fig. 1(d), L72-78: {1,2,3,6,7},
+    {4,5}, {8}, {9}, {10}); sub-columns are the dependency graph's out-degrees (Fig. 1(b))."""
+    A, fills, table = pins.read_fig1_golden(GOLDEN)
+    R = [r for r, cs in A.items() for _ in cs]
+    C = [c for r, cs in A.items() for c in cs]
+    rp, ci = gen.csr_from_edges(10, R, C)
+    r = oracle.fill2(rp, ci)
+    lv, nl = oracle.levels(r["row_ptr"], r["col_idx"], "u")
+    typ, sub, width = oracle.level_types(r["row_ptr"], r["col_idx"], lv, nl, 2, 1)
+    assert list(width) == [5, 2, 1, 1, 1]
+    outdeg = np.zeros(10, dtype=np.int64)
+    for i, j in pins.dep_edges(r["row_ptr"], r["col_idx"], "u"):
+        outdeg[i] += 1
+    assert list(sub) == [int(outdeg[[c for c in range(10) if table[c] == l]].sum())
+                         for l in range(5)]
+    assert list(typ[2:]) == [2, 2, 2]
