@@ -234,6 +234,25 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
 lu_status lu_level_schedule(int32_t n, const int32_t *d_level, int32_t num_levels,
                             int64_t *d_level_ptr, int32_t *d_level_cols, void *stream);
 
+/*
+ * GLU3.0 level types, the per-level kernel-mode choice of the
+ * numeric phase.  For level l (levels from lu_levelize): width = number of its columns,
+ * d_sub[l] = total sub-columns of its columns, where the sub-columns of column j are the
+ * columns k > j with (j,k) in L+U — the columns Alg. 2 (lines 7-14, L165-204) updates from
+ * column j, i.e. its out-edges under LU_DEP_U (reading R28).  d_type[l] =
+ *   LU_LEVEL_C  if width < min_cols                 ("a limited number of columns"),
+ *   LU_LEVEL_A  else if sub <= max_sub_a * width    ("very few associated sub-columns"),
+ *   LU_LEVEL_B  otherwise                           (many columns, many sub-columns).
+ * min_cols <= 0 => the device's SM count (fewer columns than SMs cannot fill the GPU with one
+ * CTA per column); max_sub_a <= 0 => 32 (one warp per sub-column fits one CTA per column).
+ * d_row_ptr_lu / d_col_idx_lu: CSR of L+U, rows sorted; d_level[n]; d_type int32[num_levels];
+ * d_sub int64[num_levels] or NULL.  Synchronises.  LU_ERR_ARG on null pointers / bad sizes.
+ */
+enum { LU_LEVEL_A = 0, LU_LEVEL_B = 1, LU_LEVEL_C = 2 };
+lu_status lu_level_types(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
+                         const int32_t *d_level, int32_t num_levels, int32_t min_cols,
+                         int32_t max_sub_a, int32_t *d_type, int64_t *d_sub, void *stream);
+
 /* Copy the handle's statistics to *out (host). */
 lu_status lu_sym_get_stats(const lu_sym *h, lu_sym_stats *out);
 

@@ -81,7 +81,7 @@ _lib = None
 EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sym_count",
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
             "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile",
-            "lu_level_schedule", "lu_sym_run_host"]
+            "lu_level_schedule", "lu_sym_run_host", "lu_level_types"]
 
 
 def library_path() -> str:
@@ -112,6 +112,8 @@ def load_library():
     lib.lu_sym_set_row_profile.argtypes = [P, P]
     lib.lu_level_schedule.argtypes = [I32, P, I32, P, P, P]
     lib.lu_level_schedule.restype = I32
+    lib.lu_level_types.argtypes = [I32, P, P, P, I32, I32, I32, P, P, P]
+    lib.lu_level_types.restype = I32
     lib.lu_sym_set_row_profile.restype = I32
     lib.lu_status_str.argtypes = [I32]
     lib.lu_status_str.restype = ctypes.c_char_p
@@ -331,6 +333,27 @@ def level_schedule(level: torch.Tensor, num_levels: int, stream=None):
         _dev(level_ptr, torch.int64, "level_ptr"),
         ctypes.c_void_p(level_cols.data_ptr()) if n else None, _stream_ptr(stream)))
     return level_ptr, level_cols
+
+
+LEVEL_A, LEVEL_B, LEVEL_C = 0, 1, 2
+
+
+def level_types(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, level: torch.Tensor,
+                num_levels: int, min_cols: int = 0, max_sub_a: int = 0, stream=None):
+    """GLU3.0 level types (L208; lu_level_types): (type int32[num_levels] with LEVEL_A/B/C,
+    sub-columns int64[num_levels]) on the device.  min_cols <= 0: the SM count; max_sub_a <= 0:
+    32."""
+    n = int(row_ptr_lu.numel()) - 1
+    dev = row_ptr_lu.device
+    typ = torch.empty(max(num_levels, 1), dtype=torch.int32, device=dev)[:num_levels]
+    sub = torch.empty(max(num_levels, 1), dtype=torch.int64, device=dev)[:num_levels]
+    ci = ctypes.c_void_p(col_idx_lu.data_ptr()) if col_idx_lu.numel() else None
+    _check(load_library().lu_level_types(
+        n, _dev(row_ptr_lu, torch.int64, "row_ptr_lu"), ci,
+        _dev(level, torch.int32, "level") if n else None, num_levels, min_cols, max_sub_a,
+        ctypes.c_void_p(typ.data_ptr()) if num_levels else None,
+        ctypes.c_void_p(sub.data_ptr()) if num_levels else None, _stream_ptr(stream)))
+    return typ, sub
 
 
 def symbolic_distributed(row_ptr: torch.Tensor, col_idx: torch.Tensor, group=None,

@@ -105,6 +105,9 @@ cudaError_t collect_unstaged(int32_t row_begin, int32_t row_end, const int64_t *
                              int32_t *list, unsigned long long *cnt, cudaStream_t s);
 
 // schedule_kernels.cu — columns grouped by level (Fig. 1(d) form)
+cudaError_t level_types(int32_t n, const int64_t *rp, const int32_t *ci, const int32_t *level,
+                        int32_t num_levels, int32_t min_cols, int32_t max_sub_a, int32_t *type,
+                        int64_t *sub, cudaStream_t s);
 cudaError_t level_schedule(int32_t n, const int32_t *level, int32_t num_levels,
                            int64_t *level_ptr, int32_t *level_cols, cudaStream_t s);
 

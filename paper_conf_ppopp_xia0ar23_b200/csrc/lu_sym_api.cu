@@ -1082,6 +1082,28 @@ lu_status lu_level_schedule(int32_t n, const int32_t *d_level, int32_t num_level
     return LU_OK;
 }
 
+lu_status lu_level_types(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
+                         const int32_t *d_level, int32_t num_levels, int32_t min_cols,
+                         int32_t max_sub_a, int32_t *d_type, int64_t *d_sub, void *stream)
+{
+    g_err.clear();
+    if (n < 0 || num_levels < 0) return fail(LU_ERR_ARG, "negative size");
+    if (n > 0 && num_levels < 1) return fail(LU_ERR_ARG, "num_levels must be >= 1 when n > 0");
+    if (num_levels > 0 && (!d_type || !d_row_ptr_lu || (n > 0 && (!d_level || !d_col_idx_lu))))
+        return fail(LU_ERR_ARG, "null pointer");
+    if (min_cols <= 0) {
+        int dev = 0;
+        CK(cudaGetDevice(&dev));
+        CK(cudaDeviceGetAttribute(&min_cols, cudaDevAttrMultiProcessorCount, dev));
+    }
+    if (max_sub_a <= 0) max_sub_a = 32;
+    cudaStream_t s = (cudaStream_t)stream;
+    CK(level_types(n, d_row_ptr_lu, d_col_idx_lu, d_level, num_levels, min_cols, max_sub_a,
+                   d_type, d_sub, s));
+    CK(cudaStreamSynchronize(s));
+    return LU_OK;
+}
+
 lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
 {
     g_err.clear();

@@ -2,7 +2,8 @@
 // PAPER.md Fig. 1(d) (L72-80, "Column ids for different levels") that the numeric phase's
 // level-by-level launches consume (L206-208).  level_ptr[l] .. level_ptr[l+1] delimit the
 // columns of level l in level_cols, ascending within a level (reading R15).  Not on the hot
-// path: a stable radix sort of (level, column) pairs from CUB does the grouping.
+// path: a stable radix sort of (level, column) pairs from CUB does the grouping.  Also the
+// GLU3.0 level types A/B/C (L208) that choose the numeric kernel mode per level.
 #include "internal.h"
 
 #include <cub/device/device_radix_sort.cuh>
@@ -29,7 +30,64 @@ __global__ void k_level_ptr(int32_t n, const int32_t *sorted_level, int32_t num_
         for (int k = l + 1; k <= num_levels; ++k) level_ptr[k] = n;
 }
 
+// GLU3.0 level types (L208): one thread per column j — its sub-columns (reading R28: the
+// strict-U entries of row j, As(j,k) != 0 with k > j, Alg. 2 lines 7-14) are the entries of the
+// sorted row past the binary-searched position of j; width and sub-columns are accumulated per
+// level with integer atomics (exact, order-free).
+__global__ void k_level_sub(int32_t n, const int64_t *rp, const int32_t *ci, const int32_t *level,
+                            unsigned long long *lsub, unsigned int *lwidth)
+{
+    const int j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j >= n) return;
+    int64_t lo = rp[j], hi = rp[j + 1];
+    const int64_t end = hi;
+    while (lo < hi) {  // first entry > j
+        const int64_t mid = (lo + hi) >> 1;
+        if (ci[mid] <= j) lo = mid + 1; else hi = mid;
+    }
+    const int l = level[j];
+    atomicAdd(&lsub[l], (unsigned long long)(end - lo));
+    atomicAdd(&lwidth[l], 1u);
+}
+
+__global__ void k_level_type(int32_t num_levels, const unsigned long long *lsub,
+                             const unsigned int *lwidth, int32_t min_cols, int32_t max_sub_a,
+                             int32_t *type, int64_t *sub_out)
+{
+    const int l = blockIdx.x * blockDim.x + threadIdx.x;
+    if (l >= num_levels) return;
+    const long long w = lwidth[l], sb = (long long)lsub[l];
+    type[l] = w < min_cols ? 2 : (sb <= (long long)max_sub_a * w ? 0 : 1);
+    if (sub_out) sub_out[l] = sb;
+}
+
 }  // namespace
+
+cudaError_t level_types(int32_t n, const int64_t *rp, const int32_t *ci, const int32_t *level,
+                        int32_t num_levels, int32_t min_cols, int32_t max_sub_a, int32_t *type,
+                        int64_t *sub, cudaStream_t s)
+{
+    if (num_levels <= 0) return cudaSuccess;
+    unsigned long long *lsub = nullptr;
+    unsigned int *lwidth = nullptr;
+    cudaError_t e;
+    if ((e = dev_alloc((void **)&lsub, sizeof(unsigned long long) * num_levels, s)) != cudaSuccess)
+        return e;
+    if ((e = dev_alloc((void **)&lwidth, sizeof(unsigned int) * num_levels, s)) != cudaSuccess)
+        goto out;
+    if ((e = cudaMemsetAsync(lsub, 0, sizeof(unsigned long long) * num_levels, s)) != cudaSuccess)
+        goto out;
+    if ((e = cudaMemsetAsync(lwidth, 0, sizeof(unsigned int) * num_levels, s)) != cudaSuccess)
+        goto out;
+    if (n > 0) k_level_sub<<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, level, lsub, lwidth);
+    k_level_type<<<(num_levels + 255) / 256, 256, 0, s>>>(num_levels, lsub, lwidth, min_cols,
+                                                          max_sub_a, type, sub);
+    e = cudaGetLastError();
+out:
+    dev_free(lsub, s);
+    dev_free(lwidth, s);
+    return e;
+}
 
 cudaError_t level_schedule(int32_t n, const int32_t *level, int32_t num_levels,
                            int64_t *level_ptr, int32_t *level_cols, cudaStream_t s)

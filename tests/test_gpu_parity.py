@@ -437,3 +437,24 @@ def test_run_host_capacity():
     fc, rp_lu, ci_lu = h.run_host(nnz, nchunks=4)   # the handle stays usable
     assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
     h.close()
+
+
+def test_level_types():
+    """GLU3.0 level types (L208, reading R28) vs the oracle, several thresholds + defaults."""
+    d = dev()
+    sms = torch.cuda.get_device_properties(d).multi_processor_count
+    cases = [gen.circuit(48, 2), gen.lap2d(12), gen.lap3d(6), gen.random_pattern(500, 2.0, seed=3),
+             gen.random_pattern(3000, 1.2, seed=8, sym_frac=0.3), gen.lap2d(1)]
+    for rp, ci in cases:
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+        fc, rp_lu, ci_lu = h.run()
+        for rule in ("u", "glu3"):
+            lv, nl = h.levelize(rp_lu, ci_lu, rule)
+            rph, cih, lvh = rp_lu.cpu().numpy(), ci_lu.cpu().numpy(), lv.cpu().numpy()
+            for mc, ms in ((1, 1), (2, 3), (16, 8), (0, 0), (1000, 32)):
+                typ, sub = lu.level_types(rp_lu, ci_lu, lv, nl, mc, ms)
+                t_ref, s_ref, _ = oracle.level_types(rph, cih, lvh, nl, mc if mc > 0 else sms,
+                                                     ms if ms > 0 else 32)
+                assert np.array_equal(typ.cpu().numpy(), t_ref), (rule, mc, ms)
+                assert np.array_equal(sub.cpu().numpy(), s_ref), (rule, mc, ms)
+        h.close()
