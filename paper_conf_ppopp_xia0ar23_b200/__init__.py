@@ -358,14 +358,19 @@ def level_types(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, level: torch
 
 def symbolic_distributed(row_ptr: torch.Tensor, col_idx: torch.Tensor, group=None,
                          options: Options | None = None, rule: str = "u", stream=None,
-                         handle: Symbolic | None = None, cost=None):
+                         handle: Symbolic | None = None, cost=None, output: str = "replicated"):
     """Row-sharded symbolic factorization + levelization on every rank of `group`.
 
     A is replicated; rank r runs fill2 count and emit on its contiguous, cost-balanced row block
     (rows are independent); per-row counts are all-reduced (disjoint supports),
     every rank scans them, and the pattern blocks are broadcast from their owners (allgatherv),
     so all ranks end with the identical CSR of L+U; levels are then computed replicated.
+    output="local_rows" (SURVEY 8(b) LU_OUT_LOCAL_ROWS) skips the pattern exchange: col_idx_lu
+    holds only this rank's rows [row_ptr_lu[rb], row_ptr_lu[re]) and no levels are computed
+    (level = num_levels = None; the DAG is global).
     Returns (fill_count, row_ptr_lu, col_idx_lu, level, num_levels)."""
+    if output not in ("replicated", "local_rows"):
+        raise ValueError(f"output must be 'replicated' or 'local_rows', got {output!r}")
     import torch.distributed as dist
     world = dist.get_world_size(group) if dist.is_initialized() else 1
     rank = dist.get_rank(group) if dist.is_initialized() else 0
@@ -382,6 +387,8 @@ def symbolic_distributed(row_ptr: torch.Tensor, col_idx: torch.Tensor, group=Non
     rp_lu, nnz = h.scan(fc, stream=stream)
     ci_lu = torch.empty(nnz, dtype=torch.int32, device=h.device)
     h.emit(rp_lu, ci_lu, rb, re, stream=stream)
+    if output == "local_rows":
+        return fc, rp_lu, ci_lu, None, None
     if world > 1:
         assemble_pattern(ci_lu, rp_lu, bounds, group)
     level, nl = levelize(rp_lu, ci_lu, rule, handle=h, stream=stream)

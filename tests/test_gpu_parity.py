@@ -458,3 +458,18 @@ def test_level_types():
                 assert np.array_equal(typ.cpu().numpy(), t_ref), (rule, mc, ms)
                 assert np.array_equal(sub.cpu().numpy(), s_ref), (rule, mc, ms)
         h.close()
+
+
+def test_symbolic_distributed_single_rank():
+    """The row-sharded entry point on one rank (no process group): replicated and local-rows
+    outputs equal the oracle's."""
+    d = dev()
+    rp, ci = gen.circuit(40, 4)
+    ref = oracle.fill2(rp, ci)
+    args = (torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+    fc, rp_lu, ci_lu, lv, nl = lu.symbolic_distributed(*args)
+    assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+    lref, nref = oracle.levels(ref["row_ptr"], ref["col_idx"], "u")
+    assert nl == nref and np.array_equal(lv.cpu().numpy(), lref)
+    fc, rp_lu, ci_lu, lv, nl = lu.symbolic_distributed(*args, output="local_rows")
+    assert lv is None and np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
