@@ -101,7 +101,10 @@ typedef struct {
     int32_t struct_size;           /* = sizeof(lu_sym_opts)                                  */
     int32_t flags;                 /* LU_F_*                                                 */
     uint64_t scratch_budget_bytes; /* 0 => 0.85 x free HBM at create (out-of-core planner)   */
-    int32_t threads_per_row;       /* CTA size per row in flight; 0 => planner (128..1024)   */
+    int32_t threads_per_row;       /* CTA size per row in flight; 0 => planner (128..1024);
+                                      1025 = 1024 threads with the one-CTA-per-SM register
+                                      budget (the planner picks it when shared memory allows
+                                      only one 1024-thread CTA per SM anyway)               */
     int32_t rows_in_flight;        /* 0 => planner (all resident CTAs); > 0 caps it          */
     int32_t queue_capacity;        /* shared-memory frontier entries per buffer; 0 => planner */
     int32_t ell_width;             /* traversal adjacency slots 4, 6 or 8; 0 => planner     */

@@ -36,6 +36,9 @@ namespace f2 {
 #ifndef LUSYM_BATCH_TEST  // scan_level: load every neighbour's visited word before any atomic
 #define LUSYM_BATCH_TEST 0    // (A/B on B200: 3.7% slower on cfg2, 5% on cfg5 — kept as a knob)
 #endif
+#ifndef LUSYM_TAM  // test_and_mark with one shared bit mask (0: visited() then mark())
+#define LUSYM_TAM 1
+#endif
 #ifndef LUSYM_THREADS_PER_SM  // register budget: 65536 / this
 #define LUSYM_THREADS_PER_SM 2048
 #endif
@@ -187,6 +190,29 @@ __device__ __forceinline__ bool mark(const VisMap<VIS> &m, uint32_t *sm, int v)
                      : "memory");
     (void)sm;
     return !(old & b);
+}
+
+// visited test, then test-and-set only if the bit looked clear (the atomic decides); the bit
+// mask is computed once for both.  True iff this call set the bit.
+template <int VIS>
+__device__ __forceinline__ bool test_and_mark(const VisMap<VIS> &m, uint32_t *sm, int v)
+{
+#if LUSYM_TAM
+    const uint32_t b = 1u << (v & 31);
+    const int w = v >> 5;
+    const bool sh = in_smem(m, w);
+    const uint32_t word = sh ? lds_bm(phys<VIS>(w)) : __ldcg(m.g + w);
+    if (word & b) return false;
+    const uint32_t old = sh ? atom_or_bm(phys<VIS>(w), b) : atomicOr(m.g + w, b);
+    if (old == 0)
+        asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(summary_saddr(m) + (uint32_t)(v >> 10) * 4u),
+                     "r"(1u << (w & 31))
+                     : "memory");
+    (void)sm;
+    return !(old & b);
+#else
+    return !visited(m, v) && mark(m, sm, v);
+#endif
 }
 
 // ELL slots W in {4, 6, 8}; rows are stored 4 (W = 4) or 8 (W = 6, 8) entries wide.  A light
@@ -368,8 +394,10 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
         int f = valid ? (k < p.q ? L[k] : __ldcg(gL + k)) : 0;
       for (int r = 0;; ++r) {
         int nb[ell_stride<W>()];
+#if !LUSYM_NO_NB_INIT
 #pragma unroll
         for (int s = 0; s < ell_stride<W>(); ++s) nb[s] = 0;
+#endif
         bool heavy = false;
         // new frontier vertices of this thread: the first three stay in registers (f0..f2) for
         // one warp-aggregated append (a grid vertex has up to three neighbours further from
@@ -394,7 +422,8 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
 #pragma unroll
                 for (int s = 0; s < W; ++s) {
                     const int w = nb[s];
-                    if ((um >> s & 1u) && (LUSYM_BATCH_TEST || !visited(bm, w)) && mark(bm, sm, w)) {
+                    if ((um >> s & 1u) &&
+                        (LUSYM_BATCH_TEST ? mark(bm, sm, w) : test_and_mark(bm, sm, w))) {
                         if (w < t0) {
                             if (c == 3) {
                                 put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
@@ -459,7 +488,7 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                 int w = -1;
                 if (e < len) {
                     w = __ldg(p.ci + off + e);
-                    if (!visited(bm, w) && mark(bm, sm, w)) {
+                    if (test_and_mark(bm, sm, w)) {
                         if (w < t0) {
                             fr = true;
                         } else if (w > i) {
@@ -527,11 +556,26 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_
     a.lmin = 0;  // the BFS marked vertices somewhere below t0: clear from word 0 (summary walk)
 }
 
+// Kernel key -> CTA size and register budget.  KEY = NT (128..1024): registers for
+// LUSYM_THREADS_PER_SM resident threads (32 per thread at 2048).  KEY = 1025: 1024 threads with
+// the one-CTA-per-SM budget (64 registers, no spills) for classes whose shared memory already
+// limits them to one CTA per SM (the planner picks it).
+template <int KEY>
+struct NtCfg {
+    static constexpr int NT = KEY, MINB = LUSYM_THREADS_PER_SM / KEY;
+};
+template <>
+struct NtCfg<1025> {
+    static constexpr int NT = 1024, MINB = 1;
+};
+
 // MODE: kCount (symbolic_1, counts only), kStage (counts + rows staged into the HBM pool, so
 // symbolic_2 becomes a placement copy), kEmit (symbolic_2 by traversal, into the final CSR).
-template <int NT, int W, int MODE, int VIS>
-__global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(const Fill2Params p)
+template <int KEY, int W, int MODE, int VIS>
+__global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
+    fill2_kernel(const Fill2Params p)
 {
+    constexpr int NT = NtCfg<KEY>::NT;
     constexpr bool GB = VIS == kVisGlobal;
     extern __shared__ __align__(16) unsigned char smem[];
     Hdr &h = *reinterpret_cast<Hdr *>(smem);
@@ -667,7 +711,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
 #pragma unroll
                         for (int s = 0; s < W; ++s) {
                             const int w = nb[s];
-                            if (w > t && !visited(bm, w) && mark(bm, sm, w)) {
+                            if (w > t && test_and_mark(bm, sm, w)) {
                                 if (w < i) {
                                     nm = min(nm, w);
                                 } else {
@@ -699,7 +743,7 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
                     } else {
                         for (int e = lane; e < len; e += 32) {
                             const int w = __ldg(p.ci + off + e);
-                            if (w > tt && !visited(bm, w) && mark(bm, sm, w)) {
+                            if (w > tt && test_and_mark(bm, sm, w)) {
                                 if (w < i) {
                                     nm = min(nm, w);
                                 } else {
@@ -803,12 +847,13 @@ __global__ void __launch_bounds__(NT, LUSYM_THREADS_PER_SM / NT) fill2_kernel(co
 template <int NT, int W, int VIS>
 cudaError_t launch_w_vis(const Fill2Params &p, int mode, int grid, size_t smem, cudaStream_t s)
 {
+    constexpr int B = NtCfg<NT>::NT;  // NT here is the kernel key
     if (mode == kCount)
-        fill2_kernel<NT, W, kCount, VIS><<<grid, NT, smem, s>>>(p);
+        fill2_kernel<NT, W, kCount, VIS><<<grid, B, smem, s>>>(p);
     else if (mode == kStage)
-        fill2_kernel<NT, W, kStage, VIS><<<grid, NT, smem, s>>>(p);
+        fill2_kernel<NT, W, kStage, VIS><<<grid, B, smem, s>>>(p);
     else
-        fill2_kernel<NT, W, kEmit, VIS><<<grid, NT, smem, s>>>(p);
+        fill2_kernel<NT, W, kEmit, VIS><<<grid, B, smem, s>>>(p);
     return cudaGetLastError();
 }
 
@@ -836,7 +881,7 @@ cudaError_t occupancy_w_vis(size_t smem, int *occ)
     int best = 1 << 30;
     for (const void *f : fns) {
         int o = 0;
-        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, f, NT, smem);
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&o, f, NtCfg<NT>::NT, smem);
         if (e != cudaSuccess) return e;
         best = o < best ? o : best;
     }

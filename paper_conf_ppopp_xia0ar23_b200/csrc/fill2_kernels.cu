@@ -21,6 +21,7 @@ size_t fill2_smem_bytes(int n, int smem_words, int q)
     case 256: return FN<256>(__VA_ARGS__);                                                   \
     case 512: return FN<512>(__VA_ARGS__);                                                   \
     case 1024: return FN<1024>(__VA_ARGS__);                                                 \
+    case 1025: return FN<1025>(__VA_ARGS__);                                                 \
     default: return cudaErrorInvalidValue;                                                   \
     }
 

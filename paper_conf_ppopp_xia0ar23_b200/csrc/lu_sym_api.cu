@@ -4,6 +4,7 @@
 
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <algorithm>
 #include <cstring>
 #include <string>
@@ -259,12 +260,16 @@ struct Cfg {
 
 lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out)
 {
-    const int nts[4] = {128, 256, 512, 1024};
+    // kernel keys: CTA sizes 128..1024, and 1025 = 1024 threads with the one-CTA-per-SM
+    // register budget (chosen on a tie, i.e. when shared memory allows one CTA per SM anyway)
+    const int nts[5] = {128, 256, 512, 1024, 1025};
     const int qs[4] = {512, 1024, 2048, 4096};
     Cfg best = {0, 0, 0, 0, -1};
-    for (int a = 0; a < 4; ++a) {
+    for (int a = 0; a < 5; ++a) {
         const int nt = nts[a];
-        if (h->opts.threads_per_row > 0 && nt != h->opts.threads_per_row) continue;
+        const int tpr = h->opts.threads_per_row;
+        if (tpr > 0 && nt != tpr && !(tpr == 1024 && nt == 1025)) continue;
+        const int threads = nt > 1024 ? 1024 : nt;
         for (int b = 0; b < 4; ++b) {
             int q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : qs[b];
             if (h->opts.queue_capacity > 0 && b > 0) break;
@@ -277,8 +282,9 @@ lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out)
             int occ = 0;
             CK(fill2_occupancy(nt, h->w, vis, smem, &occ));
             if (occ < 1) continue;
-            const long key = ((long)occ * nt << 24) | ((long)occ << 14) | q;
-            if (key > best.key) best = Cfg{nt, q, occ, smem, key};
+            const long key = ((long)occ * threads << 24) | ((long)occ << 14) | q;
+            if (key > best.key || (key == best.key && nt == 1025))
+                best = Cfg{nt, q, occ, smem, key};
         }
     }
     *out = best;
@@ -295,8 +301,8 @@ lu_status plan(lu_sym *h)
     const int nw32 = (nw + 31) / 32 * 32;  // whole swizzle groups
     if (h->opts.threads_per_row > 0 && h->opts.threads_per_row != 128 &&
         h->opts.threads_per_row != 256 && h->opts.threads_per_row != 512 &&
-        h->opts.threads_per_row != 1024)
-        return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512 or 1024 (got %d)",
+        h->opts.threads_per_row != 1024 && h->opts.threads_per_row != 1025)
+        return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512, 1024 or 1025 (got %d)",
                     h->opts.threads_per_row);
     // top class: the whole visited map in shared memory, else in HBM
     Cfg cur;
@@ -403,6 +409,13 @@ lu_status plan(lu_sym *h)
     if (h->staging) {
         if ((st = salloc(h, &h->stg, need_stg)) != LU_OK) return st;
         if ((st = salloc(h, &h->row_off, (size_t)n)) != LU_OK) return st;
+    }
+    if (getenv("LUSYM_DEBUG_PLAN")) {
+        for (auto &c : h->classes)
+            fprintf(stderr,
+                    "lusym plan: rows [%d,%d) vis %d smem_words %d lbw %d nt %d q %d occ %d "
+                    "smem %zu grid %d\n",
+                    c.lo, c.hi, c.vis, c.smem_words, c.lbw, c.nt, c.q, c.occ, c.smem, c.grid);
     }
     // summary fields (the top class)
     const RowClass &top = h->classes.front();
@@ -1129,7 +1142,7 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
     }
     h->stats.scratch_bytes = h->scratch_bytes;
     h->stats.rows_in_flight = h->grid;
-    h->stats.threads_per_row = h->nt;
+    h->stats.threads_per_row = h->nt > 1024 ? 1024 : h->nt;
     h->stats.smem_bytes_per_row = (int32_t)h->smem;
     h->stats.visited_in_smem = h->gb ? 0 : 1;
     h->stats.row_classes = (int32_t)h->classes.size();

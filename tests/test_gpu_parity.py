@@ -137,6 +137,8 @@ KNOBS = [
     dict(queue_capacity=32),                         # forces frontier spills to HBM
     dict(rows_in_flight=1), dict(rows_in_flight=3), dict(rows_in_flight=17),
     dict(threads_per_row=128), dict(threads_per_row=512), dict(threads_per_row=1024),
+    dict(threads_per_row=1025),                      # 1024 threads, one-CTA-per-SM registers
+    dict(threads_per_row=1025, queue_capacity=32, flags=lu.F_FORCE_CLASSES),
     dict(ell_width=4), dict(ell_width=6), dict(ell_width=8),
     dict(flags=lu.F_GLOBAL_BITMAP, queue_capacity=32, rows_in_flight=5),
     dict(flags=lu.F_NO_PRUNE), dict(flags=lu.F_KAHN_WIDE_ONLY), dict(flags=lu.F_NO_CONTRACT),
