@@ -674,16 +674,17 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
         int cap = p.wcap;
         // ---- thresholds in increasing order (L130)
         for (;;) {
+            // the previous window's tns/newmin were read before its last barrier; collect ends
+            // with a barrier, so this reset is visible before the window's atomicMin's
+            if (tid == 0) {
+                h.tns = INT_MAX;
+                h.newmin = INT_MAX;
+            }
             const int wc = collect<NT, VIS>(bm, sm, dused ? dm : nullptr, ptr + 1, i, qA, cap,
                                            h.scan);
             if (wc == 0) break;
             ++n_win;
-            if (tid == 0) {
-                h.tns = INT_MAX;
-                h.newmin = INT_MAX;
-                h.sv += wc;
-            }
-            __syncthreads();
+            if (tid == 0) h.sv += wc;
             int nm = INT_MAX;
             for (int base = 0; base < wc; base += NT) {
                 const int k = base + tid;
