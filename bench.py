@@ -189,22 +189,33 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------------------- CPU oracle
-def cpu_oracle_sample(rp, ci, stride, rule="u"):
-    """Time the oracle (as it stands) on every stride-th row (both passes, all host cores) and
-    on the full Kahn levelization; extrapolate the symbolic time by exact TE share."""
+def cpu_oracle_sample(rp, ci, stride, rule="u", te_total=None, threads=None):
+    """Time the oracle (as it stands) on every stride-th row (both passes, all host cores by
+    default) and extrapolate the symbolic time by TE share (te_total: the exact per-config TE
+    of tests/golden/work_units.json, else the grid closed form sum row_ptr[i+1])."""
     import oracle
     n = len(rp) - 1
     rows = np.arange(n - 1, -1, -stride, dtype=np.int32)
-    threads = os.cpu_count() or 1
+    threads = threads or os.cpu_count() or 1
     t0 = time.perf_counter()
     r = oracle.fill2(rp, ci, rows=rows, emit=True, threads=threads)
     t_sym = time.perf_counter() - t0
-    te_total = int(rp[1:].sum())
+    if te_total is None:
+        te_total = int(rp[1:].sum())
     te_sample = int(r["te"].sum())
     scale = te_total / max(te_sample, 1)
     t_sym_full = t_sym * scale
     return dict(rows=rows, t_sample=t_sym, t_sym_full=t_sym_full, threads=threads,
                 entries_sample=int(r["counts"].sum()), te_sample=te_sample, scale=scale)
+
+
+def cpu_one_core_rate(rp, ci, te_total, seconds=1.0):
+    """the oracle on ONE thread over a row sample of about `seconds` of work ->
+    traversed edges per second per core (both passes)."""
+    stride = max(1, int(round(te_total / (3e8 * seconds))))
+    s = cpu_oracle_sample(rp, ci, stride, te_total=te_total, threads=1)
+    return {"te_per_s": 2 * s["te_sample"] / max(s["t_sample"], 1e-9), "rows": len(s["rows"]),
+            "seconds": s["t_sample"]}
 
 
 def cpu_levels_time(rp, ci, rule, nnz_hint=None):
@@ -234,7 +245,7 @@ def run_reference(args, rank, world):
     stride = args.cpu_sample_stride or auto_stride(n, te)
     times, entries = [], None
     for k in range(args.warmup + args.steps):
-        s = cpu_oracle_sample(rp, ci, stride)
+        s = cpu_oracle_sample(rp, ci, stride, te_total=te)
         if k >= args.warmup:
             times.append(s["t_sym_full"])
         entries = s
@@ -450,7 +461,8 @@ def run_ours(args, rank, world, local_rank):
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
         stride = args.cpu_sample_stride or auto_stride(n, te)
-        s = cpu_oracle_sample(rp_np, ci_np, stride)
+        s = cpu_oracle_sample(rp_np, ci_np, stride, te_total=te)
+        one = cpu_one_core_rate(rp_np, ci_np, te)
         import oracle
         rpl = state["rp_lu"].cpu().numpy()
         cil = state["ci_lu"].cpu().numpy()
@@ -462,7 +474,9 @@ def run_ours(args, rank, world, local_rank):
                "sample": f"fill2 count+emit on every {stride}-th row ({len(s['rows'])} rows) in "
                          f"{s['t_sample']:.2f} s, extrapolated by exact TE share "
                          f"x{s['scale']:.2f}; Kahn levels on the full pattern {t_lev:.2f} s "
-                         f"(1 thread)"}
+                         f"(1 thread)",
+               "one_core": {"traversed_edges_per_s": one["te_per_s"], "rows": one["rows"],
+                            "note": "oracle on 1 thread, count+emit (2 traversals per row)"}}
     out = {
         "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -495,6 +509,10 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    # test hook: run every rank on one GPU over gloo (exercises the N>1 path where only one GPU
+    # exists); never used for a reported number
+    if os.environ.get("LUSYM_BENCH_ONE_GPU"):
+        local_rank = 0
     if args.impl == "reference":
         run_reference(args, rank, world)
         return
@@ -502,7 +520,11 @@ def main():
         import torch
         import torch.distributed as dist
         torch.cuda.set_device(local_rank)
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        backend = os.environ.get("LUSYM_BENCH_BACKEND", "nccl")
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local_rank))
+        else:
+            dist.init_process_group(backend)
     try:
         run_ours(args, rank, world, local_rank)
     finally:

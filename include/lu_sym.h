@@ -196,7 +196,7 @@ lu_status lu_sym_run(lu_sym *h, int32_t *d_fill_count, int64_t *d_row_ptr_lu,
 /*
  * Whole symbolic pass with the result streamed to the host while later rows are still being
  * traversed: Alg. 3's out-of-core chunks (L239-270) taken in INCREASING row order, nchunks row
- * ranges of equal a-priori traversal cost (0 => 16; at most 64).  Per chunk: symbolic_1 with
+ * ranges of equal a-priori traversal cost (0 => min(16, max(1, n/4096)); at most 64).  Per chunk: symbolic_1 with
  * staging (the traversal; chunk k+1 runs on a second scratch set so it fills the SMs chunk k
  * drains), the chained prefix sum of its counts (L262), symbolic_2 as a placement of its
  * staged rows (L264-270) and the device->host copy of its rows, the last three behind the

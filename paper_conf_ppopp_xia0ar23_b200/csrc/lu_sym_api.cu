@@ -890,7 +890,8 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
     cudaStream_t s = (cudaStream_t)stream;
     h->stream = s;
     const int32_t n = h->n;
-    if (nchunks == 0) nchunks = 16;
+    if (nchunks == 0)  // 16 chunks, but none under 4096 rows (each chunk costs a host sync)
+        nchunks = std::max(1, std::min(16, n / 4096));
     if (nchunks > n) nchunks = n > 0 ? n : 1;
     if (h->staging) {
         if ((st = ensure_pool(h)) != LU_OK) return st;

@@ -1,6 +1,8 @@
+#!/bin/bash
+# Queue-capacity sweep (lu_sym_opts.queue_capacity): QS per config in CFGS (under gpurun).
 cd "${GRAFT_REPO_ROOT:-/root/repo}"
-for c in 2 5; do for q in 512 640 768 1024 1536; do
-  timeout 600 python bench.py --config $c --steps 5 --warmup 2 --no-cpu-baseline --no-e2e --queue-capacity $q 2>&1 | python -c "
+for c in ${CFGS:-2 5}; do for q in ${QS:-256 384 512 1024}; do
+  timeout 900 python bench.py --config $c --steps ${STEPS:-5} --warmup 2 --no-cpu-baseline --no-e2e --queue-capacity $q 2>&1 | python -c "
 import sys, json
 for l in sys.stdin:
     if l.startswith('{'):
