@@ -64,7 +64,7 @@ lu_status fail(lu_status s, const char *fmt, ...)
 
 enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvN = 4 };
 enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11, kSlotClassCounter = 16,
-       kSlotSetStride = 32, kStatSlots = 80, kMaxChunks = 64 };
+       kSlotSetStride = 32, kStatSlots = 128, kMaxChunks = 64, kSets = 3 };
 
 }  // namespace
 
@@ -130,16 +130,18 @@ struct lu_sym {
     int64_t *row_prof = nullptr;  // borrowed, set by lu_sym_set_row_profile
     cudaStream_t stream = nullptr;  // stream of the last call (scratch is freed on it)
     std::vector<void *> managed;    // LU_F_MANAGED scratch (freed with cudaFree)
-    // second traversal scratch set (lu_sym_run_host: two row chunks in flight at once, so the
-    // next chunk's CTAs take over SMs while the previous chunk drains); allocated on first use
-    int32_t *gspill1 = nullptr, *stg1 = nullptr;
-    uint32_t *gbitmap1 = nullptr, *dbitmap1 = nullptr;
-    std::vector<cudaStream_t> cls_stream1;
-    std::vector<cudaEvent_t> cls_done1;
-    cudaStream_t pipe_stream[3] = {};  // lu_sym_run_host: second count stream, place, copy
+    // extra traversal scratch sets 1..kSets-1 (lu_sym_run_host: the heaviest row chunk on set
+    // 0 while the others alternate on sets 1 and 2, so a chunk's CTAs take over the SMs the
+    // previous one leaves while it drains); allocated on first use
+    int32_t *gspillS[kSets] = {}, *stgS[kSets] = {};
+    uint32_t *gbitmapS[kSets] = {}, *dbitmapS[kSets] = {};
+    std::vector<cudaStream_t> cls_streamS[kSets];
+    std::vector<cudaEvent_t> cls_doneS[kSets];
+    cudaStream_t pipe_stream[4] = {};  // lu_sym_run_host: count streams of sets 1/2, place, copy
     cudaEvent_t pipe_ev[4][kMaxChunks + 1] = {};  // count done, scanned, placed, copied
     int64_t *pin = nullptr;                       // pinned host slot (chunk end offset)
     std::vector<int32_t> chunk_bounds;            // lu_sym_run_host row chunks (cached)
+    bool heavy_last = false;                      // ... and whether the last chunk goes first
 };
 
 namespace {
@@ -205,10 +207,14 @@ void free_handle(lu_sym *h)
 {
     cudaStream_t s = h->stream;
     void *bufs[] = {h->ell,      h->gbitmap,  h->dbitmap, h->gspill, h->dstats,  h->scan_blk,
-                    h->dbad,     h->stg,      h->pool,    h->row_off, h->unstaged, h->gspill1,
-                    h->gbitmap1, h->dbitmap1, h->stg1};
+                    h->dbad,     h->stg,      h->pool,    h->row_off, h->unstaged};
     if (!h->managed.empty()) cudaStreamSynchronize(s);
-    for (void *b : bufs) {
+    std::vector<void *> all(std::begin(bufs), std::end(bufs));
+    for (int k = 1; k < kSets; ++k)
+        for (void *b : {(void *)h->gspillS[k], (void *)h->stgS[k], (void *)h->gbitmapS[k],
+                        (void *)h->dbitmapS[k]})
+            all.push_back(b);
+    for (void *b : all) {
         if (!b) continue;
         if (std::find(h->managed.begin(), h->managed.end(), b) != h->managed.end())
             cudaFree(b);
@@ -220,10 +226,12 @@ void free_handle(lu_sym *h)
         if (c.stream) cudaStreamDestroy(c.stream);
         if (c.done) cudaEventDestroy(c.done);
     }
-    for (auto cs : h->cls_stream1)
-        if (cs) cudaStreamDestroy(cs);
-    for (auto ce : h->cls_done1)
-        if (ce) cudaEventDestroy(ce);
+    for (int k = 1; k < kSets; ++k) {
+        for (auto cs : h->cls_streamS[k])
+            if (cs) cudaStreamDestroy(cs);
+        for (auto ce : h->cls_doneS[k])
+            if (ce) cudaEventDestroy(ce);
+    }
     for (auto ps : h->pipe_stream)
         if (ps) cudaStreamDestroy(ps);
     for (auto &row : h->pipe_ev)
@@ -453,10 +461,10 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
 {
     const bool emit = mode == kEmit;
     unsigned long long *st = h->dstats + (emit ? 5 : 1);
-    int32_t *gspill = set ? h->gspill1 : h->gspill;
-    int32_t *stg = set ? h->stg1 : h->stg;
-    uint32_t *gbitmap = set ? h->gbitmap1 : h->gbitmap;
-    uint32_t *dbitmap = set ? h->dbitmap1 : h->dbitmap;
+    int32_t *gspill = set ? h->gspillS[set] : h->gspill;
+    int32_t *stg = set ? h->stgS[set] : h->stg;
+    uint32_t *gbitmap = set ? h->gbitmapS[set] : h->gbitmap;
+    uint32_t *dbitmap = set ? h->dbitmapS[set] : h->dbitmap;
     unsigned long long *counters = h->dstats + kSlotClassCounter + set * kSlotSetStride;
     if (reset_stats) CK(cudaMemsetAsync(st, 0, sizeof(unsigned long long) * kStatCount, s));
     if (gbitmap) CK(cudaMemsetAsync(gbitmap, 0, sizeof(uint32_t) * h->map_words, s));
@@ -496,12 +504,12 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
         if (rows <= 0) continue;
         cudaStream_t cs = s;
         if (k > 0) {
-            cudaEvent_t fork_ev = set ? h->cls_done1[0] : h->classes[0].done;
+            cudaEvent_t fork_ev = set ? h->cls_doneS[set][0] : h->classes[0].done;
             if (!forked) {
                 CK(cudaEventRecord(fork_ev, s));
                 forked = true;
             }
-            cs = set ? h->cls_stream1[k] : c.stream;
+            cs = set ? h->cls_streamS[set][k] : c.stream;
             CK(cudaStreamWaitEvent(cs, fork_ev, 0));
         }
         p.row_begin = lo;
@@ -546,39 +554,45 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     }
     if (forked)  // join
         for (size_t k = 1; k < h->classes.size(); ++k) {
-            cudaEvent_t je = set ? h->cls_done1[k] : h->classes[k].done;
-            CK(cudaEventRecord(je, set ? h->cls_stream1[k] : h->classes[k].stream));
+            cudaEvent_t je = set ? h->cls_doneS[set][k] : h->classes[k].done;
+            CK(cudaEventRecord(je, set ? h->cls_streamS[set][k] : h->classes[k].stream));
             CK(cudaStreamWaitEvent(s, je, 0));
         }
     return LU_OK;
 }
 
-// The second traversal scratch set (same sizes as the first), its class streams and the
-// pipeline's streams/events; allocated on the first lu_sym_run_host call.
-lu_status ensure_set1(lu_sym *h)
+// Extra traversal scratch sets 1..kSets-1 (same sizes as set 0), their class streams and the
+// pipeline's streams; allocated on the first pipelined lu_sym_run_host call.
+lu_status ensure_sets(lu_sym *h)
 {
-    if (h->dbitmap1) return LU_OK;
+    if (h->dbitmapS[kSets - 1]) return LU_OK;
     int64_t need_spill = 0, need_stg = 0;
     for (auto &c : h->classes) {
         need_spill = std::max<int64_t>(need_spill, c.spill_off + 2 * c.cap * (int64_t)c.grid);
         need_stg = std::max<int64_t>(need_stg, c.stg_off + c.cap * (int64_t)c.grid);
     }
     lu_status st;
-    if ((st = salloc(h, &h->gspill1, (size_t)need_spill)) != LU_OK) return st;
-    if (h->gbitmap && (st = salloc(h, &h->gbitmap1, (size_t)h->map_words)) != LU_OK) return st;
-    if ((st = salloc(h, &h->dbitmap1, (size_t)h->map_words)) != LU_OK) return st;
-    if (h->staging && (st = salloc(h, &h->stg1, (size_t)need_stg)) != LU_OK) return st;
-    h->cls_stream1.assign(h->classes.size(), nullptr);
-    h->cls_done1.assign(h->classes.size(), nullptr);
-    for (size_t k = 0; k < h->classes.size(); ++k) {
-        CK(cudaEventCreateWithFlags(&h->cls_done1[k], cudaEventDisableTiming));
-        if (k > 0) CK(cudaStreamCreateWithFlags(&h->cls_stream1[k], cudaStreamNonBlocking));
+    for (int k = 1; k < kSets; ++k) {
+        if ((st = salloc(h, &h->gspillS[k], (size_t)need_spill)) != LU_OK) return st;
+        if (h->gbitmap && (st = salloc(h, &h->gbitmapS[k], (size_t)h->map_words)) != LU_OK)
+            return st;
+        if (h->staging && (st = salloc(h, &h->stgS[k], (size_t)need_stg)) != LU_OK) return st;
+        h->cls_streamS[k].assign(h->classes.size(), nullptr);
+        h->cls_doneS[k].assign(h->classes.size(), nullptr);
+        for (size_t c = 0; c < h->classes.size(); ++c) {
+            CK(cudaEventCreateWithFlags(&h->cls_doneS[k][c], cudaEventDisableTiming));
+            if (c > 0)
+                CK(cudaStreamCreateWithFlags(&h->cls_streamS[k][c], cudaStreamNonBlocking));
+        }
+        if ((st = salloc(h, &h->dbitmapS[k], (size_t)h->map_words)) != LU_OK) return st;
     }
     int lo = 0, hi = 0;
     CK(cudaDeviceGetStreamPriorityRange(&lo, &hi));
-    // [0] second count stream (normal priority); [1] scan + place and [2] device->host copies
-    // at the highest priority, so a chunk's placement CTAs go ahead of queued traversal CTAs
+    // [0], [3] count streams of sets 1 and 2 (normal priority); [1] scan + place and [2]
+    // device->host copies at the highest priority, so a chunk's placement CTAs go ahead of
+    // queued traversal CTAs
     CK(cudaStreamCreateWithPriority(&h->pipe_stream[0], cudaStreamNonBlocking, lo));
+    CK(cudaStreamCreateWithPriority(&h->pipe_stream[3], cudaStreamNonBlocking, lo));
     CK(cudaStreamCreateWithPriority(&h->pipe_stream[1], cudaStreamNonBlocking, hi));
     CK(cudaStreamCreateWithPriority(&h->pipe_stream[2], cudaStreamNonBlocking, hi));
     CK(cudaMallocHost(reinterpret_cast<void **>(&h->pin), 2 * sizeof(int64_t)));
@@ -896,8 +910,8 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
     if (h->staging) {
         if ((st = ensure_pool(h)) != LU_OK) return st;
     }
-    if (!h->staging || !h->pool || n == 0) {
-        // two-pass mode (or no pool): the plain calls, then the copies
+    if (!h->staging || !h->pool || n == 0 || nchunks == 1) {
+        // one chunk, two-pass mode or no pool: the plain calls, then the copies
         int64_t nnz = 0;
         if ((st = lu_sym_run(h, d_fill_count, d_row_ptr_lu, nullptr, 0, &nnz, stream)) != LU_OK)
             return st;
@@ -916,9 +930,9 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
         CK(cudaStreamSynchronize(s));
         return LU_OK;
     }
-    if ((st = ensure_set1(h)) != LU_OK) return st;
+    if ((st = ensure_sets(h)) != LU_OK) return st;
     // row chunks of equal a-priori traversal cost (row_ptr[i+1]: the TE bound of row i, exact on
-    // the grids), in increasing row order so that each chunk's offsets follow its predecessor's
+    // the grids); offsets are chained in increasing row order
     if ((int)h->chunk_bounds.size() != nchunks + 1) {
         std::vector<int64_t> rp((size_t)n + 1);
         CK(cudaMemcpyAsync(rp.data(), h->rp, sizeof(int64_t) * rp.size(), cudaMemcpyDeviceToHost,
@@ -936,13 +950,19 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
         }
         while ((int)h->chunk_bounds.size() < nchunks + 1) h->chunk_bounds.push_back(n);
         h->chunk_bounds.back() = n;
+        // rows of very high degree (circuit hubs, ordered last) make the last chunk's rows the
+        // critical path: start that chunk first (a-priori test: max degree > 64 x mean)
+        int64_t maxdeg = 0;
+        for (int32_t i = 0; i < n; ++i)
+            maxdeg = std::max<int64_t>(maxdeg, rp[(size_t)i + 1] - rp[(size_t)i]);
+        h->heavy_last = (double)maxdeg > 64.0 * ((double)rp[(size_t)n] / n + 1.0);
     }
     const std::vector<int32_t> &b = h->chunk_bounds;
     for (auto &row : h->pipe_ev)  // events of chunks 0..nchunks-1 and the fork slot
         for (int k = 0; k <= kMaxChunks; ++k)
             if (!row[k] && (k < nchunks || k == kMaxChunks))
                 CK(cudaEventCreateWithFlags(&row[k], cudaEventDisableTiming));
-    cudaStream_t cs[2] = {s, h->pipe_stream[0]};
+    cudaStream_t cs[kSets] = {s, h->pipe_stream[0], h->pipe_stream[3]};
     cudaStream_t sp = h->pipe_stream[1], sc = h->pipe_stream[2];
     cudaEvent_t *ev_count = h->pipe_ev[0], *ev_scan = h->pipe_ev[1], *ev_place = h->pipe_ev[2],
                 *ev_copy = h->pipe_ev[3];
@@ -956,17 +976,24 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
     CK(cudaMemsetAsync(h->dstats + 1, 0, sizeof(unsigned long long) * kStatCount, s));
     CK(cudaMemsetAsync(d_row_ptr_lu, 0, sizeof(int64_t), s));
     CK(cudaEventRecord(ev_count[kMaxChunks], s));
-    for (cudaStream_t x : {cs[1], sp, sc}) CK(cudaStreamWaitEvent(x, ev_count[kMaxChunks], 0));
-    // symbolic_1 with staging, chunk k on scratch set k & 1: chunk k+1's CTAs fill the SMs that
-    // chunk k's CTAs leave while it drains
-    for (int k = 0; k < nchunks; ++k) {
+    for (cudaStream_t x : {cs[1], cs[2], sp, sc})
+        CK(cudaStreamWaitEvent(x, ev_count[kMaxChunks], 0));
+    // symbolic_1 with staging, chunks in increasing order alternating on sets 1 and 2, so chunk
+    // k+1's CTAs fill the SMs chunk k leaves as it drains.  With heavy_last, the last chunk
+    // (holding the critical-path rows, L272) starts first on set 0.
+    const bool hl = h->heavy_last;
+    auto set_of = [&](int k) { return hl && k == nchunks - 1 ? 0 : 1 + (k & 1); };
+    for (int pos = 0; pos < nchunks; ++pos) {
+        const int k = hl ? (pos == 0 ? nchunks - 1 : pos - 1) : pos;
+        const int set = set_of(k);
         if (b[k] < b[k + 1] &&
-            (st = run_pass(h, kStage, b[k], b[k + 1], d_fill_count, nullptr, nullptr, cs[k & 1],
-                           nullptr, 0, k & 1, false)) != LU_OK)
+            (st = run_pass(h, kStage, b[k], b[k + 1], d_fill_count, nullptr, nullptr, cs[set],
+                           nullptr, 0, set, false)) != LU_OK)
             return st;
-        CK(cudaEventRecord(ev_count[k], cs[k & 1]));
+        CK(cudaEventRecord(ev_count[k], cs[set]));
     }
-    if (nchunks > 1) CK(cudaStreamWaitEvent(s, ev_count[nchunks - 1 - ((nchunks - 1) & 1 ? 0 : 1)], 0));
+    for (int k = nchunks - 1; k >= 0 && k >= nchunks - 3; --k)  // the last chunk of each set
+        CK(cudaStreamWaitEvent(s, ev_count[k], 0));
     CK(cudaEventRecord(h->ev[kEvCount][1], s));  // s now follows every chunk's traversal
     h->ev_used[kEvCount] = true;
     // per chunk, behind its traversal: chained prefix sum, placement (symbolic_2 of staged

@@ -405,8 +405,18 @@ def test_run_host_pipelined(nchunks, knob):
     """lu_sym_run_host: chunked count -> chained scan -> place -> D2H, bit-exact on the device
     and host copies, repeated on the same handle (fresh pool and scratch sets each call)."""
     d = dev()
+    # a matrix whose last rows are hubs (degree > 64 x mean: the heavy-last chunk order)
+    n = 3000
+    rp0, ci0 = gen.random_pattern(n, 1.5, seed=70_001)
+    R = [np.repeat(np.arange(n), np.diff(rp0))]
+    C = [ci0.astype(np.int64)]
+    for hub in range(n - 6, n):
+        nb = np.random.default_rng(hub).choice(n, 900, replace=False)
+        R += [np.full(nb.size, hub), nb]
+        C += [nb, np.full(nb.size, hub)]
+    hubs = gen.csr_from_edges(n, np.concatenate(R), np.concatenate(C))
     for rp, ci in (gen.lap3d(11), gen.circuit(48, 7), gen.random_pattern(900, 2.0, seed=5),
-                   gen.lap2d(1), gen.random_pattern(40, 0.5, seed=1)):
+                   gen.lap2d(1), gen.random_pattern(40, 0.5, seed=1), hubs):
         ref = oracle.fill2(rp, ci)
         nnz = int(ref["row_ptr"][-1])
         h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d), **knob)
