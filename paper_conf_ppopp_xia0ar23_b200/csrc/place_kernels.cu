@@ -14,6 +14,23 @@ constexpr int kPlaceNT = 256;
 constexpr int kPlaceTile = 4096;
 constexpr int kPlaceRows = 1024;
 
+// Largest r in [lo, hi) with rp[r] <= x, given rp[lo] <= x (rp non-decreasing): a 32-ary
+// search by one warp, about log32(rows) dependent loads instead of log2(rows).
+__device__ __forceinline__ int warp_row_search(const int64_t *rp, int lo, int hi, int64_t x)
+{
+    const int lane = threadIdx.x & 31;
+    while (hi - lo > 1) {
+        const int step = (hi - lo + 31) / 32;
+        const int probe = lo + lane * step;
+        const bool ok = probe < hi && rp[probe] <= x;
+        const unsigned b = __ballot_sync(0xffffffffu, ok);
+        const int j = 31 - __clz(b);  // last probe <= x (probe 0 = lo always is)
+        lo = lo + j * step;
+        hi = min(hi, lo + step);
+    }
+    return lo;
+}
+
 __global__ void __launch_bounds__(kPlaceNT)
     k_place(int32_t rb, int32_t re, const int64_t *rp_lu, const int64_t *row_off,
             const int32_t *pool, int32_t *ci_lu, int64_t base, int64_t total)
@@ -25,20 +42,13 @@ __global__ void __launch_bounds__(kPlaceNT)
          t0 += (int64_t)gridDim.x * kPlaceTile) {
         const int64_t s = base + t0;
         const int64_t e = base + (t0 + kPlaceTile < total ? t0 + kPlaceTile : total);
-        if (threadIdx.x == 0) {
-            int lo = rb, hi = re;  // first row with rp_lu[r] > s
-            while (lo < hi) {
-                const int mid = (lo + hi) >> 1;
-                if (rp_lu[mid] <= s) lo = mid + 1; else hi = mid;
+        if (threadIdx.x < 32) {  // rows r0 .. r1 overlap [s, e)
+            const int r0 = warp_row_search(rp_lu, rb, re, s);
+            const int r1 = warp_row_search(rp_lu, r0, re, e - 1);
+            if (threadIdx.x == 0) {
+                s_r0 = r0;
+                s_nr = r1 - r0 + 1;
             }
-            const int r0 = lo - 1;
-            hi = re;  // first row with rp_lu[r] >= e
-            while (lo < hi) {
-                const int mid = (lo + hi) >> 1;
-                if (rp_lu[mid] < e) lo = mid + 1; else hi = mid;
-            }
-            s_r0 = r0;
-            s_nr = lo - r0;
         }
         __syncthreads();
         const int r0 = s_r0, nr = s_nr;
@@ -46,14 +56,32 @@ __global__ void __launch_bounds__(kPlaceNT)
             for (int k = threadIdx.x; k <= nr; k += kPlaceNT) srp[k] = rp_lu[r0 + k];
             for (int k = threadIdx.x; k < nr; k += kPlaceNT) soff[k] = row_off[r0 + k];
             __syncthreads();
-            for (int64_t pos = s + threadIdx.x; pos < e; pos += kPlaceNT) {
-                int lo = 0, hi = nr;  // last k with srp[k] <= pos
-                while (hi - lo > 1) {
-                    const int mid = (lo + hi) >> 1;
-                    if (srp[mid] <= pos) lo = mid; else hi = mid;
+            // kPlaceU positions per thread per round, loads issued before any store
+            constexpr int kPlaceU = 4;
+            for (int64_t p0 = s + threadIdx.x; p0 < e; p0 += kPlaceNT * kPlaceU) {
+                int32_t v[kPlaceU];
+                bool ok[kPlaceU];
+#pragma unroll
+                for (int u = 0; u < kPlaceU; ++u) {
+                    const int64_t pos = p0 + (int64_t)u * kPlaceNT;
+                    ok[u] = false;
+                    v[u] = 0;
+                    if (pos < e) {
+                        int lo = 0, hi = nr;  // last k with srp[k] <= pos
+                        while (hi - lo > 1) {
+                            const int mid = (lo + hi) >> 1;
+                            if (srp[mid] <= pos) lo = mid; else hi = mid;
+                        }
+                        const int64_t off = soff[lo];
+                        if (off >= 0) {
+                            ok[u] = true;
+                            v[u] = __ldcs(pool + off + (pos - srp[lo]));
+                        }
+                    }
                 }
-                const int64_t off = soff[lo];
-                if (off >= 0) ci_lu[pos] = pool[off + (pos - srp[lo])];
+#pragma unroll
+                for (int u = 0; u < kPlaceU; ++u)
+                    if (ok[u]) __stcs(ci_lu + p0 + (int64_t)u * kPlaceNT, v[u]);
             }
         } else {
             for (int64_t pos = s + threadIdx.x; pos < e; pos += kPlaceNT) {

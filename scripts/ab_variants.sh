@@ -12,7 +12,7 @@ for l in sys.stdin:
     if l.startswith('{'):
         d = json.loads(l)
         print('$(basename $lib)', 'cfg$CFG', '%.3f ms/step' % d['ms_per_step'],
-              'count %.3f' % d['phases_ms']['count'], 'rows', d['plan']['rows_in_flight'])
+              'count %.3f' % d['phases_ms']['count'], 'emit %.3f' % d['phases_ms']['emit'], 'rows', d['plan']['rows_in_flight'])
 "
   done
 done
