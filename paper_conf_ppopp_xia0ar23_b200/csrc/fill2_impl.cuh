@@ -628,6 +628,17 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
         const long long t_row = p.row_prof ? clock64() : 0;
         const unsigned long long sv_row = h.sv;  // read and written by thread 0 only
         int n_bfs = 0, n_win = 0;
+#if LUSYM_PHASE_PROF  // diagnostic build: per-row cycles by phase of the threshold loop
+        long long ph_col = 0, ph_win = 0, ph_bfs = 0, ph_t = 0;
+#define PH_MARK(acc)                                         \
+    do {                                                     \
+        const long long ph_now = clock64();                  \
+        if (ph_t) acc += ph_now - ph_t;                      \
+        ph_t = ph_now;                                       \
+    } while (0)
+#else
+#define PH_MARK(acc) do { } while (0)
+#endif
         a.ucnt = 0;
         a.lmin = i;
         a.lmax = i;
@@ -680,8 +691,10 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                 h.tns = INT_MAX;
                 h.newmin = INT_MAX;
             }
+            PH_MARK(ph_bfs);
             const int wc = collect<NT, VIS>(bm, sm, dused ? dm : nullptr, ptr + 1, i, qA, cap,
                                            h.scan);
+            PH_MARK(ph_col);
             if (wc == 0) break;
             ++n_win;
             if (tid == 0) h.sv += wc;
@@ -777,6 +790,7 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                 dused = true;
             }
             __syncthreads();
+            PH_MARK(ph_win);
             if (m <= last && m == tns) {  // smallest pending threshold: below-exploration
                 bfs<NT, W, VIS>(p, h, bm, sm, qA, i, m, a);
                 ++n_bfs;
@@ -828,9 +842,18 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
         }
         if (p.row_prof && tid == 0) {
             p.row_prof[4 * (size_t)i + 0] = clock64() - t_row;
+#if LUSYM_PHASE_PROF
+            p.row_prof[4 * (size_t)i + 1] = ph_col;
+            p.row_prof[4 * (size_t)i + 2] = ph_win;
+            p.row_prof[4 * (size_t)i + 3] = ph_bfs;
+            (void)n_bfs;
+            (void)n_win;
+            (void)sv_row;
+#else
             p.row_prof[4 * (size_t)i + 1] = (long long)(h.sv - sv_row);
             p.row_prof[4 * (size_t)i + 2] = n_bfs;
             p.row_prof[4 * (size_t)i + 3] = n_win;
+#endif
         }
         // ---- clear the dirty word range (fill(:) = 0 for the next row, L115)
         clear_words<NT, VIS>(bm, sm, gmin >> 5, gmax >> 5);
