@@ -36,6 +36,9 @@ namespace f2 {
 #ifndef LUSYM_BATCH_TEST  // scan_level: load every neighbour's visited word before any atomic
 #define LUSYM_BATCH_TEST 0    // (A/B on B200: 3.7% slower on cfg2, 5% on cfg5 — kept as a knob)
 #endif
+#ifndef LUSYM_VPT  // frontier vertices per thread per round in plain BFS levels (1: scan_level)
+#define LUSYM_VPT 1
+#endif
 #ifndef LUSYM_TAM  // test_and_mark with one shared bit mask (0: visited() then mark())
 #define LUSYM_TAM 1
 #endif
@@ -514,6 +517,104 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
     if (SC && lane == 0 && nloc) atomicAdd(&h.sv, (unsigned long long)nloc);
 }
 
+// Plain level-synchronous variant of scan_level with VPT frontier vertices per thread per
+// round (LUSYM_VPT > 1): the per-round overhead (queue index, ballots, shared append) is
+// shared by VPT vertices; new frontier vertices still collect in f0..f2 across them.
+template <int NT, int W, int VIS, int VPT>
+__device__ __forceinline__ void scan_level_multi(const Fill2Params &p, Hdr &h,
+                                                 const VisMap<VIS> &bm, uint32_t *sm,
+                                                 const int32_t *L, const int32_t *gL, int cnt,
+                                                 int *ncnt, int32_t *NF, int32_t *gNF,
+                                                 const int i, const int t0, RowAcc &a)
+{
+    const int tid = threadIdx.x, lane = tid & 31;
+    const unsigned lt = (1u << lane) - 1u;
+    const uint32_t ncnt_s = (uint32_t)__cvta_generic_to_shared(ncnt);
+    for (int base = 0; base < cnt; base += NT * VPT) {
+        int c = 0, f0 = 0, f1 = 0, f2 = 0;
+#pragma unroll
+        for (int v = 0; v < VPT; ++v) {
+            const int k = base + v * NT + tid;
+            const bool valid = k < cnt;
+            int nb[ell_stride<W>()];
+#pragma unroll
+            for (int s = 0; s < ell_stride<W>(); ++s) nb[s] = 0;
+            bool heavy = false;
+            if (valid) {
+                const int f = k < p.q ? L[k] : __ldcg(gL + k);
+                load_nb<W>(p.ell, f, nb);
+                heavy = nb[0] == kHeavy;
+                if (!heavy) {
+#pragma unroll
+                    for (int s = 0; s < W; ++s) {
+                        const int w = nb[s];
+                        if (test_and_mark(bm, sm, w)) {
+                            if (w < t0) {
+                                if (c == 3) {
+                                    put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
+                                } else {
+                                    f2 = f1;
+                                    f1 = f0;
+                                    f0 = w;
+                                    ++c;
+                                }
+                            } else if (w > i) {
+                                ++a.ucnt;
+                                a.lmax = max(a.lmax, w);
+                            }
+                        }
+                    }
+                }
+            }
+            unsigned hm = __ballot_sync(kFull, valid && heavy);
+            while (hm) {
+                const int src = __ffs(hm) - 1;
+                hm &= hm - 1;
+                const int len = __shfl_sync(kFull, nb[1], src);
+                const int64_t off =
+                    heavy_off(__shfl_sync(kFull, nb[2], src), __shfl_sync(kFull, nb[3], src));
+                if (lane == 0) atomicAdd(&h.te, (unsigned long long)len);
+                for (int eb = 0; eb < len; eb += 32) {
+                    const int e = eb + lane;
+                    bool fr = false;
+                    int w = -1;
+                    if (e < len) {
+                        w = __ldg(p.ci + off + e);
+                        if (test_and_mark(bm, sm, w)) {
+                            if (w < t0) {
+                                fr = true;
+                            } else if (w > i) {
+                                ++a.ucnt;
+                                a.lmax = max(a.lmax, w);
+                            }
+                        }
+                    }
+                    push(fr, w, ncnt, NF, gNF, p.q);
+                }
+            }
+        }
+        const unsigned b1 = __ballot_sync(kFull, c & 1), b2 = __ballot_sync(kFull, c & 2);
+        if (b1 | b2) {
+            const int tot = __popc(b1) + 2 * __popc(b2);
+            int wbase = 0;
+            if (lane == 0)
+                asm volatile("atom.shared.add.u32 %0, [%1], %2;"
+                             : "=r"(wbase) : "r"(ncnt_s), "r"(tot) : "memory");
+            wbase = __shfl_sync(kFull, wbase, 0);
+            const int pos = wbase + __popc(b1 & lt) + 2 * __popc(b2 & lt);
+            if (wbase + tot <= p.q) {
+                if (c) NF[pos] = f0;
+                if (c >= 2) NF[pos + 1] = f1;
+                if (c == 3) NF[pos + 2] = f2;
+            } else {
+                if (c) put(pos, f0, NF, gNF, p.q);
+                if (c >= 2) put(pos + 1, f1, NF, gNF, p.q);
+                if (c == 3) put(pos + 2, f2, NF, gNF, p.q);
+            }
+        }
+    }
+}
+
 // Level-synchronous BFS from threshold t0 over unvisited vertices < t0 (Alg. 1).
 // Level lev reads queue lev&1 and writes queue (lev+1)&1 (shared, spilling to the CTA's two
 // HBM halves); the level counters rotate through h.cnt[0..2] so one barrier per level suffices.
@@ -539,6 +640,11 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_
             scan_level<NT, W, VIS, true>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
                                          fsize, &h.cnt[nxt], qA + (par ^ 1) * p.q,
                                          gA + (par ^ 1) * p.spill_cap, i, t0, a);
+        else if (LUSYM_VPT > 1)
+            scan_level_multi<NT, W, VIS, LUSYM_VPT>(p, h, bm, sm, qA + par * p.q,
+                                                    gA + par * p.spill_cap, fsize, &h.cnt[nxt],
+                                                    qA + (par ^ 1) * p.q,
+                                                    gA + (par ^ 1) * p.spill_cap, i, t0, a);
         else
             scan_level<NT, W, VIS, false>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
                                           fsize, &h.cnt[nxt], qA + (par ^ 1) * p.q,
