@@ -254,7 +254,7 @@ void free_handle(lu_sym *h)
 // classes fit more rows per SM.  Within a class the CTA size and queue capacity maximise
 // resident threads, then rows in flight; the HBM budget caps rows in flight.
 #ifndef LUSYM_KLOC  // self-continuation rounds in latency-bound classes (scan_level)
-#define LUSYM_KLOC 2
+#define LUSYM_KLOC 4
 #endif
 #ifndef LUSYM_KLOC_OCC  // ... those with at most this many rows per SM
 #define LUSYM_KLOC_OCC 2
