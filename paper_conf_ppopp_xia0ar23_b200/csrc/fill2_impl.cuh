@@ -36,6 +36,9 @@ namespace f2 {
 #ifndef LUSYM_BATCH_TEST  // scan_level: load every neighbour's visited word before any atomic
 #define LUSYM_BATCH_TEST 0    // (A/B on B200: 3.7% slower on cfg2, 5% on cfg5 — kept as a knob)
 #endif
+#ifndef LUSYM_FAST_SCAN  // scan_bits: warp-0 path for short ranges / full first windows
+#define LUSYM_FAST_SCAN 1
+#endif
 #ifndef LUSYM_VPT  // frontier vertices per thread per round in plain BFS levels (1: scan_level)
 #define LUSYM_VPT 1
 #endif
@@ -305,6 +308,48 @@ __device__ int scan_bits(const VisMap<VIS> &bm, const uint32_t *sm, const uint32
 {
     if (lo >= hi) return 0;
     const int wlo = lo >> 5, whi = (hi - 1) >> 5;
+#if LUSYM_FAST_SCAN
+    // warp 0 alone, two barriers instead of a block scan: the range fits 32 words, or (collect)
+    // its first 32 words already hold cap set bits — the common case on the serial threshold
+    // chain of heavy rows, where the pointer advances by a few words per window
+    if (whi - wlo < 32 || CAPPED) {
+        if (threadIdx.x < 32) {
+            const int lane = threadIdx.x;
+            const int w = wlo + lane;
+            uint32_t word = 0;
+            if (w <= whi) {
+                word = bm_word(bm, w);
+                if (w == wlo) word &= kFull << (lo & 31);
+                if (w == whi) {
+                    const int hb = (hi - 1) & 31;
+                    word &= (hb == 31) ? kFull : ((2u << hb) - 1u);
+                }
+                if (dm && word) word &= ~__ldcg(dm + w);
+            }
+            const int c = __popc(word);
+            int inc = c;
+#pragma unroll
+            for (int o = 1; o < 32; o <<= 1) {
+                const int y = __shfl_up_sync(kFull, inc, o);
+                if (lane >= o) inc += y;
+            }
+            const int total = __shfl_sync(kFull, inc, 31);
+            const bool ok = whi - wlo < 32 || total >= cap;
+            if (ok && WRITE) {
+                int pos = inc - c;
+                for (; word && !(CAPPED && pos >= cap); word &= word - 1, ++pos) {
+                    const int64_t o = base + pos;
+                    if (o < dcap) dst[o] = (w << 5) + __ffs(word) - 1;
+                }
+            }
+            if (lane == 0) sscan[33] = ok ? total : -1;
+        }
+        __syncthreads();
+        const int r = sscan[33];
+        __syncthreads();
+        if (r >= 0) return CAPPED && r > cap ? cap : r;
+    }
+#endif
     const bool wide = whi - wlo >= NT;
     int count = 0;
     for (int w0 = wlo; w0 <= whi; w0 += NT) {
