@@ -931,8 +931,6 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
             const int nptr = m > last ? last : (m == tns ? m : m - 1);
             // every visited bit in (ptr, nptr] is an L entry now (no BFS has marked below m yet):
             // emit / count them in increasing order as the pointer passes (L122-143)
-            Lcnt += emit_range<NT, VIS, MODE != kCount>(bm, sm, ptr + 1, nptr + 1, ldst, Lcnt, lcap,
-                                                       h.scan);
             if (nptr < last) {  // simple candidates beyond the pointer are finished: mark them
                 for (int k = tid; k < wc; k += NT) {
                     const int t = qA[k];
@@ -940,7 +938,11 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                 }
                 dused = true;
             }
-            __syncthreads();
+            // the barriers inside emit_range order these marks (and the reads of qA/qB) before
+            // the next collect and the BFS; an empty range has none, so add one
+            Lcnt += emit_range<NT, VIS, MODE != kCount>(bm, sm, ptr + 1, nptr + 1, ldst, Lcnt, lcap,
+                                                       h.scan);
+            if (nptr <= ptr) __syncthreads();
             PH_MARK(ph_win);
             if (m <= last && m == tns) {  // smallest pending threshold: below-exploration
                 bfs<NT, W, VIS>(p, h, bm, sm, qA, i, m, a);
