@@ -93,8 +93,8 @@ cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, in
 cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,
                         cudaStream_t s, bool chained = false);
 size_t scan_scratch_elems(int32_t n);
-cudaError_t count_far_rows(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
-                           unsigned long long *d_cnt, cudaStream_t s);
+cudaError_t count_far_entries(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
+                              unsigned long long *d_cnt, cudaStream_t s);
 
 // place_kernels.cu — symbolic_2 for staged rows: copy pool rows to their CSR slots
 cudaError_t place_rows(int32_t row_begin, int32_t row_end, const int64_t *rp_lu,

@@ -346,15 +346,17 @@ lu_status plan(lu_sym *h)
         }
         if (c.occ <= cur.occ && !(h->opts.flags & LU_F_FORCE_CLASSES)) break;
         if (!(h->opts.flags & LU_F_FORCE_CLASSES)) {
-            // rows of the new class with neighbours above its shared part would send their
-            // pattern marks to HBM; split only when that is rare (grids: rows within k of the
-            // boundary; circuits with hubs at the end: most rows)
-            unsigned long long far = 0;
-            CK(count_far_rows(n, h->rp, h->ci, nl * 32, h->dstats + 14, h->stream));
-            CK(cudaMemcpyAsync(&far, h->dstats + 14, 8, cudaMemcpyDeviceToHost, h->stream));
-            CK(cudaStreamSynchronize(h->stream));
+            // the new class's pattern marks above its shared part go to HBM atomics: split
+            // only while they are under a quarter of its entries (grids: the k entries per
+            // boundary row; ND-ordered circuits with hubs last: the hub and top-separator
+            // incidences, ~8%; unordered random matrices: about half, so no split)
+            unsigned long long far = 0, ent = 0;
             const int rows = nl * 32 < n ? nl * 32 : n;
-            if (far * 20 > (unsigned long long)rows) break;
+            CK(count_far_entries(n, h->rp, h->ci, nl * 32, h->dstats + 14, h->stream));
+            CK(cudaMemcpyAsync(&far, h->dstats + 14, 8, cudaMemcpyDeviceToHost, h->stream));
+            CK(cudaMemcpyAsync(&ent, h->rp + rows, 8, cudaMemcpyDeviceToHost, h->stream));
+            CK(cudaStreamSynchronize(h->stream));
+            if (far * 4 > ent) break;
         }
         const int lo = nl * 32 < hi ? nl * 32 : hi;  // rows i < 32*nl fit the smaller map
         const int sw_words = vis == kVisSmem ? nw32 : (vis == kVisSplit ? lbw : 0);

@@ -111,18 +111,18 @@ __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int
     if constexpr (S == 8) dst[1] = make_int4(out[4], out[5], out[6], out[7]);
 }
 
-// rows i < bound whose largest column is >= bound (their marks would leave a split map)
+// entries (i, j) of rows i < bound with j >= bound: pattern marks a split map sends to HBM
 __global__ void k_count_far(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
                             unsigned long long *cnt)
 {
     const int i = blockIdx.x * blockDim.x + threadIdx.x;
-    bool far = false;
+    unsigned c = 0;
     if (i < n && i < bound) {
-        const int64_t b = rp[i + 1];
-        far = b > rp[i] && ci[b - 1] >= bound;
+        const int64_t a = rp[i];
+        for (int64_t k = rp[i + 1] - 1; k >= a && ci[k] >= bound; --k) ++c;  // rows are sorted
     }
-    const unsigned m = __ballot_sync(kFull, far);
-    if ((threadIdx.x & 31) == 0 && m) atomicAdd(cnt, (unsigned long long)__popc(m));
+    c = __reduce_add_sync(kFull, c);
+    if ((threadIdx.x & 31) == 0 && c) atomicAdd(cnt, (unsigned long long)c);
 }
 
 // ---------------------------------------------------------------- scan (int32 -> int64)
@@ -245,8 +245,8 @@ cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, in
     return cudaGetLastError();
 }
 
-cudaError_t count_far_rows(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
-                           unsigned long long *d_cnt, cudaStream_t s)
+cudaError_t count_far_entries(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
+                              unsigned long long *d_cnt, cudaStream_t s)
 {
     cudaError_t e = cudaMemsetAsync(d_cnt, 0, sizeof(unsigned long long), s);
     const int rows = bound < n ? bound : n;
