@@ -20,7 +20,7 @@ import numpy as np
 __all__ = [
     "csr_from_edges", "lap2d", "lap3d", "circuit", "random_pattern",
     "tridiag", "arrow_first", "arrow_last", "band", "diag_only",
-    "config", "CONFIGS",
+    "config", "CONFIGS", "dominant_values",
 ]
 
 
@@ -38,6 +38,24 @@ def csr_from_edges(n: int, rows, cols):
     row_ptr = np.zeros(n + 1, dtype=np.int64)
     np.cumsum(counts, out=row_ptr[1:])
     return row_ptr, c
+
+
+def dominant_values(row_ptr, col_idx, seed: int, dtype=np.float64):
+    """Seeded values for a pattern (numeric phase): off-diagonal entries uniform
+    in [-1, 1), the diagonal 1 + (sum of |off-diagonal| in its row) + (same in its column), so
+    A is strictly diagonally dominant by rows and by columns and the pivot-free LU (reading
+    R29) is stable.  Rows without a stored diagonal keep only their off-diagonal values."""
+    rp = np.asarray(row_ptr, dtype=np.int64)
+    ci = np.asarray(col_idx, dtype=np.int64)
+    n = rp.size - 1
+    rng = np.random.default_rng(seed)
+    val = rng.uniform(-1.0, 1.0, size=ci.size)
+    row = np.repeat(np.arange(n, dtype=np.int64), np.diff(rp))
+    diag = row == ci
+    off = np.where(diag, 0.0, np.abs(val))
+    val[diag] = 1.0 + np.bincount(row, weights=off, minlength=n)[row[diag]] + \
+        np.bincount(ci, weights=off, minlength=n)[ci[diag]]
+    return val.astype(dtype)
 
 
 def _diag(n):
