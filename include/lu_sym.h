@@ -256,6 +256,38 @@ lu_status lu_level_types(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *
                          const int32_t *d_level, int32_t num_levels, int32_t min_cols,
                          int32_t max_sub_a, int32_t *d_type, int64_t *d_sub, void *stream);
 
+/*
+ * Numeric factorization (not part of the symbolic hot path) — Algorithm 2 of
+ * PAPER.md, the hybrid column-based right-looking LU (L165-204), pivot-free (reading R29),
+ * float values (the paper's precision).  As = "the non-zero filled-in matrix of A after
+ * symbolic analysis" (L175) is stored in the CSR of L+U (d_row_ptr_lu int64[n+1],
+ * d_col_idx_lu int32[nnz_lu], rows sorted, as lu_sym_emit writes them) as d_val_lu
+ * float[nnz_lu], one value per pattern entry.
+ *
+ * lu_numeric_scatter: d_val_lu = A's values (d_val_a float[nnz_a], on A's CSR d_row_ptr_a /
+ *   d_col_idx_a) at their L+U positions, 0 at fill entries.  LU_ERR_INPUT if an entry of A is
+ *   not in the pattern (the pattern is not A's L+U).  Synchronises.
+ *
+ * lu_numeric_factor: Algorithm 2 in place on d_val_lu: afterwards the strictly lower entries
+ *   hold L (unit diagonal implied) and the upper entries, diagonal included, hold U, A = L U.
+ *   Columns are processed level by level (L206-208) from the level schedule d_level_ptr
+ *   int64[num_levels+1] / d_level_cols int32[n] (lu_level_schedule), which MUST come from
+ *   lu_levelize with LU_DEP_GLU3: that rule makes every value a level reads final before the
+ *   level starts (under LU_DEP_U alone a U row may still be updated while it is read).
+ *   Columns of one level update shared sub-columns with float atomics, so the rounding order
+ *   (not the arithmetic) may vary from run to run.  The diagonal of every column must be in
+ *   the pattern and non-zero when its column is reached: else LU_ERR_INPUT ("zero pivot");
+ *   an update outside the pattern (a pattern that is not closed under elimination) is also
+ *   LU_ERR_INPUT.  Scratch (O(n + nnz(L))) is allocated per call.  Synchronises.
+ */
+lu_status lu_numeric_scatter(int32_t n, const int64_t *d_row_ptr_a, const int32_t *d_col_idx_a,
+                             const float *d_val_a, const int64_t *d_row_ptr_lu,
+                             const int32_t *d_col_idx_lu, int64_t nnz_lu, float *d_val_lu,
+                             void *stream);
+lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
+                            const int64_t *d_level_ptr, const int32_t *d_level_cols,
+                            int32_t num_levels, float *d_val_lu, void *stream);
+
 /* Copy the handle's statistics to *out (host). */
 lu_status lu_sym_get_stats(const lu_sym *h, lu_sym_stats *out);
 

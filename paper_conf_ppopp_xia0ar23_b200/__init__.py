@@ -28,7 +28,8 @@ from .parallel import (assemble_counts, assemble_pattern, partition_rows,  # noq
 
 __all__ = ["Symbolic", "LuSymError", "levelize", "level_schedule", "load_library", "library_path",
            "partition_rows", "assemble_counts", "assemble_pattern", "symbolic_distributed",
-           "row_cost_upper_bound", "DEP_U", "DEP_GLU3"]
+           "row_cost_upper_bound", "DEP_U", "DEP_GLU3", "numeric_scatter", "numeric_factor",
+           "factorize"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 # LUSYM_LIB selects an alternative build of the same library (kernel-variant experiments)
@@ -81,7 +82,8 @@ _lib = None
 EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sym_count",
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
             "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile",
-            "lu_level_schedule", "lu_sym_run_host", "lu_level_types"]
+            "lu_level_schedule", "lu_sym_run_host", "lu_level_types", "lu_numeric_scatter",
+            "lu_numeric_factor"]
 
 
 def library_path() -> str:
@@ -114,6 +116,10 @@ def load_library():
     lib.lu_level_schedule.restype = I32
     lib.lu_level_types.argtypes = [I32, P, P, P, I32, I32, I32, P, P, P]
     lib.lu_level_types.restype = I32
+    lib.lu_numeric_scatter.argtypes = [I32, P, P, P, P, P, I64, P, P]
+    lib.lu_numeric_scatter.restype = I32
+    lib.lu_numeric_factor.argtypes = [I32, P, P, P, P, I32, P, P]
+    lib.lu_numeric_factor.restype = I32
     lib.lu_sym_set_row_profile.restype = I32
     lib.lu_status_str.argtypes = [I32]
     lib.lu_status_str.restype = ctypes.c_char_p
@@ -354,6 +360,57 @@ def level_types(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, level: torch
         ctypes.c_void_p(typ.data_ptr()) if num_levels else None,
         ctypes.c_void_p(sub.data_ptr()) if num_levels else None, _stream_ptr(stream)))
     return typ, sub
+
+
+def numeric_scatter(row_ptr: torch.Tensor, col_idx: torch.Tensor, val: torch.Tensor,
+                    row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, stream=None):
+    """As (Alg. 2's input, L175): A's float values at their positions in the L+U pattern, 0 at
+    fill entries (lu_numeric_scatter).  Returns val_lu float32[nnz_lu] on the device."""
+    n = int(row_ptr_lu.numel()) - 1
+    nnz_lu = int(col_idx_lu.numel())
+    val_lu = torch.empty(max(nnz_lu, 1), dtype=torch.float32, device=row_ptr_lu.device)[:nnz_lu]
+    opt = lambda t: ctypes.c_void_p(t.data_ptr()) if t.numel() else None  # noqa: E731
+    _check(load_library().lu_numeric_scatter(
+        n, _dev(row_ptr, torch.int64, "row_ptr"), opt(col_idx), opt(val),
+        _dev(row_ptr_lu, torch.int64, "row_ptr_lu"), opt(col_idx_lu), nnz_lu, opt(val_lu),
+        _stream_ptr(stream)))
+    return val_lu
+
+
+def numeric_factor(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, level_ptr: torch.Tensor,
+                   level_cols: torch.Tensor, val_lu: torch.Tensor, stream=None):
+    """Algorithm 2 (L165-204) in place on val_lu (float32, CSR of L+U), level by level over a
+    schedule of GLU3-rule levels (lu_numeric_factor): L strictly below, U on and above the
+    diagonal.  Returns val_lu."""
+    n = int(row_ptr_lu.numel()) - 1
+    if val_lu.dtype != torch.float32 or not val_lu.is_cuda or not val_lu.is_contiguous():
+        raise TypeError("val_lu must be a contiguous CUDA float32 tensor")
+    nl = int(level_ptr.numel()) - 1
+    _check(load_library().lu_numeric_factor(
+        n, _dev(row_ptr_lu, torch.int64, "row_ptr_lu"),
+        ctypes.c_void_p(col_idx_lu.data_ptr()) if col_idx_lu.numel() else None,
+        _dev(level_ptr, torch.int64, "level_ptr"),
+        ctypes.c_void_p(level_cols.data_ptr()) if level_cols.numel() else None, nl,
+        ctypes.c_void_p(val_lu.data_ptr()) if val_lu.numel() else None, _stream_ptr(stream)))
+    return val_lu
+
+
+def factorize(row_ptr: torch.Tensor, col_idx: torch.Tensor, val: torch.Tensor,
+              options: Options | None = None, stream=None):
+    """End to end on this GPU: symbolic (fill2, Alg. 1/3), GLU3-rule levels (Alg. 5), the
+    level schedule and the numeric phase (Alg. 2).  Returns (row_ptr_lu, col_idx_lu, val_lu,
+    level_ptr, level_cols)."""
+    h = Symbolic(row_ptr, col_idx, options, stream=stream)
+    try:
+        _, rp_lu, ci_lu = h.run(stream=stream)
+        level, nl = levelize(rp_lu, ci_lu, rule="glu3", stream=stream)
+    finally:
+        h.close()
+    level_ptr, level_cols = level_schedule(level, max(nl, 1) if level.numel() else 0,
+                                           stream=stream)
+    val_lu = numeric_scatter(row_ptr, col_idx, val, rp_lu, ci_lu, stream=stream)
+    numeric_factor(rp_lu, ci_lu, level_ptr, level_cols, val_lu, stream=stream)
+    return rp_lu, ci_lu, val_lu, level_ptr, level_cols
 
 
 def symbolic_distributed(row_ptr: torch.Tensor, col_idx: torch.Tensor, group=None,

@@ -111,6 +111,15 @@ cudaError_t level_types(int32_t n, const int64_t *rp, const int32_t *ci, const i
 cudaError_t level_schedule(int32_t n, const int32_t *level, int32_t num_levels,
                            int64_t *level_ptr, int32_t *level_cols, cudaStream_t s);
 
+// numeric_kernels.cu — Algorithm 2 (numeric LU) on the L+U pattern, SURVEY 8(f4)
+cudaError_t numeric_scatter(int32_t n, const int64_t *rpa, const int32_t *cia, const float *va,
+                            const int64_t *rp, const int32_t *ci, int64_t nnz_lu, float *val,
+                            int *h_err, cudaStream_t s);
+cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
+                           const int64_t *h_level_ptr, const int32_t *level_cols,
+                           int32_t num_levels, int32_t num_sms, float *val, int *h_err,
+                           cudaStream_t s);
+
 // levelize_kernels.cu
 struct LevelizeScratch {
     int64_t *ustart = nullptr;  // [n] first strict-U position of row i

@@ -1147,6 +1147,51 @@ lu_status lu_level_types(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *
     return LU_OK;
 }
 
+lu_status lu_numeric_scatter(int32_t n, const int64_t *d_row_ptr_a, const int32_t *d_col_idx_a,
+                             const float *d_val_a, const int64_t *d_row_ptr_lu,
+                             const int32_t *d_col_idx_lu, int64_t nnz_lu, float *d_val_lu,
+                             void *stream)
+{
+    g_err.clear();
+    if (n < 0 || nnz_lu < 0) return fail(LU_ERR_ARG, "negative size");
+    if (n > 0 && (!d_row_ptr_a || !d_row_ptr_lu || (nnz_lu > 0 && (!d_col_idx_lu || !d_val_lu))))
+        return fail(LU_ERR_ARG, "null pointer");
+    int err = 0;
+    CK(numeric_scatter(n, d_row_ptr_a, d_col_idx_a, d_val_a, d_row_ptr_lu, d_col_idx_lu, nnz_lu,
+                       d_val_lu, &err, (cudaStream_t)stream));
+    if (err) return fail(LU_ERR_INPUT, "an entry of A is not in the L+U pattern");
+    return LU_OK;
+}
+
+lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
+                            const int64_t *d_level_ptr, const int32_t *d_level_cols,
+                            int32_t num_levels, float *d_val_lu, void *stream)
+{
+    g_err.clear();
+    if (n < 0 || num_levels < 0) return fail(LU_ERR_ARG, "negative size");
+    if (n == 0) return LU_OK;
+    if (num_levels < 1) return fail(LU_ERR_ARG, "num_levels must be >= 1 when n > 0");
+    if (!d_row_ptr_lu || !d_col_idx_lu || !d_level_ptr || !d_level_cols || !d_val_lu)
+        return fail(LU_ERR_ARG, "null pointer");
+    cudaStream_t s = (cudaStream_t)stream;
+    std::vector<int64_t> lp(num_levels + 1);
+    CK(cudaMemcpyAsync(lp.data(), d_level_ptr, sizeof(int64_t) * (num_levels + 1),
+                       cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (lp[0] != 0 || lp[num_levels] != n) return fail(LU_ERR_ARG, "level_ptr does not cover n");
+    for (int32_t l = 0; l < num_levels; ++l)
+        if (lp[l + 1] < lp[l]) return fail(LU_ERR_ARG, "level_ptr not monotone");
+    int dev = 0, sms = 0;
+    CK(cudaGetDevice(&dev));
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    int err = 0;
+    CK(numeric_factor(n, d_row_ptr_lu, d_col_idx_lu, lp.data(), d_level_cols, num_levels, sms,
+                      d_val_lu, &err, s));
+    if (err & 1) return fail(LU_ERR_INPUT, "zero pivot");
+    if (err) return fail(LU_ERR_INPUT, "update outside the L+U pattern");
+    return LU_OK;
+}
+
 lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
 {
     g_err.clear();

@@ -1,0 +1,290 @@
+// Numeric factorization on the symbolic pattern: Algorithm 2 of PAPER.md, the
+// hybrid column-based right-looking LU (L165-204), scheduled level by level (L206-208) on the
+// level-grouped column schedule (lu_level_schedule, Fig. 1(d)).  float values (the paper's
+// precision, L487), no pivoting (reading R29).
+//
+// Layout: As lives in the CSR of L+U that lu_sym_emit writes (rows sorted, reading R9) — the
+// paper's numeric phase reads a sorted CSC with a binary search for As(i,k) (Alg. 6);
+// here the search runs over the sorted ROW i for column k, the same search on the transposed
+// storage, so the symbolic output is consumed without a transpose of its values.  The only
+// derived structure is the column view of strict L (lines 2-6 and 9-11 walk "As(k,j) != 0 for
+// k > j"): per column j the rows i and CSR positions of its strict-lower entries, built with a
+// counting pass, a CUB scan and an atomic scatter (order inside a column is free: the updates
+// of one column commute).
+//
+// One launch per level (L206-208).  GLU3.0 picks one of three kernel modes per level type
+// (L208: block per column, warp per sub-column, kernel per column); here one kernel covers
+// all three: the level's (sub-column, L entry) pairs are flattened over a grid sized to them,
+// so a narrow level (type C, often a single column on a chain of levels) spreads its pairs
+// over the whole GPU and a wide one (type A) gets one pass.  Each pair locates As(i,k) by
+// binary search and subtracts with a float atomic: columns of one level may update the same
+// As(i,k) (a sub-column shared by independent columns).  The GLU3 dependency rule (reading
+// R12, LU_DEP_GLU3) guarantees that nothing a level reads — its own L columns, its U rows —
+// is written within that level.  The update uses the column's undivided entries (reading
+// R31), As(i,k) -= As(i,j) * (As(j,k) / As(j,j)), and lines 2-6 (As(k,j) /= As(j,j)) run once
+// for all columns at the end: a column's strict-L entries are read only by its own update and
+// are final once its level starts, so no barrier separates lines 2-6 from lines 7-14.
+#include "internal.h"
+
+#include <cub/device/device_scan.cuh>
+
+#include <vector>
+
+namespace lusym {
+namespace {
+
+constexpr int kErrPivot = 1, kErrPattern = 2;
+
+// warp per row i: diagonal position (or -1) and the strict-lower entry count of every column
+__global__ void k_diag_lcount(int32_t n, const int64_t *rp, const int32_t *ci, int64_t *dpos,
+                              int32_t *lcnt)
+{
+    const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    const int lane = threadIdx.x & 31;
+    if (i >= n) return;
+    if (lane == 0) dpos[i] = -1;
+    __syncwarp();
+    for (int64_t p = rp[i] + lane; p < rp[i + 1]; p += 32) {
+        const int c = ci[p];
+        if (c < i)
+            atomicAdd(&lcnt[c], 1);
+        else if (c == i)
+            dpos[i] = p;
+    }
+}
+
+// warp per row i: strict-lower entry (i, c) -> slot of column c (rows i and CSR positions)
+__global__ void k_lfill(int32_t n, const int64_t *rp, const int32_t *ci, int64_t *cursor,
+                        int32_t *lrow, int64_t *lpos)
+{
+    const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    const int lane = threadIdx.x & 31;
+    if (i >= n) return;
+    for (int64_t p = rp[i] + lane; p < rp[i + 1]; p += 32) {
+        const int c = ci[p];
+        if (c >= i) break;  // rows are sorted: the strict-lower entries come first
+        const int64_t e = atomicAdd(reinterpret_cast<unsigned long long *>(cursor + c), 1ull);
+        lrow[e] = i;
+        lpos[e] = p;
+    }
+}
+
+// position of column k in the sorted row [lo, hi) of ci, -1 if absent (Alg. 6's binary search,
+// L322-348, on the row-sorted storage)
+__device__ __forceinline__ int64_t find_col(const int32_t *ci, int64_t lo, int64_t hi, int k)
+{
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        const int c = __ldg(ci + mid);
+        if (c == k) return mid;
+        if (c < k)
+            lo = mid + 1;
+        else
+            hi = mid;
+    }
+    return -1;
+}
+
+// warp per row: As = A's values at their L+U positions, 0 at fill (Alg. 2's input, L175)
+__global__ void k_scatter(int32_t n, const int64_t *rpa, const int32_t *cia, const float *va,
+                          const int64_t *rp, const int32_t *ci, float *val, int *err)
+{
+    const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    const int lane = threadIdx.x & 31;
+    if (i >= n) return;
+    for (int64_t q = rpa[i] + lane; q < rpa[i + 1]; q += 32) {
+        const int64_t p = find_col(ci, rp[i], rp[i + 1], cia[q]);
+        if (p < 0)
+            atomicOr(err, kErrPattern);
+        else
+            val[p] = va[q];
+    }
+}
+
+__global__ void k_zero(int64_t m, float *v)
+{
+    for (int64_t p = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; p < m;
+         p += (int64_t)gridDim.x * blockDim.x)
+        v[p] = 0.f;
+}
+
+// Alg. 2 pairs of a column: |strict L(:,j)| * |U(j, >j)| rank-1 updates (0 without a diagonal)
+__global__ void k_pairs(int32_t n, const int32_t *cols, const int64_t *rp, const int64_t *dpos,
+                        const int64_t *cptr, int64_t *cost)
+{
+    const int pos = blockIdx.x * blockDim.x + threadIdx.x;
+    if (pos > n) return;
+    if (pos == n) {
+        cost[n] = 0;
+        return;
+    }
+    const int j = cols[pos];
+    const int64_t dp = dpos[j];
+    cost[pos] = dp < 0 ? 0 : (cptr[j + 1] - cptr[j]) * (rp[j + 1] - dp - 1);
+}
+
+// One level of Algorithm 2 (lines 7-14), its (sub-column, L entry) pairs flattened over the
+// grid: pair g of the level belongs to the column at position pos of level_cols with
+// W[pos] <= g < W[pos+1] (W = exclusive scan of the per-column pair counts in schedule order).
+// The update uses the column's undivided entries, As(i,k) -= As(i,j) * (As(j,k) / As(j,j)),
+// so it needs no barrier after lines 2-6, which k_divide applies at the end (reading R31).
+__global__ void __launch_bounds__(256) k_update_level(
+    int32_t pos0, int32_t pos1, int64_t total, const int64_t *__restrict__ W,
+    const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
+    const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
+    const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
+    const int64_t *__restrict__ lpos, float *val, int *err)
+{
+    const int64_t wbase = W[pos0];
+    for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total;
+         t += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t g = wbase + t;
+        int lo = pos0, hi = pos1 - 1;  // last pos in [pos0, pos1) with W[pos] <= g
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (__ldg(W + mid) <= g)
+                lo = mid;
+            else
+                hi = mid - 1;
+        }
+        const int j = __ldg(cols + lo);
+        const int64_t r = g - __ldg(W + lo);
+        const int64_t e0 = __ldg(cptr + j), nl = __ldg(cptr + j + 1) - e0;
+        const int64_t qu = r / nl, e = r - qu * nl;
+        const int64_t dp = __ldg(dpos + j), q = dp + 1 + qu;
+        const int k = __ldg(ci + q);
+        const float d = val[dp];
+        const float u = val[q] / d;
+        const int i = __ldg(lrow + e0 + e);
+        const float l = val[__ldg(lpos + e0 + e)];
+        const int64_t p = find_col(ci, __ldg(rp + i), __ldg(rp + i + 1), k);
+        if (p < 0) {
+            atomicOr(err, kErrPattern);
+            continue;
+        }
+        atomicAdd(val + p, -l * u);
+    }
+}
+
+// lines 2-6 for every column at once (each column's strict-L entries and pivot are final once
+// its level has run), and the pivot check of every column: warp per row i
+__global__ void k_divide(int32_t n, const int64_t *rp, const int32_t *ci, const int64_t *dpos,
+                         float *val, int *err)
+{
+    const int i = (int)((blockIdx.x * (int64_t)blockDim.x + threadIdx.x) >> 5);
+    const int lane = threadIdx.x & 31;
+    if (i >= n) return;
+    if (lane == 0 && (dpos[i] < 0 || val[dpos[i]] == 0.f)) atomicOr(err, kErrPivot);
+    for (int64_t p = rp[i] + lane; p < rp[i + 1]; p += 32) {
+        const int c = ci[p];
+        if (c >= i) break;
+        const int64_t dp = dpos[c];
+        if (dp >= 0) val[p] = val[p] / val[dp];
+    }
+}
+
+}  // namespace
+
+cudaError_t numeric_scatter(int32_t n, const int64_t *rpa, const int32_t *cia, const float *va,
+                            const int64_t *rp, const int32_t *ci, int64_t nnz_lu, float *val,
+                            int *h_err, cudaStream_t s)
+{
+    *h_err = 0;
+    if (n <= 0) return cudaSuccess;
+    int *err = nullptr;
+    cudaError_t e;
+    if ((e = dev_alloc((void **)&err, sizeof(int), s)) != cudaSuccess) return e;
+    if ((e = cudaMemsetAsync(err, 0, sizeof(int), s)) != cudaSuccess) goto out;
+    if (nnz_lu > 0) k_zero<<<1184, 256, 0, s>>>(nnz_lu, val);
+    k_scatter<<<(int)(((int64_t)n * 32 + 255) / 256), 256, 0, s>>>(n, rpa, cia, va, rp, ci, val,
+                                                                      err);
+    if ((e = cudaGetLastError()) != cudaSuccess) goto out;
+    if ((e = cudaMemcpyAsync(h_err, err, sizeof(int), cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+        goto out;
+    e = cudaStreamSynchronize(s);
+out:
+    dev_free(err, s);
+    return e;
+}
+
+cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
+                           const int64_t *h_level_ptr, const int32_t *level_cols,
+                           int32_t num_levels, int32_t num_sms, float *val, int *h_err,
+                           cudaStream_t s)
+{
+    *h_err = 0;
+    if (n <= 0) return cudaSuccess;
+    int64_t *dpos = nullptr, *cptr = nullptr, *cursor = nullptr, *lpos = nullptr, *cost = nullptr,
+            *W = nullptr;
+    int32_t *lcnt = nullptr, *lrow = nullptr;
+    int *err = nullptr;
+    void *tmp = nullptr;
+    size_t tmp_bytes = 0, tmp2_bytes = 0;
+    int64_t nl_total = 0;
+    std::vector<int64_t> hW;
+    const int wgrid = (int)(((int64_t)n * 32 + 255) / 256);
+    cudaError_t e;
+#define NK(x)                                                                                  \
+    do {                                                                                       \
+        if ((e = (x)) != cudaSuccess) goto out;                                                \
+    } while (0)
+    NK(dev_alloc((void **)&dpos, sizeof(int64_t) * n, s));
+    NK(dev_alloc((void **)&cptr, sizeof(int64_t) * (n + 1), s));
+    NK(dev_alloc((void **)&cursor, sizeof(int64_t) * (n + 1), s));
+    NK(dev_alloc((void **)&cost, sizeof(int64_t) * (n + 1), s));
+    NK(dev_alloc((void **)&W, sizeof(int64_t) * (n + 1), s));
+    NK(dev_alloc((void **)&lcnt, sizeof(int32_t) * (n + 1), s));
+    NK(dev_alloc((void **)&err, sizeof(int), s));
+    NK(cudaMemsetAsync(lcnt, 0, sizeof(int32_t) * (n + 1), s));
+    NK(cudaMemsetAsync(err, 0, sizeof(int), s));
+    // column view of strict L: counts, offsets (CUB scan), atomic scatter
+    k_diag_lcount<<<wgrid, 256, 0, s>>>(n, rp, ci, dpos, lcnt);
+    NK(cudaGetLastError());
+    NK(cub::DeviceScan::ExclusiveSum(nullptr, tmp_bytes, lcnt, cptr, n + 1, s));
+    NK(cub::DeviceScan::ExclusiveSum(nullptr, tmp2_bytes, cost, W, n + 1, s));
+    NK(dev_alloc(&tmp, tmp_bytes > tmp2_bytes ? tmp_bytes : tmp2_bytes, s));
+    NK(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, lcnt, cptr, n + 1, s));
+    NK(cudaMemcpyAsync(&nl_total, cptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NK(cudaStreamSynchronize(s));
+    NK(dev_alloc((void **)&lrow, sizeof(int32_t) * (nl_total ? nl_total : 1), s));
+    NK(dev_alloc((void **)&lpos, sizeof(int64_t) * (nl_total ? nl_total : 1), s));
+    NK(cudaMemcpyAsync(cursor, cptr, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToDevice, s));
+    k_lfill<<<wgrid, 256, 0, s>>>(n, rp, ci, cursor, lrow, lpos);
+    // pair counts in schedule order and their scan W: level l owns pairs [W[lp[l]], W[lp[l+1]])
+    k_pairs<<<(n + 256) / 256, 256, 0, s>>>(n, level_cols, rp, dpos, cptr, cost);
+    NK(cudaGetLastError());
+    NK(cub::DeviceScan::ExclusiveSum(tmp, tmp2_bytes, cost, W, n + 1, s));
+    hW.resize(n + 1);
+    NK(cudaMemcpyAsync(hW.data(), W, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, s));
+    NK(cudaStreamSynchronize(s));
+    // levels in order (L206-208), one launch each, grid sized to the level's pairs
+    for (int32_t l = 0; l < num_levels; ++l) {
+        const int32_t p0 = (int32_t)h_level_ptr[l], p1 = (int32_t)h_level_ptr[l + 1];
+        const int64_t total = hW[p1] - hW[p0];
+        if (p1 <= p0 || total <= 0) continue;
+        const int64_t blocks = (total + 255) / 256;
+        const int grid = (int)(blocks < (int64_t)num_sms * 8 ? blocks : (int64_t)num_sms * 8);
+        k_update_level<<<grid, 256, 0, s>>>(p0, p1, total, W, level_cols, rp, ci, dpos, cptr,
+                                            lrow, lpos, val, err);
+    }
+    NK(cudaGetLastError());
+    k_divide<<<wgrid, 256, 0, s>>>(n, rp, ci, dpos, val, err);
+    NK(cudaGetLastError());
+    NK(cudaMemcpyAsync(h_err, err, sizeof(int), cudaMemcpyDeviceToHost, s));
+    NK(cudaStreamSynchronize(s));
+#undef NK
+out:
+    dev_free(dpos, s);
+    dev_free(cptr, s);
+    dev_free(cursor, s);
+    dev_free(cost, s);
+    dev_free(W, s);
+    dev_free(lcnt, s);
+    dev_free(lrow, s);
+    dev_free(lpos, s);
+    dev_free(err, s);
+    dev_free(tmp, s);
+    return e;
+}
+
+}  // namespace lusym
