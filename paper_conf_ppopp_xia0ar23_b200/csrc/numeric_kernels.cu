@@ -17,7 +17,8 @@
 // all three: the level's (sub-column, L entry) pairs are flattened over a grid sized to them,
 // so a narrow level (type C, often a single column on a chain of levels) spreads its pairs
 // over the whole GPU and a wide one (type A) gets one pass.  Each pair locates As(i,k) by
-// binary search and subtracts with a float atomic: columns of one level may update the same
+// (first entry of row i past j, then rank) and subtracts with a float atomic: columns of one
+// level may update the same
 // As(i,k) (a sub-column shared by independent columns).  The GLU3 dependency rule (reading
 // R12, LU_DEP_GLU3) guarantees that nothing a level reads — its own L columns, its U rows —
 // is written within that level.  The update uses the column's undivided entries (reading
@@ -149,15 +150,23 @@ __global__ void __launch_bounds__(256) k_update_level(
         }
         const int j = __ldg(cols + lo);
         const int64_t r = g - __ldg(W + lo);
-        const int64_t e0 = __ldg(cptr + j), nl = __ldg(cptr + j + 1) - e0;
-        const int64_t qu = r / nl, e = r - qu * nl;
-        const int64_t dp = __ldg(dpos + j), q = dp + 1 + qu;
-        const int k = __ldg(ci + q);
+        const int64_t e0 = __ldg(cptr + j);
+        const int64_t dp = __ldg(dpos + j), u0 = dp + 1, nu = __ldg(rp + j + 1) - u0;
+        // L entry outer, sub-column inner: the lanes of a warp share row i and walk U(j,:),
+        // so their loads and atomics hit consecutive addresses of row j and row i
+        const int64_t e = r / nu, qu = r - e * nu;
+        const int k = __ldg(ci + u0 + qu);
         const float d = val[dp];
-        const float u = val[q] / d;
+        const float u = val[u0 + qu] / d;
         const int i = __ldg(lrow + e0 + e);
-        const float l = val[__ldg(lpos + e0 + e)];
-        const int64_t p = find_col(ci, __ldg(rp + i), __ldg(rp + i + 1), k);
+        const int64_t pij = __ldg(lpos + e0 + e);
+        const float l = val[pij];
+        // row i's entries above j contain U(j,:) (the pattern is closed under elimination) and
+        // start right after As(i,j), so k sits at rank >= qu among them: a direct hit when the
+        // two rows agree (a full band), else a binary search of the rest (Alg. 6)
+        const int64_t rend = __ldg(rp + i + 1);
+        int64_t p = pij + 1 + qu;
+        if (p >= rend || __ldg(ci + p) != k) p = p < rend ? find_col(ci, p, rend, k) : -1;
         if (p < 0) {
             atomicOr(err, kErrPattern);
             continue;
