@@ -116,7 +116,8 @@ cudaError_t numeric_scatter(int32_t n, const int64_t *rpa, const int32_t *cia, c
                             const int64_t *rp, const int32_t *ci, int64_t nnz_lu, float *val,
                             int *h_err, cudaStream_t s);
 cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
-                           const int64_t *h_level_ptr, const int32_t *level_cols,
+                           const int64_t *h_level_ptr, const int64_t *level_ptr_d,
+                           const int32_t *level_cols,
                            int32_t num_levels, int32_t num_sms, float *val, int *h_err,
                            cudaStream_t s);
 

@@ -1185,7 +1185,8 @@ lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_
     CK(cudaGetDevice(&dev));
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
     int err = 0;
-    CK(numeric_factor(n, d_row_ptr_lu, d_col_idx_lu, lp.data(), d_level_cols, num_levels, sms,
+    CK(numeric_factor(n, d_row_ptr_lu, d_col_idx_lu, lp.data(), d_level_ptr, d_level_cols,
+                      num_levels, sms,
                       d_val_lu, &err, s));
     if (err & 1) return fail(LU_ERR_INPUT, "zero pivot");
     if (err) return fail(LU_ERR_INPUT, "update outside the L+U pattern");

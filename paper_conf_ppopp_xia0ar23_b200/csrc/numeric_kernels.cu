@@ -27,12 +27,17 @@
 // are final once its level starts, so no barrier separates lines 2-6 from lines 7-14.
 #include "internal.h"
 
+#include <cooperative_groups.h>
 #include <cub/device/device_scan.cuh>
+
+#include <cstdlib>
 
 #include <vector>
 
 namespace lusym {
 namespace {
+
+namespace cg = cooperative_groups;
 
 constexpr int kErrPivot = 1, kErrPattern = 2;
 
@@ -129,6 +134,47 @@ __global__ void k_pairs(int32_t n, const int32_t *cols, const int64_t *rp, const
 // W[pos] <= g < W[pos+1] (W = exclusive scan of the per-column pair counts in schedule order).
 // The update uses the column's undivided entries, As(i,k) -= As(i,j) * (As(j,k) / As(j,j)),
 // so it needs no barrier after lines 2-6, which k_divide applies at the end (reading R31).
+__device__ __forceinline__ void update_pair(
+    int64_t g, int32_t pos0, int32_t pos1, const int64_t *__restrict__ W,
+    const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
+    const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
+    const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
+    const int64_t *__restrict__ lpos, float *val, int *err)
+{
+    int lo = pos0, hi = pos1 - 1;  // last pos in [pos0, pos1) with W[pos] <= g
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (__ldg(W + mid) <= g)
+            lo = mid;
+        else
+            hi = mid - 1;
+    }
+    const int j = __ldg(cols + lo);
+    const int64_t r = g - __ldg(W + lo);
+    const int64_t e0 = __ldg(cptr + j);
+    const int64_t dp = __ldg(dpos + j), u0 = dp + 1, nu = __ldg(rp + j + 1) - u0;
+    // L entry outer, sub-column inner: the lanes of a warp share row i and walk U(j,:),
+    // so their loads and atomics hit consecutive addresses of row j and row i
+    const int64_t e = r / nu, qu = r - e * nu;
+    const int k = __ldg(ci + u0 + qu);
+    const float d = val[dp];
+    const float u = val[u0 + qu] / d;
+    const int i = __ldg(lrow + e0 + e);
+    const int64_t pij = __ldg(lpos + e0 + e);
+    const float l = val[pij];
+    // row i's entries above j contain U(j,:) (the pattern is closed under elimination) and
+    // start right after As(i,j), so k sits at rank >= qu among them: a direct hit when the
+    // two rows agree (a full band), else a binary search of the rest (Alg. 6)
+    const int64_t rend = __ldg(rp + i + 1);
+    int64_t p = pij + 1 + qu;
+    if (p >= rend || __ldg(ci + p) != k) p = p < rend ? find_col(ci, p, rend, k) : -1;
+    if (p < 0) {
+        atomicOr(err, kErrPattern);
+        return;
+    }
+    atomicAdd(val + p, -l * u);
+}
+
 __global__ void __launch_bounds__(256) k_update_level(
     int32_t pos0, int32_t pos1, int64_t total, const int64_t *__restrict__ W,
     const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
@@ -138,40 +184,31 @@ __global__ void __launch_bounds__(256) k_update_level(
 {
     const int64_t wbase = W[pos0];
     for (int64_t t = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; t < total;
-         t += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t g = wbase + t;
-        int lo = pos0, hi = pos1 - 1;  // last pos in [pos0, pos1) with W[pos] <= g
-        while (lo < hi) {
-            const int mid = (lo + hi + 1) >> 1;
-            if (__ldg(W + mid) <= g)
-                lo = mid;
-            else
-                hi = mid - 1;
-        }
-        const int j = __ldg(cols + lo);
-        const int64_t r = g - __ldg(W + lo);
-        const int64_t e0 = __ldg(cptr + j);
-        const int64_t dp = __ldg(dpos + j), u0 = dp + 1, nu = __ldg(rp + j + 1) - u0;
-        // L entry outer, sub-column inner: the lanes of a warp share row i and walk U(j,:),
-        // so their loads and atomics hit consecutive addresses of row j and row i
-        const int64_t e = r / nu, qu = r - e * nu;
-        const int k = __ldg(ci + u0 + qu);
-        const float d = val[dp];
-        const float u = val[u0 + qu] / d;
-        const int i = __ldg(lrow + e0 + e);
-        const int64_t pij = __ldg(lpos + e0 + e);
-        const float l = val[pij];
-        // row i's entries above j contain U(j,:) (the pattern is closed under elimination) and
-        // start right after As(i,j), so k sits at rank >= qu among them: a direct hit when the
-        // two rows agree (a full band), else a binary search of the rest (Alg. 6)
-        const int64_t rend = __ldg(rp + i + 1);
-        int64_t p = pij + 1 + qu;
-        if (p >= rend || __ldg(ci + p) != k) p = p < rend ? find_col(ci, p, rend, k) : -1;
-        if (p < 0) {
-            atomicOr(err, kErrPattern);
-            continue;
-        }
-        atomicAdd(val + p, -l * u);
+         t += (int64_t)gridDim.x * blockDim.x)
+        update_pair(wbase + t, pos0, pos1, W, cols, rp, ci, dpos, cptr, lrow, lpos, val, err);
+}
+
+// All levels in one cooperative launch (persistent grid, kCoopNT threads x co-resident CTAs):
+// a grid-wide barrier separates consecutive levels instead of a kernel boundary, which on a
+// chain of single-column levels (natural-order grids) is most of the per-level cost.
+constexpr int kCoopNT = 1024;
+__global__ void __launch_bounds__(kCoopNT, 2) k_update_levels_coop(
+    int32_t num_levels, const int64_t *__restrict__ lptr, const int64_t *__restrict__ W,
+    const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
+    const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
+    const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
+    const int64_t *__restrict__ lpos, float *val, int *err)
+{
+    cg::grid_group grid = cg::this_grid();
+    const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
+    const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+    for (int32_t l = 0; l < num_levels; ++l) {
+        const int32_t pos0 = (int32_t)__ldg(lptr + l), pos1 = (int32_t)__ldg(lptr + l + 1);
+        const int64_t wbase = __ldg(W + pos0), total = __ldg(W + pos1) - wbase;
+        if (total <= 0) continue;  // uniform across the grid: no barrier needed
+        for (int64_t t = tid; t < total; t += stride)
+            update_pair(wbase + t, pos0, pos1, W, cols, rp, ci, dpos, cptr, lrow, lpos, val, err);
+        grid.sync();
     }
 }
 
@@ -217,7 +254,8 @@ out:
 }
 
 cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
-                           const int64_t *h_level_ptr, const int32_t *level_cols,
+                           const int64_t *h_level_ptr, const int64_t *level_ptr_d,
+                           const int32_t *level_cols,
                            int32_t num_levels, int32_t num_sms, float *val, int *h_err,
                            cudaStream_t s)
 {
@@ -266,15 +304,36 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
     hW.resize(n + 1);
     NK(cudaMemcpyAsync(hW.data(), W, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, s));
     NK(cudaStreamSynchronize(s));
-    // levels in order (L206-208), one launch each, grid sized to the level's pairs
-    for (int32_t l = 0; l < num_levels; ++l) {
-        const int32_t p0 = (int32_t)h_level_ptr[l], p1 = (int32_t)h_level_ptr[l + 1];
-        const int64_t total = hW[p1] - hW[p0];
-        if (p1 <= p0 || total <= 0) continue;
-        const int64_t blocks = (total + 255) / 256;
-        const int grid = (int)(blocks < (int64_t)num_sms * 8 ? blocks : (int64_t)num_sms * 8);
-        k_update_level<<<grid, 256, 0, s>>>(p0, p1, total, W, level_cols, rp, ci, dpos, cptr,
-                                            lrow, lpos, val, err);
+    // levels in order (L206-208): one cooperative launch with a grid barrier per level, or
+    // (LUSYM_NUMERIC_LAUNCH_PER_LEVEL=1, or no co-residency) one launch per level with a grid
+    // sized to the level's pairs
+    {
+        int occ = 0;
+        const char *ev = getenv("LUSYM_NUMERIC_LAUNCH_PER_LEVEL");
+        const bool per_level = ev && ev[0] == '1';
+        if (!per_level)
+            NK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_update_levels_coop, kCoopNT,
+                                                             0));
+        if (!per_level && occ > 0) {
+            int32_t nlv = num_levels;
+            const int64_t *lptr_d = level_ptr_d;
+            void *args[] = {&nlv, &lptr_d, &W, &level_cols, &rp, &ci, &dpos, &cptr, &lrow, &lpos,
+                            &val, &err};
+            NK(cudaLaunchCooperativeKernel((const void *)k_update_levels_coop,
+                                           dim3(num_sms * (occ < 2 ? occ : 2)), dim3(kCoopNT),
+                                           args, 0, s));
+        } else {
+            for (int32_t l = 0; l < num_levels; ++l) {
+                const int32_t p0 = (int32_t)h_level_ptr[l], p1 = (int32_t)h_level_ptr[l + 1];
+                const int64_t total = hW[p1] - hW[p0];
+                if (p1 <= p0 || total <= 0) continue;
+                const int64_t blocks = (total + 255) / 256;
+                const int grid =
+                    (int)(blocks < (int64_t)num_sms * 8 ? blocks : (int64_t)num_sms * 8);
+                k_update_level<<<grid, 256, 0, s>>>(p0, p1, total, W, level_cols, rp, ci, dpos,
+                                                    cptr, lrow, lpos, val, err);
+            }
+        }
     }
     NK(cudaGetLastError());
     k_divide<<<wgrid, 256, 0, s>>>(n, rp, ci, dpos, val, err);

@@ -42,7 +42,9 @@ def run(name, rp, ci, reps=3):
         if r:
             ts.append(e0.elapsed_time(e1))
     ms = float(np.median(ts))
-    print(json.dumps({"workload": name, "n": n, "nnz_lu": int(len(cih)), "levels_glu3": nl,
+    import os
+    mode = "per-level" if os.environ.get("LUSYM_NUMERIC_LAUNCH_PER_LEVEL") == "1" else "coop"
+    print(json.dumps({"workload": name, "mode": mode, "n": n, "nnz_lu": int(len(cih)), "levels_glu3": nl,
                       "updates": updates, "ms": ms, "gflops": 2 * updates / ms / 1e6,
                       "us_per_level": 1e3 * ms / max(nl, 1)}), flush=True)
 

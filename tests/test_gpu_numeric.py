@@ -153,3 +153,11 @@ def test_empty():
     ci = np.zeros(0, dtype=np.int32)
     out = gpu_factor(rp, ci, np.zeros(0, dtype=np.float32))
     assert out[2].size == 0
+
+
+def test_per_level_launches(monkeypatch):
+    """The per-level launch path (LUSYM_NUMERIC_LAUNCH_PER_LEVEL=1) against the same bars."""
+    monkeypatch.setenv("LUSYM_NUMERIC_LAUNCH_PER_LEVEL", "1")
+    for k, (rp, ci) in enumerate([gen.lap2d(20), gen.circuit(32, 2),
+                                  gen.random_pattern(150, 3.0, seed=4, zero_free_diag=True)]):
+        check_case(rp, ci, 20 + k, tag=f"per-level {k}")
