@@ -188,11 +188,64 @@ __global__ void __launch_bounds__(256) k_update_level(
         update_pair(wbase + t, pos0, pos1, W, cols, rp, ci, dpos, cptr, lrow, lpos, val, err);
 }
 
+// Positions one pair touches, from the read-only index arrays only (row j's U entry q, the
+// pivot dp, As(i,j) at pij, the target As(i,k) at p, -1 if outside the pattern).  The values
+// are read after the level barrier; the indices can be resolved before it.
+struct PairPos {
+    int64_t q, dp, pij, p;
+};
+
+__device__ __forceinline__ PairPos pair_pos(
+    int64_t g, int32_t pos0, int32_t pos1, const int64_t *__restrict__ W,
+    const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
+    const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
+    const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
+    const int64_t *__restrict__ lpos)
+{
+    int lo = pos0, hi = pos1 - 1;
+    while (lo < hi) {
+        const int mid = (lo + hi + 1) >> 1;
+        if (__ldg(W + mid) <= g)
+            lo = mid;
+        else
+            hi = mid - 1;
+    }
+    const int j = __ldg(cols + lo);
+    const int64_t r = g - __ldg(W + lo);
+    const int64_t e0 = __ldg(cptr + j);
+    PairPos pp;
+    pp.dp = __ldg(dpos + j);
+    const int64_t u0 = pp.dp + 1, nu = __ldg(rp + j + 1) - u0;
+    const int64_t e = r / nu, qu = r - e * nu;
+    pp.q = u0 + qu;
+    const int k = __ldg(ci + pp.q);
+    const int i = __ldg(lrow + e0 + e);
+    pp.pij = __ldg(lpos + e0 + e);
+    const int64_t rend = __ldg(rp + i + 1);
+    int64_t p = pp.pij + 1 + qu;
+    if (p >= rend || __ldg(ci + p) != k) p = p < rend ? find_col(ci, p, rend, k) : -1;
+    pp.p = p;
+    return pp;
+}
+
+__device__ __forceinline__ void pair_apply(const PairPos &pp, float *val, int *err)
+{
+    if (pp.p < 0) {
+        atomicOr(err, kErrPattern);
+        return;
+    }
+    const float u = val[pp.q] / val[pp.dp];
+    atomicAdd(val + pp.p, -val[pp.pij] * u);
+}
+
 // All levels in one cooperative launch (persistent grid, kCoopNT threads x co-resident CTAs):
 // a grid-wide barrier separates consecutive levels instead of a kernel boundary, which on a
-// chain of single-column levels (natural-order grids) is most of the per-level cost.
-constexpr int kCoopNT = 1024;
-__global__ void __launch_bounds__(kCoopNT, 2) k_update_levels_coop(
+// chain of single-column levels (natural-order grids) is most of the per-level cost.  Each
+// thread resolves the positions of its first pair of the NEXT level before the barrier (index
+// arrays are read-only), so after it only the three value loads and the atomic remain on the
+// chain.
+constexpr int kCoopNT = 1024;  // one CTA per SM: 64 registers, no spills
+__global__ void __launch_bounds__(kCoopNT, 1) k_update_levels_coop(
     int32_t num_levels, const int64_t *__restrict__ lptr, const int64_t *__restrict__ W,
     const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
     const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
@@ -202,12 +255,31 @@ __global__ void __launch_bounds__(kCoopNT, 2) k_update_levels_coop(
     cg::grid_group grid = cg::this_grid();
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    for (int32_t l = 0; l < num_levels; ++l) {
-        const int32_t pos0 = (int32_t)__ldg(lptr + l), pos1 = (int32_t)__ldg(lptr + l + 1);
-        const int64_t wbase = __ldg(W + pos0), total = __ldg(W + pos1) - wbase;
-        if (total <= 0) continue;  // uniform across the grid: no barrier needed
-        for (int64_t t = tid; t < total; t += stride)
-            update_pair(wbase + t, pos0, pos1, W, cols, rp, ci, dpos, cptr, lrow, lpos, val, err);
+    // next non-empty level at or after l: (pos0, pos1, wbase, total); l = num_levels if none
+    auto next_level = [&](int32_t l, int32_t &p0, int32_t &p1, int64_t &wb, int64_t &tot) {
+        for (; l < num_levels; ++l) {
+            p0 = (int32_t)__ldg(lptr + l);
+            p1 = (int32_t)__ldg(lptr + l + 1);
+            wb = __ldg(W + p0);
+            tot = __ldg(W + p1) - wb;
+            if (tot > 0) break;
+        }
+        return l;
+    };
+    int32_t p0 = 0, p1 = 0;
+    int64_t wb = 0, tot = 0;
+    int32_t l = next_level(0, p0, p1, wb, tot);
+    PairPos pre{};
+    if (l < num_levels && tid < tot)
+        pre = pair_pos(wb + tid, p0, p1, W, cols, rp, ci, dpos, cptr, lrow, lpos);
+    while (l < num_levels) {
+        if (tid < tot) pair_apply(pre, val, err);
+        for (int64_t t = tid + stride; t < tot; t += stride)
+            pair_apply(pair_pos(wb + t, p0, p1, W, cols, rp, ci, dpos, cptr, lrow, lpos), val,
+                       err);
+        l = next_level(l + 1, p0, p1, wb, tot);
+        if (l < num_levels && tid < tot)
+            pre = pair_pos(wb + tid, p0, p1, W, cols, rp, ci, dpos, cptr, lrow, lpos);
         grid.sync();
     }
 }
@@ -320,7 +392,7 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
             void *args[] = {&nlv, &lptr_d, &W, &level_cols, &rp, &ci, &dpos, &cptr, &lrow, &lpos,
                             &val, &err};
             NK(cudaLaunchCooperativeKernel((const void *)k_update_levels_coop,
-                                           dim3(num_sms * (occ < 2 ? occ : 2)), dim3(kCoopNT),
+                                           dim3(num_sms * occ), dim3(kCoopNT),
                                            args, 0, s));
         } else {
             for (int32_t l = 0; l < num_levels; ++l) {
