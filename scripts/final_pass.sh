@@ -15,3 +15,4 @@ for c in 3 5 4; do
 done
 CFG=2 bash scripts/profile_round.sh > gpurun_out/profile_round.log 2>&1
 tail -n 3 gpurun_out/smoke.log gpurun_out/pytest_gpu.log
+timeout 400 python scripts/numeric_time.py > gpurun_out/numeric_time.log 2>&1
