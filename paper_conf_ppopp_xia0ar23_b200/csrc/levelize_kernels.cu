@@ -23,6 +23,8 @@
 
 #include <cooperative_groups.h>
 
+#include <climits>
+
 namespace cg = cooperative_groups;
 
 namespace lusym {
@@ -50,8 +52,9 @@ __device__ __forceinline__ int64_t lower_bound_dev(const int32_t *ci, int64_t lo
 }
 
 // One warp per row: strict-U start and (pruned) successor end.
+// psym (GLU3 rule with pruning, else null): psym[i] = p_i, or INT_MAX without a symmetric pair.
 __global__ void k_urange(int32_t n, const int64_t *rp, const int32_t *ci, int prune,
-                         int64_t *ustart, int64_t *uend)
+                         int64_t *ustart, int64_t *uend, int32_t *psym)
 {
     const int lane = threadIdx.x & 31;
     const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -63,6 +66,7 @@ __global__ void k_urange(int32_t n, const int64_t *rp, const int32_t *ci, int pr
         if (lane == 0) us = lower_bound_dev(ci, a, b, i + 1);
         us = __shfl_sync(kFull, us, 0);
         int64_t ue = b;
+        bool sym = false;
         if (prune) {
             for (int64_t c0 = us; c0 < b; c0 += 32) {
                 const int64_t k = c0 + lane;
@@ -76,6 +80,7 @@ __global__ void k_urange(int32_t n, const int64_t *rp, const int32_t *ci, int pr
                 const unsigned bal = __ballot_sync(kFull, hit);
                 if (bal) {
                     ue = c0 + (__ffs(bal) - 1) + 1;
+                    sym = true;
                     break;
                 }
             }
@@ -83,13 +88,16 @@ __global__ void k_urange(int32_t n, const int64_t *rp, const int32_t *ci, int pr
         if (lane == 0) {
             ustart[i] = us;
             uend[i] = ue;
+            if (psym) psym[i] = sym ? ci[ue - 1] : INT_MAX;
         }
     }
 }
 
-// GLU3 reading: count strict-L entries per column (transpose sizes).
+// GLU3 reading: count strict-L entries per column (transpose sizes).  With psym (pruning,
+// reading R32) the entry (r, c) is kept only for r < p_c: a successor r > p_c of c is implied
+// through p_c (the fill rule on (r,c),(c,p_c) gives (r,p_c)), and r = p_c is already c's U edge.
 __global__ void k_lt_count(int32_t n, const int64_t *rp, const int32_t *ci,
-                           const int64_t *ustart, int32_t *cnt)
+                           const int64_t *ustart, const int32_t *psym, int32_t *cnt)
 {
     const int lane = threadIdx.x & 31;
     const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -98,13 +106,13 @@ __global__ void k_lt_count(int32_t n, const int64_t *rp, const int32_t *ci,
         const int64_t a = rp[r], b = ustart[r];
         for (int64_t k = a + lane; k < b; k += 32) {
             const int c = ci[k];
-            if (c < r) atomicAdd(cnt + c, 1);
+            if (c < r && (!psym || r < psym[c])) atomicAdd(cnt + c, 1);
         }
     }
 }
 
 __global__ void k_lt_fill(int32_t n, const int64_t *rp, const int32_t *ci, const int64_t *ustart,
-                          unsigned long long *cursor, int32_t *lt_idx)
+                          const int32_t *psym, unsigned long long *cursor, int32_t *lt_idx)
 {
     const int lane = threadIdx.x & 31;
     const int64_t wg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -113,7 +121,7 @@ __global__ void k_lt_fill(int32_t n, const int64_t *rp, const int32_t *ci, const
         const int64_t a = rp[r], b = ustart[r];
         for (int64_t k = a + lane; k < b; k += 32) {
             const int c = ci[k];
-            if (c < r) lt_idx[atomicAdd(cursor + c, 1ull)] = (int)r;
+            if (c < r && (!psym || r < psym[c])) lt_idx[atomicAdd(cursor + c, 1ull)] = (int)r;
         }
     }
 }
@@ -443,7 +451,9 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
     const int g = aux_grid(n);
     const int gt = (n + 255) / 256;
     // cons_graph: strict-U ranges (pruned for the U rule)
-    k_urange<<<g, kAuxNT, 0, st>>>(n, rp_lu, ci_lu, (prune && !glu3) ? 1 : 0, s.ustart, s.uend);
+    // psym lives in `best` until k_init_queue writes it
+    int32_t *psym = (prune && glu3) ? best : nullptr;
+    k_urange<<<g, kAuxNT, 0, st>>>(n, rp_lu, ci_lu, prune ? 1 : 0, s.ustart, s.uend, psym);
     LV_CK(cudaGetLastError());
     info->launches = 1;
     const int64_t *ltp = nullptr;
@@ -451,7 +461,7 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
     if (glu3) {
         int32_t *cnt = s.indeg;  // reuse as a temporary int32[n]
         LV_CK(cudaMemsetAsync(cnt, 0, sizeof(int32_t) * n, st));
-        k_lt_count<<<g, kAuxNT, 0, st>>>(n, rp_lu, ci_lu, s.ustart, cnt);
+        k_lt_count<<<g, kAuxNT, 0, st>>>(n, rp_lu, ci_lu, s.ustart, psym, cnt);
         LV_CK(cudaGetLastError());
         LV_CK(scan_counts(n, cnt, s.lt_ptr, s.scan_blk, st));
         int64_t nl = 0;
@@ -465,7 +475,7 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
         }
         LV_CK(cudaMemcpyAsync(s.lt_fill, s.lt_ptr, sizeof(int64_t) * n, cudaMemcpyDeviceToDevice,
                               st));
-        k_lt_fill<<<g, kAuxNT, 0, st>>>(n, rp_lu, ci_lu, s.ustart,
+        k_lt_fill<<<g, kAuxNT, 0, st>>>(n, rp_lu, ci_lu, s.ustart, psym,
                                         reinterpret_cast<unsigned long long *>(s.lt_fill),
                                         s.lt_idx);
         LV_CK(cudaGetLastError());

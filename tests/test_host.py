@@ -160,3 +160,30 @@ def test_distributed_assembly_gloo(world):
     spans = [(a, b) for _, _, a, b in res]
     assert spans[0][0] == 0 and spans[-1][1] == 1600
     assert all(spans[k][1] == spans[k + 1][0] for k in range(world - 1))
+
+
+def test_reading_r32_glu3_pruning_preserves_levels():
+    """R32: on a fill-closed pattern P, keeping for column i only its U successors up
+    to the first symmetric pair p_i and its strict-L rows j < p_i leaves every GLU3-rule level
+    unchanged (the device levelization relies on it; the oracle does not prune)."""
+    import oracle
+    from inputs import gen
+    rng = np.random.default_rng(32)
+    for case in range(200):
+        n = int(rng.integers(1, 60))
+        rp, ci = gen.random_pattern(n, float(rng.uniform(0.3, 3.5)), seed=7000 + case,
+                                    zero_free_diag=bool(case % 3), sym_frac=float(rng.uniform(0, 1)))
+        r = oracle.fill2(rp, ci)
+        P = [set(r["col_idx"][r["row_ptr"][i]:r["row_ptr"][i + 1]].tolist()) for i in range(n)]
+        succ = [[] for _ in range(n)]
+        for i in range(n):
+            up = sorted(k for k in P[i] if k > i)
+            p = next((k for k in up if i in P[k]), None)
+            succ[i] += [k for k in up if p is None or k <= p]
+            succ[i] += [j for j in range(i + 1, n) if i in P[j] and (p is None or j < p)]
+        level = [0] * n
+        for i in range(n):            # index order is a topological order (edges go up)
+            for k in succ[i]:
+                level[k] = max(level[k], level[i] + 1)
+        ref, _ = oracle.levels(r["row_ptr"], r["col_idx"], "glu3")
+        assert level == ref.tolist(), f"case {case}"
