@@ -30,6 +30,7 @@
 #include <cooperative_groups.h>
 #include <cub/device/device_scan.cuh>
 
+#include <cstdint>
 #include <cstdlib>
 
 #include <vector>
@@ -40,6 +41,7 @@ namespace {
 namespace cg = cooperative_groups;
 
 constexpr int kErrPivot = 1, kErrPattern = 2;
+constexpr int64_t kTableBudget = 1ll << 30;  // bytes of pair-position table (16 B per pair)
 
 // warp per row i: diagonal position (or -1) and the strict-lower entry count of every column
 __global__ void k_diag_lcount(int32_t n, const int64_t *rp, const int32_t *ci, int64_t *dpos,
@@ -244,13 +246,17 @@ __device__ __forceinline__ void pair_apply(const PairPos &pp, float *val, int *e
 // thread resolves the positions of its first pair of the NEXT level before the barrier (index
 // arrays are read-only), so after it only the three value loads and the atomic remain on the
 // chain.
+// With TAB, the positions of every pair come from a table built beforehand by one parallel
+// pass (k_pair_table, when it fits the budget): one coalesced 16-byte load per pair instead of
+// the dependent index chain.
 constexpr int kCoopNT = 1024;  // one CTA per SM: 64 registers, no spills
+template <bool TAB>
 __global__ void __launch_bounds__(kCoopNT, 1) k_update_levels_coop(
     int32_t num_levels, const int64_t *__restrict__ lptr, const int64_t *__restrict__ W,
     const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
     const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
     const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
-    const int64_t *__restrict__ lpos, float *val, int *err)
+    const int64_t *__restrict__ lpos, const int4 *__restrict__ tab, float *val, int *err)
 {
     cg::grid_group grid = cg::this_grid();
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
@@ -268,19 +274,38 @@ __global__ void __launch_bounds__(kCoopNT, 1) k_update_levels_coop(
     };
     int32_t p0 = 0, p1 = 0;
     int64_t wb = 0, tot = 0;
+    auto get = [&](int64_t g) -> PairPos {
+        if constexpr (TAB) {
+            const int4 v = __ldg(tab + g);
+            return PairPos{v.x, v.y, v.z, v.w};
+        } else {
+            return pair_pos(g, p0, p1, W, cols, rp, ci, dpos, cptr, lrow, lpos);
+        }
+    };
     int32_t l = next_level(0, p0, p1, wb, tot);
     PairPos pre{};
-    if (l < num_levels && tid < tot)
-        pre = pair_pos(wb + tid, p0, p1, W, cols, rp, ci, dpos, cptr, lrow, lpos);
+    if (l < num_levels && tid < tot) pre = get(wb + tid);
     while (l < num_levels) {
         if (tid < tot) pair_apply(pre, val, err);
-        for (int64_t t = tid + stride; t < tot; t += stride)
-            pair_apply(pair_pos(wb + t, p0, p1, W, cols, rp, ci, dpos, cptr, lrow, lpos), val,
-                       err);
+        for (int64_t t = tid + stride; t < tot; t += stride) pair_apply(get(wb + t), val, err);
         l = next_level(l + 1, p0, p1, wb, tot);
-        if (l < num_levels && tid < tot)
-            pre = pair_pos(wb + tid, p0, p1, W, cols, rp, ci, dpos, cptr, lrow, lpos);
+        if (l < num_levels && tid < tot) pre = get(wb + tid);
         grid.sync();
+    }
+}
+
+// The pair-position table: entry g = positions of pair g (global pair ids, W over all of
+// level_cols), int32 fields (callers check nnz(L+U) < 2^31).
+__global__ void k_pair_table(int64_t total, int32_t n, const int64_t *__restrict__ W,
+                             const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
+                             const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
+                             const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
+                             const int64_t *__restrict__ lpos, int4 *tab)
+{
+    for (int64_t g = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; g < total;
+         g += (int64_t)gridDim.x * blockDim.x) {
+        const PairPos pp = pair_pos(g, 0, n, W, cols, rp, ci, dpos, cptr, lrow, lpos);
+        tab[g] = make_int4((int)pp.q, (int)pp.dp, (int)pp.pij, (int)pp.p);
     }
 }
 
@@ -336,8 +361,10 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
     int64_t *dpos = nullptr, *cptr = nullptr, *cursor = nullptr, *lpos = nullptr, *cost = nullptr,
             *W = nullptr;
     int32_t *lcnt = nullptr, *lrow = nullptr;
+    int4 *tab = nullptr;
     int *err = nullptr;
     void *tmp = nullptr;
+    int64_t h_nnz_lu = 0;
     size_t tmp_bytes = 0, tmp2_bytes = 0;
     int64_t nl_total = 0;
     std::vector<int64_t> hW;
@@ -364,6 +391,7 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
     NK(dev_alloc(&tmp, tmp_bytes > tmp2_bytes ? tmp_bytes : tmp2_bytes, s));
     NK(cub::DeviceScan::ExclusiveSum(tmp, tmp_bytes, lcnt, cptr, n + 1, s));
     NK(cudaMemcpyAsync(&nl_total, cptr + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    NK(cudaMemcpyAsync(&h_nnz_lu, rp + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
     NK(cudaStreamSynchronize(s));
     NK(dev_alloc((void **)&lrow, sizeof(int32_t) * (nl_total ? nl_total : 1), s));
     NK(dev_alloc((void **)&lpos, sizeof(int64_t) * (nl_total ? nl_total : 1), s));
@@ -383,17 +411,28 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
         int occ = 0;
         const char *ev = getenv("LUSYM_NUMERIC_LAUNCH_PER_LEVEL");
         const bool per_level = ev && ev[0] == '1';
-        if (!per_level)
-            NK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_update_levels_coop, kCoopNT,
-                                                             0));
+        // pair table when it fits kTableBudget and the int32 fields (LUSYM_NUMERIC_TABLE=0: off)
+        const char *et = getenv("LUSYM_NUMERIC_TABLE");
+        const int64_t pairs = hW[n], nnz_lu = h_nnz_lu;
+        const bool use_tab = !per_level && !(et && et[0] == '0') && pairs > 0 &&
+                             pairs * (int64_t)sizeof(int4) <= kTableBudget &&
+                             nnz_lu < INT32_MAX;
+        const void *kfn = use_tab ? (const void *)k_update_levels_coop<true>
+                                  : (const void *)k_update_levels_coop<false>;
+        if (!per_level) NK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kfn, kCoopNT, 0));
         if (!per_level && occ > 0) {
+            if (use_tab) {
+                NK(dev_alloc((void **)&tab, sizeof(int4) * pairs, s));
+                k_pair_table<<<num_sms * 8, 256, 0, s>>>(pairs, n, W, level_cols, rp, ci, dpos,
+                                                          cptr, lrow, lpos, tab);
+                NK(cudaGetLastError());
+            }
             int32_t nlv = num_levels;
             const int64_t *lptr_d = level_ptr_d;
+            const int4 *tab_c = tab;
             void *args[] = {&nlv, &lptr_d, &W, &level_cols, &rp, &ci, &dpos, &cptr, &lrow, &lpos,
-                            &val, &err};
-            NK(cudaLaunchCooperativeKernel((const void *)k_update_levels_coop,
-                                           dim3(num_sms * occ), dim3(kCoopNT),
-                                           args, 0, s));
+                            &tab_c, &val, &err};
+            NK(cudaLaunchCooperativeKernel(kfn, dim3(num_sms * occ), dim3(kCoopNT), args, 0, s));
         } else {
             for (int32_t l = 0; l < num_levels; ++l) {
                 const int32_t p0 = (int32_t)h_level_ptr[l], p1 = (int32_t)h_level_ptr[l + 1];
@@ -424,6 +463,7 @@ out:
     dev_free(lpos, s);
     dev_free(err, s);
     dev_free(tmp, s);
+    dev_free(tab, s);
     return e;
 }
 

@@ -53,6 +53,8 @@ def run(name, rp, ci, reps=3):
     ms = float(np.median(ts))
     import os
     mode = "per-level" if os.environ.get("LUSYM_NUMERIC_LAUNCH_PER_LEVEL") == "1" else "coop"
+    if mode == "coop" and os.environ.get("LUSYM_NUMERIC_TABLE") == "0":
+        mode = "coop-no-table"
     print(json.dumps({"workload": name, "mode": mode, "n": n, "nnz_lu": int(len(cih)), "levels_glu3": nl,
                       "updates": updates, "levelize_glu3_ms": float(np.median(lv_ms)), "ms": ms, "gflops": 2 * updates / ms / 1e6,
                       "us_per_level": 1e3 * ms / max(nl, 1)}), flush=True)
