@@ -54,6 +54,8 @@ def parse():
     ap.add_argument("--cpu-sample-stride", type=int, default=0,
                     help="oracle sample: every s-th row (0 = auto, ~10-30 s of CPU work)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras)")
+    ap.add_argument("--no-numeric", action="store_true",
+                    help="skip the side measurement of the numeric phase (SURVEY 8(f4))")
     ap.add_argument("--flags", type=int, default=0, help="lu_sym_opts.flags (LU_F_*)")
     ap.add_argument("--threads-per-row", type=int, default=0)
     ap.add_argument("--queue-capacity", type=int, default=0)
@@ -236,6 +238,49 @@ def auto_stride(n, te_total):
 
 
 # --------------------------------------------------------------------------- reference arm
+def numeric_side(reps=5, warmup=2):
+    """Side measurement of the numeric phase (Alg. 2) on cfg1's pattern: not part of
+    `value`.  lu_numeric_factor timed with CUDA events on the current stream (median of reps,
+    after warm-up); the scatter of A's values is outside the events.  Latency-bound: one
+    grid barrier per GLU3 level."""
+    import numpy as np
+    import torch
+    import paper_conf_ppopp_xia0ar23_b200 as lu
+    from inputs import gen
+    d = torch.device("cuda", torch.cuda.current_device())
+    rp, ci = gen.lap2d(64)
+    val = gen.dominant_values(rp, ci, 1, dtype=np.float32)
+    trp, tci, tv = (torch.from_numpy(x).to(d) for x in (rp, ci, val))
+    h = lu.Symbolic(trp, tci)
+    _, rp_lu, ci_lu = h.run()
+    level, nl = lu.levelize(rp_lu, ci_lu, rule="glu3", handle=h)
+    h.close()
+    lptr, lcols = lu.level_schedule(level, nl)
+    rph, cih = rp_lu.cpu().numpy(), ci_lu.cpu().numpy()
+    n = len(rph) - 1
+    row = np.repeat(np.arange(n), np.diff(rph))
+    updates = int((np.bincount(cih[cih < row], minlength=n).astype(np.int64)
+                   * np.bincount(row[cih > row], minlength=n)).sum())
+    s = torch.cuda.current_stream()
+    ts = []
+    for r in range(warmup + reps):
+        v = lu.numeric_scatter(trp, tci, tv, rp_lu, ci_lu)
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        lu.numeric_factor(rp_lu, ci_lu, lptr, lcols, v)
+        e1.record(s)
+        torch.cuda.synchronize()
+        if r >= warmup:
+            ts.append(e0.elapsed_time(e1))
+    ms = float(np.median(ts))
+    return {"workload": "cfg1 lap2d_k64, numeric phase (Alg. 2, float), not in value",
+            "ms": ms, "updates": updates, "gflops": 2 * updates / ms / 1e6,
+            "levels_glu3": nl, "us_per_level": 1e3 * ms / max(nl, 1),
+            "bound": "latency: one grid barrier per GLU3 level (DESIGN.md 6.1)",
+            "parity": "tests/test_gpu_numeric.py vs oracle/numeric.py (float64)"}
+
+
 def run_reference(args, rank, world):
     if rank != 0:
         return
@@ -495,6 +540,7 @@ def run_ours(args, rank, world, local_rank):
         "e2e": e2e,
         "gpu_launches": int(launches),
         "clocks": clk.summary(),
+        "numeric": None if (world > 1 or args.no_numeric) else numeric_side(),
         "plan": {k: stats[k] for k in ("rows_in_flight", "threads_per_row", "smem_bytes_per_row",
                                         "visited_in_smem", "ell_width", "queue_capacity",
                                         "row_classes", "pool_bytes", "rows_retraversed",
