@@ -414,9 +414,10 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
         // pair table when it fits kTableBudget and the int32 fields (LUSYM_NUMERIC_TABLE=0: off)
         const char *et = getenv("LUSYM_NUMERIC_TABLE");
         const int64_t pairs = hW[n], nnz_lu = h_nnz_lu;
+        const char *eb = getenv("LUSYM_NUMERIC_TABLE_GB");  // budget override (A/B)
+        const int64_t budget = eb ? (int64_t)(atof(eb) * (1ll << 30)) : kTableBudget;
         const bool use_tab = !per_level && !(et && et[0] == '0') && pairs > 0 &&
-                             pairs * (int64_t)sizeof(int4) <= kTableBudget &&
-                             nnz_lu < INT32_MAX;
+                             pairs * (int64_t)sizeof(int4) <= budget && nnz_lu < INT32_MAX;
         const void *kfn = use_tab ? (const void *)k_update_levels_coop<true>
                                   : (const void *)k_update_levels_coop<false>;
         if (!per_level) NK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kfn, kCoopNT, 0));
