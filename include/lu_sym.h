@@ -278,7 +278,12 @@ lu_status lu_level_types(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *
  *   (not the arithmetic) may vary from run to run.  The diagonal of every column must be in
  *   the pattern and non-zero when its column is reached: else LU_ERR_INPUT ("zero pivot");
  *   an update outside the pattern (a pattern that is not closed under elimination) is also
- *   LU_ERR_INPUT.  Scratch (O(n + nnz(L))) is allocated per call.  Synchronises.
+ *   LU_ERR_INPUT.  Scratch (O(n + nnz(L)), plus a 16-byte-per-update position table when
+ *   it fits 1 GiB) is allocated per call from the stream-ordered pool.  All levels run in one
+ *   cooperative launch with a grid barrier per level; environment knobs for A/B runs (results
+ *   unchanged): LUSYM_NUMERIC_LAUNCH_PER_LEVEL=1 (one launch per level),
+ *   LUSYM_NUMERIC_TABLE=0 (no position table), LUSYM_NUMERIC_TABLE_GB=<budget>.
+ *   Synchronises.
  */
 lu_status lu_numeric_scatter(int32_t n, const int64_t *d_row_ptr_a, const int32_t *d_col_idx_a,
                              const float *d_val_a, const int64_t *d_row_ptr_lu,
