@@ -250,9 +250,18 @@ __device__ __forceinline__ void pair_apply(const PairPos &pp, float *val, int *e
 // pass (k_pair_table, when it fits the budget): one coalesced 16-byte load per pair instead of
 // the dependent index chain.
 constexpr int kCoopNT = 1024;  // one CTA per SM: 64 registers, no spills
+// Non-empty levels in order, built on the host from the pair offsets: one 32-byte record per
+// level, so finding the next level is one load instead of lptr -> W.
+struct LevelDesc {
+    int32_t p0, p1;
+    int64_t wb, tot;
+    int64_t pad;
+};
+static_assert(sizeof(LevelDesc) == 32, "LevelDesc is two 16-byte loads");
+
 template <bool TAB>
 __global__ void __launch_bounds__(kCoopNT, 1) k_update_levels_coop(
-    int32_t num_levels, const int64_t *__restrict__ lptr, const int64_t *__restrict__ W,
+    int32_t num_levels, const LevelDesc *__restrict__ ld, const int64_t *__restrict__ W,
     const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
     const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
     const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
@@ -261,14 +270,15 @@ __global__ void __launch_bounds__(kCoopNT, 1) k_update_levels_coop(
     cg::grid_group grid = cg::this_grid();
     const int64_t tid = blockIdx.x * (int64_t)blockDim.x + threadIdx.x;
     const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-    // next non-empty level at or after l: (pos0, pos1, wbase, total); l = num_levels if none
+    // level l of the non-empty ones: (pos0, pos1, wbase, total); l = num_levels if none
     auto next_level = [&](int32_t l, int32_t &p0, int32_t &p1, int64_t &wb, int64_t &tot) {
-        for (; l < num_levels; ++l) {
-            p0 = (int32_t)__ldg(lptr + l);
-            p1 = (int32_t)__ldg(lptr + l + 1);
-            wb = __ldg(W + p0);
-            tot = __ldg(W + p1) - wb;
-            if (tot > 0) break;
+        if (l < num_levels) {
+            const int4 a = __ldg(reinterpret_cast<const int4 *>(ld + l));
+            const longlong2 b = __ldg(reinterpret_cast<const longlong2 *>(ld + l) + 1);
+            p0 = a.x;
+            p1 = a.y;
+            wb = (int64_t)(uint32_t)a.z | ((int64_t)a.w << 32);
+            tot = b.x;
         }
         return l;
     };
@@ -362,6 +372,7 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
             *W = nullptr;
     int32_t *lcnt = nullptr, *lrow = nullptr;
     int4 *tab = nullptr;
+    LevelDesc *ldesc = nullptr;
     int *err = nullptr;
     void *tmp = nullptr;
     int64_t h_nnz_lu = 0;
@@ -428,10 +439,20 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
                                                           cptr, lrow, lpos, tab);
                 NK(cudaGetLastError());
             }
-            int32_t nlv = num_levels;
-            const int64_t *lptr_d = level_ptr_d;
+            std::vector<LevelDesc> hd;
+            hd.reserve(num_levels);
+            for (int32_t l = 0; l < num_levels; ++l) {
+                const int32_t a = (int32_t)h_level_ptr[l], b = (int32_t)h_level_ptr[l + 1];
+                if (hW[b] > hW[a]) hd.push_back(LevelDesc{a, b, hW[a], hW[b] - hW[a], 0});
+            }
+            int32_t nlv = (int32_t)hd.size();
+            NK(dev_alloc((void **)&ldesc, sizeof(LevelDesc) * (hd.empty() ? 1 : hd.size()), s));
+            if (!hd.empty())
+                NK(cudaMemcpyAsync(ldesc, hd.data(), sizeof(LevelDesc) * hd.size(),
+                                   cudaMemcpyHostToDevice, s));
+            const LevelDesc *ld_c = ldesc;
             const int4 *tab_c = tab;
-            void *args[] = {&nlv, &lptr_d, &W, &level_cols, &rp, &ci, &dpos, &cptr, &lrow, &lpos,
+            void *args[] = {&nlv, &ld_c, &W, &level_cols, &rp, &ci, &dpos, &cptr, &lrow, &lpos,
                             &tab_c, &val, &err};
             NK(cudaLaunchCooperativeKernel(kfn, dim3(num_sms * occ), dim3(kCoopNT), args, 0, s));
         } else {
@@ -465,6 +486,7 @@ out:
     dev_free(err, s);
     dev_free(tmp, s);
     dev_free(tab, s);
+    dev_free(ldesc, s);
     return e;
 }
 
