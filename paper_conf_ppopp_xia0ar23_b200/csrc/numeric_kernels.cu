@@ -12,16 +12,18 @@
 // counting pass, a CUB scan and an atomic scatter (order inside a column is free: the updates
 // of one column commute).
 //
-// One launch per level (L206-208).  GLU3.0 picks one of three kernel modes per level type
-// (L208: block per column, warp per sub-column, kernel per column); here one kernel covers
-// all three: the level's (sub-column, L entry) pairs are flattened over a grid sized to them,
-// so a narrow level (type C, often a single column on a chain of levels) spreads its pairs
-// over the whole GPU and a wide one (type A) gets one pass.  Each pair locates As(i,k) by
-// (first entry of row i past j, then rank) and subtracts with a float atomic: columns of one
-// level may update the same
-// As(i,k) (a sub-column shared by independent columns).  The GLU3 dependency rule (reading
-// R12, LU_DEP_GLU3) guarantees that nothing a level reads — its own L columns, its U rows —
-// is written within that level.  The update uses the column's undivided entries (reading
+// Levels in order (L206-208), by default all in ONE cooperative launch with a grid barrier
+// between levels (k_update_levels_coop; one launch per level, k_update_level, is the fallback).
+// GLU3.0 picks one of three kernel modes per level type (L208: block per column, warp per
+// sub-column, kernel per column); here one kernel covers all three: the level's (sub-column,
+// L entry) pairs are flattened over the grid, so a narrow level (type C, often a single column
+// on a chain of levels) spreads its pairs over the whole GPU and a wide one (type A) gets one
+// pass.  Each pair locates As(i,k) from As(i,j)'s position (rank of k among row i's entries
+// past j, Alg. 6's binary search over the rest) and subtracts with a float atomic: columns of
+// one level may update the same As(i,k) (a sub-column shared by independent columns).  The
+// GLU3 dependency rule (reading R12, LU_DEP_GLU3) guarantees that nothing a level reads — its
+// own L columns, its U rows — is written within that level.  The update uses the column's
+// undivided entries (reading
 // R31), As(i,k) -= As(i,j) * (As(j,k) / As(j,j)), and lines 2-6 (As(k,j) /= As(j,j)) run once
 // for all columns at the end: a column's strict-L entries are read only by its own update and
 // are final once its level starts, so no barrier separates lines 2-6 from lines 7-14.
