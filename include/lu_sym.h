@@ -39,7 +39,7 @@
 extern "C" {
 #endif
 
-#define LU_SYM_ABI_VERSION 1
+#define LU_SYM_ABI_VERSION 2
 
 typedef enum {
     LU_OK = 0,
@@ -93,8 +93,14 @@ enum {
                                     done maps, frontier spill, L staging, staging pool, row
                                     offsets) comes from cudaMallocManaged and migrates to the
                                     GPU on first touch (page faults)                         */
-    LU_F_MANAGED_PREFETCH = 1 << 13 /* with LU_F_MANAGED: cudaMemAdvise(preferred location =
+    LU_F_MANAGED_PREFETCH = 1 << 13,/* with LU_F_MANAGED: cudaMemAdvise(preferred location =
                                     this GPU) + cudaMemPrefetchAsync after each allocation    */
+    LU_F_NO_DEFER = 1 << 14,     /* no deferred rows: every row is finished by its fill2
+                                    traversal (see lu_sym_opts.defer_windows)                 */
+    LU_F_NO_SPARSE = 1 << 15     /* planner: never replace shared-memory row classes by the
+                                    sparse class (HBM visited slots, 16 rows per SM) that a
+                                    create-time sample of rows selects when they visit < n/16
+                                    vertices on average (reading G9)              */
 };
 
 typedef struct {
@@ -111,7 +117,16 @@ typedef struct {
     uint64_t pool_bytes;           /* HBM staging pool for the rows found by lu_sym_count, so
                                       lu_sym_emit places them instead of re-traversing;
                                       0 => min(32 GiB, what the budget leaves)              */
-    int32_t reserved[6];
+    int32_t defer_windows;         /* deferred rows (reading G8): a row whose fill2
+                                      threshold loop exceeds this many threshold windows is
+                                      abandoned and finished after the pass by the row-merge
+                                      closure over the rows below it, read from the staging
+                                      pool (Theorem 1, split at the largest intermediate
+                                      vertex).  Only rows whose lower rows are all staged by
+                                      this handle qualify.  0 => 4096; < 0 => never          */
+    int32_t defer_max;             /* at most this many deferred rows per call (0 => 1024,
+                                      capped at 4096)                                       */
+    int32_t reserved[4];
 } lu_sym_opts;
 
 typedef struct {
@@ -137,6 +152,14 @@ typedef struct {
     int64_t pool_bytes;           /* staging pool size (0: two-pass mode)                    */
     int64_t rows_retraversed;     /* rows of the last emit that were not staged              */
     int64_t kernel_launches;      /* kernels this handle launched since create (all calls)  */
+    int64_t rows_deferred;        /* last count call: rows handed to the row-merge tail      */
+    int64_t rows_merge_failed;    /* ... of which the tail could not finish (re-traversed)   */
+    int64_t merge_entries_read;   /* ... strict-U entries of staged rows the tail read       */
+    double ms_tail;               /* ... device time of the tail (included in ms_count)     */
+    int64_t merge_rounds;         /* ... frontier rounds of the tail, summed over its rows   */
+    int64_t merge_waits;          /* ... members that were deferred rows still in progress   */
+    double sample_mean_sv;        /* planner: mean vertices scanned per sampled row (reading
+                                     G9); -1 if create did not sample                        */
 } lu_sym_stats;
 
 typedef struct lu_sym lu_sym;

@@ -41,7 +41,7 @@ DEP_U, DEP_GLU3 = 0, 1
 F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4, 8, 16
 F_NO_CONTRACT, F_TWO_PASS, F_ONE_CLASS, F_FORCE_CLASSES = 32, 64, 128, 256
 F_SELF_CONT, F_NO_SELF_CONT, F_PAPER_CHUNKS = 512, 1024, 2048
-F_MANAGED, F_MANAGED_PREFETCH = 4096, 8192
+F_MANAGED, F_MANAGED_PREFETCH, F_NO_DEFER, F_NO_SPARSE = 4096, 8192, 16384, 32768
 
 
 class LuSymError(RuntimeError):
@@ -55,7 +55,8 @@ class _Opts(ctypes.Structure):
                 ("scratch_budget_bytes", ctypes.c_uint64), ("threads_per_row", ctypes.c_int32),
                 ("rows_in_flight", ctypes.c_int32), ("queue_capacity", ctypes.c_int32),
                 ("ell_width", ctypes.c_int32), ("pool_bytes", ctypes.c_uint64),
-                ("reserved", ctypes.c_int32 * 6)]
+                ("defer_windows", ctypes.c_int32), ("defer_max", ctypes.c_int32),
+                ("reserved", ctypes.c_int32 * 4)]
 
 
 class _Stats(ctypes.Structure):
@@ -74,10 +75,14 @@ class _Stats(ctypes.Structure):
                 ("levelize_rank_rounds", ctypes.c_int32), ("row_classes", ctypes.c_int32),
                 ("reserved", ctypes.c_int32 * 1),
                 ("pool_bytes", ctypes.c_int64), ("rows_retraversed", ctypes.c_int64),
-                ("kernel_launches", ctypes.c_int64)]
+                ("kernel_launches", ctypes.c_int64), ("rows_deferred", ctypes.c_int64),
+                ("rows_merge_failed", ctypes.c_int64), ("merge_entries_read", ctypes.c_int64),
+                ("ms_tail", ctypes.c_double), ("merge_rounds", ctypes.c_int64),
+                ("merge_waits", ctypes.c_int64), ("sample_mean_sv", ctypes.c_double)]
 
 
 _lib = None
+ABI_VERSION = 2
 
 EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sym_count",
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
@@ -127,7 +132,7 @@ def load_library():
     for f in ("lu_sym_create", "lu_sym_count", "lu_sym_scan", "lu_sym_emit", "lu_sym_run",
               "lu_levelize", "lu_sym_get_stats", "lu_sym_run_host"):
         getattr(lib, f).restype = I32
-    if lib.lu_sym_abi_version() != 1:
+    if lib.lu_sym_abi_version() != ABI_VERSION:
         raise ImportError("liblusym.so ABI version mismatch")
     _lib = lib
     return lib
@@ -164,6 +169,8 @@ class Options:
     queue_capacity: int = 0
     ell_width: int = 0
     pool_bytes: int = 0
+    defer_windows: int = 0
+    defer_max: int = 0
 
     def to_c(self) -> _Opts:
         o = _Opts()
@@ -175,6 +182,8 @@ class Options:
         o.queue_capacity = self.queue_capacity
         o.ell_width = self.ell_width
         o.pool_bytes = self.pool_bytes
+        o.defer_windows = self.defer_windows
+        o.defer_max = self.defer_max
         return o
 
 

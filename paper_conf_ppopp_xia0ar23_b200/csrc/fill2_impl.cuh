@@ -55,7 +55,7 @@ constexpr int kSmallWin = 32;  // threshold window after a window was cut short
 struct Hdr {
     int row, minseed, diag, tns, newmin, ucnt, lmin, lmax;
     int cnt[3];
-    int pad;
+    int defer;
     long long stage_off;
     unsigned long long te, sv, spills;  // statistics of this CTA (thread 0 / shared atomics)
     int scan[40];
@@ -762,7 +762,9 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
             const unsigned long long c = atomicAdd(p.row_counter, 1ull);
             int r = -1;
             if (p.row_list) {
-                if (c < (unsigned long long)p.list_len) r = p.row_list[c];
+                const unsigned long long len =
+                    p.list_len_dev ? *p.list_len_dev : (unsigned long long)p.list_len;
+                if (c < len) r = p.row_list[c];
             } else if (c < (unsigned long long)nrows) {
                 r = p.descending ? p.row_end - 1 - (int)c : p.row_begin + (int)c;
             }
@@ -833,6 +835,7 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
         // shrinks to kSmallWin after it was cut short and doubles back while it is consumed
         uint32_t *dm = p.dbitmap + (size_t)blockIdx.x * p.gbitmap_stride;
         bool dused = false;
+        bool deferred = false;  // block-uniform
         int cap = p.wcap;
         // ---- thresholds in increasing order (L130)
         for (;;) {
@@ -848,6 +851,30 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
             PH_MARK(ph_col);
             if (wc == 0) break;
             ++n_win;
+            if constexpr (MODE != kEmit) {
+                // reading G8: a row whose threshold chain is this long is abandoned here and
+                // finished after the pass by the row-merge tail (block-uniform decision); in
+                // kCount mode without a list (the planner's sample) it is just abandoned
+                if (n_win == p.defer_win + 1 && p.defer_win > 0 && i >= p.defer_from) {
+                    if (tid == 0) {
+                        bool ok = true;
+                        if (p.defer_list) {
+                            const unsigned long long slot = atomicAdd(p.defer_cnt, 1ull);
+                            ok = slot < (unsigned long long)p.defer_max;
+                            if (ok) {
+                                p.defer_list[slot] = i;
+                                p.row_off[i] = kRowDeferred;
+                            }
+                        }
+                        h.defer = ok;
+                    }
+                    __syncthreads();
+                    if (h.defer) {
+                        deferred = true;
+                        break;
+                    }
+                }
+            }
             if (tid == 0) h.sv += wc;
             int nm = INT_MAX;
             for (int base = 0; base < wc; base += NT) {
@@ -952,7 +979,9 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
             ptr = nptr;
         }
         // thresholds finished ahead of the pointer and never re-collected: the rest of (ptr, i)
-        Lcnt += emit_range<NT, VIS, MODE != kCount>(bm, sm, ptr + 1, i, ldst, Lcnt, lcap, h.scan);
+        if (!deferred)
+            Lcnt += emit_range<NT, VIS, MODE != kCount>(bm, sm, ptr + 1, i, ldst, Lcnt, lcap,
+                                                       h.scan);
         if (dused)  // leave the done map zero for the next row
             for (int w = (h.minseed >> 5) + tid; w <= ((i - 1) >> 5); w += NT) dm[w] = 0;
 
@@ -964,11 +993,13 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
         const int ucnt = h.ucnt, diag = h.diag, gmin = h.lmin, gmax = h.lmax;
         const int len = Lcnt + diag + ucnt;
         if constexpr (MODE == kCount) {
-            if (tid == 0) p.fill_count[i] = len;
+            if (tid == 0 && !deferred) p.fill_count[i] = len;
         } else if constexpr (MODE == kStage) {
+          if (!deferred) {
             // reserve len entries of the pool; rows that do not fit are re-traversed by emit
             if (tid == 0) {
                 p.fill_count[i] = len;
+                p.ucut[i] = Lcnt + diag;
                 const unsigned long long off = atomicAdd(p.pool_cursor, (unsigned long long)len);
                 const bool fits = off + (unsigned long long)len <= (unsigned long long)p.pool_cap;
                 h.stage_off = fits ? (long long)off : -1ll;
@@ -984,6 +1015,7 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                 emit_range<NT, VIS, true>(bm, sm, i + 1, gmax + 1, dst + Lcnt + diag, 0, INT64_MAX,
                                          h.scan);
             }
+          }
         } else {
             if (lcap != (int64_t)len) {
                 if (tid == 0) atomicAdd(p.stats + kStatErr, 1ull);

@@ -17,6 +17,7 @@ size_t fill2_smem_bytes(int n, int smem_words, int q)
 
 #define LUSYM_NT_SWITCH(FN, ...)                                                             \
     switch (nt) {                                                                            \
+    case 64: return FN<64>(__VA_ARGS__);                                                     \
     case 128: return FN<128>(__VA_ARGS__);                                                   \
     case 256: return FN<256>(__VA_ARGS__);                                                   \
     case 512: return FN<512>(__VA_ARGS__);                                                   \

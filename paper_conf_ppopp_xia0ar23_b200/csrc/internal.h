@@ -52,8 +52,55 @@ struct Fill2Params {
     int64_t *row_prof;
     // self-continuation rounds per BFS level (scan_level); 0 = plain level-synchronous BFS
     int32_t kloc;
+    // row_list length read on the device (a list built by an earlier kernel), when non-null
+    const unsigned long long *list_len_dev = nullptr;
+    // kStage: entries <= i of each staged row (L part + diagonal), for the row-merge tail
+    int32_t *ucut = nullptr;
+    // deferral (kStage, reading G8): a row i >= defer_from whose threshold loop reaches
+    // defer_win + 1 windows is abandoned and listed (at most defer_max rows) for the
+    // row-merge tail; defer_win = 0 disables it
+    int32_t defer_win = 0, defer_from = 0, defer_max = 0;
+    int32_t *defer_list = nullptr;
+    unsigned long long *defer_cnt = nullptr;
 };
 enum Fill2Mode { kCount = 0, kEmit = 1, kStage = 2 };
+// row_off value of a row deferred to the row-merge tail and not finished yet
+constexpr int64_t kRowDeferred = -2;
+
+// merge_kernels.cu — deferred rows by row-merge closure over staged rows (reading G8)
+struct MergeParams {
+    int32_t n;
+    const int64_t *rp;                 // A
+    const int32_t *ci;
+    int32_t *pool;                     // staging pool (read: rows t < i; written: row i)
+    int64_t pool_cap;
+    unsigned long long *pool_cursor;
+    int64_t *row_off;                  // [n] pool offset, -1 unstaged, kRowDeferred pending
+    int32_t *ucut;                     // [n] entries <= t of staged row t
+    int32_t *fill_count;               // [n]
+    const int32_t *list;               // deferred rows, ascending, list_cnt[0] (<= list_max)
+    const unsigned long long *list_cnt;
+    int32_t list_max;
+    unsigned long long *counter;       // row claims
+    uint32_t *gbitmap;                 // per-CTA visited slot (when not in shared memory)
+    int64_t gb_stride;
+    int32_t *spill;                    // per CTA: 2 x spill_cap frontier entries
+    int64_t spill_cap;
+    int32_t *wait;                     // per CTA: list_max deferred rows waited on
+    int32_t *fail_list;                // rows the tail could not finish (-> fill2 fallback)
+    unsigned long long *fail_cnt;
+    unsigned long long *stats;         // [0] U entries read, [1] rounds, [2] waits
+    int32_t q;                         // shared frontier capacity per buffer
+};
+size_t merge_smem_bytes(int n, bool smem_bitmap, int q);
+cudaError_t merge_configure(size_t smem);
+// sort list[0..min(*cnt, max)) ascending (one CTA; max <= 4096)
+cudaError_t merge_sort_list(int32_t *list, const unsigned long long *cnt, int32_t max,
+                            cudaStream_t s);
+cudaError_t merge_launch(const MergeParams &p, bool smem_bitmap, int grid, size_t smem,
+                         cudaStream_t s);
+constexpr int kMergeNT = 1024;
+constexpr int kMergeSortMax = 4096;
 
 // Visited storage of a row in flight (frontiers are lists in shared memory, spilling to HBM).
 //   kVisSmem   : visited bitmap in shared memory

@@ -62,9 +62,10 @@ lu_status fail(lu_status s, const char *fmt, ...)
                         "%s: %s (%s:%d)", #x, cudaGetErrorString(e_), __FILE__, __LINE__);   \
     } while (0)
 
-enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvN = 4 };
+enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvTail = 4, kEvN = 5 };
 enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11, kSlotClassCounter = 16,
-       kSlotSetStride = 32, kStatSlots = 128, kMaxChunks = 64, kSets = 3 };
+       kSlotSetStride = 32, kSlotDefer = 112 /* [0] deferred rows, [1] tail claims,
+       [2] failed rows, [3..5] tail statistics */, kStatSlots = 128, kMaxChunks = 64, kSets = 3 };
 
 }  // namespace
 
@@ -142,6 +143,20 @@ struct lu_sym {
     int64_t *pin = nullptr;                       // pinned host slot (chunk end offset)
     std::vector<int32_t> chunk_bounds;            // lu_sym_run_host row chunks (cached)
     bool heavy_last = false;                      // ... and whether the last chunk goes first
+    // deferred rows (reading G8): fill2 abandons a row after defer_win threshold windows; the
+    // row-merge tail (merge_kernels.cu) finishes it from the staged rows below it
+    int32_t *ucut = nullptr;       // [n] entries <= i of each staged row
+    int defer_win = 512, defer_max = 1024;
+    bool defer_active = false;     // the pass being launched may defer rows >= defer_from
+    int32_t defer_from = 0;
+    int32_t *defer_list = nullptr, *fail_list = nullptr;  // [defer_max] each
+    int32_t *mspill = nullptr, *mwait = nullptr;
+    uint32_t *mgbitmap = nullptr;
+    int merge_grid = 0, merge_q = 2048;
+    bool merge_smem_bm = true;
+    size_t merge_smem = 0;
+    bool tail_ran = false;
+    double sparse_sv = -1;         // planner sample: mean SV per row (-1: not sampled)
 };
 
 namespace {
@@ -206,8 +221,10 @@ lu_status salloc(lu_sym *h, T **p, size_t elems)
 void free_handle(lu_sym *h)
 {
     cudaStream_t s = h->stream;
-    void *bufs[] = {h->ell,      h->gbitmap,  h->dbitmap, h->gspill, h->dstats,  h->scan_blk,
-                    h->dbad,     h->stg,      h->pool,    h->row_off, h->unstaged};
+    void *bufs[] = {h->ell,        h->gbitmap,   h->dbitmap, h->gspill, h->dstats,
+                    h->scan_blk,   h->dbad,      h->stg,     h->pool,   h->row_off,
+                    h->unstaged,   h->ucut,      h->defer_list, h->fail_list, h->mspill,
+                    h->mwait,      h->mgbitmap};
     if (!h->managed.empty()) cudaStreamSynchronize(s);
     std::vector<void *> all(std::begin(bufs), std::end(bufs));
     for (int k = 1; k < kSets; ++k)
@@ -266,19 +283,23 @@ struct Cfg {
     long key;
 };
 
-lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out)
+lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out, int want_nt = 0,
+                   int min_q = 512)
 {
     // kernel keys: CTA sizes 128..1024, and 1025 = 1024 threads with the one-CTA-per-SM
     // register budget (chosen on a tie, i.e. when shared memory allows one CTA per SM anyway)
-    const int nts[5] = {128, 256, 512, 1024, 1025};
-    const int qs[4] = {512, 1024, 2048, 4096};
+    // (64: only on request — a sparse class or threads_per_row = 64)
+    const int nts[6] = {64, 128, 256, 512, 1024, 1025};
+    const int qs[5] = {256, 512, 1024, 2048, 4096};
     Cfg best = {0, 0, 0, 0, -1};
-    for (int a = 0; a < 5; ++a) {
+    for (int a = 0; a < 6; ++a) {
         const int nt = nts[a];
-        const int tpr = h->opts.threads_per_row;
+        const int tpr = want_nt > 0 ? want_nt : h->opts.threads_per_row;
         if (tpr > 0 && nt != tpr && !(tpr == 1024 && nt == 1025)) continue;
+        if (tpr <= 0 && nt == 64) continue;
         const int threads = nt > 1024 ? 1024 : nt;
-        for (int b = 0; b < 4; ++b) {
+        for (int b = 0; b < 5; ++b) {
+            if (qs[b] < min_q && h->opts.queue_capacity <= 0) continue;
             int q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : qs[b];
             if (h->opts.queue_capacity > 0 && b > 0) break;
             if (q < 32) q = 32;
@@ -299,6 +320,85 @@ lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out)
     return LU_OK;
 }
 
+// Mean vertices scanned per row (SV, reading R24) over `cnt` rows evenly spread over [lo, hi),
+// measured by running the count kernel on them with the configuration c (its own temporary
+// scratch).  A row whose threshold chain exceeds 64 windows is abandoned where it stands
+// (the circuit hubs would otherwise dominate the sample's time); its SV so far still counts.
+lu_status sample_mean_sv(lu_sym *h, const RowClass &c, int32_t lo, int32_t hi, int cnt,
+                         int sms, double *mean_sv)
+{
+    const int32_t n = h->n;
+    cnt = std::max(1, std::min(cnt, hi - lo));
+    std::vector<int32_t> rows((size_t)cnt);
+    for (int k = 0; k < cnt; ++k)
+        rows[(size_t)k] = lo + (int32_t)(((double)k + 0.5) * (hi - lo) / cnt);
+    const int grid = std::min(cnt, sms * c.occ);
+    const int64_t words = ((int64_t)n + 31) / 32 + 31;
+    int32_t *d_rows = nullptr, *fc = nullptr, *spill = nullptr;
+    uint32_t *dmap = nullptr, *gmap = nullptr;
+    const size_t need = (size_t)cnt * 4 + (size_t)n * 4 + (size_t)grid * 2 * (size_t)n * 4 +
+                        (size_t)grid * (size_t)words * 4 * (c.vis == kVisSmem ? 1 : 2);
+    if (need > h->budget / 4) {  // never worth a large share of the budget
+        *mean_sv = -1;
+        return LU_OK;
+    }
+    cudaStream_t s = h->stream;
+    CK(dev_alloc((void **)&d_rows, (size_t)cnt * 4, s));
+    CK(dev_alloc((void **)&fc, (size_t)n * 4, s));
+    CK(dev_alloc((void **)&spill, (size_t)grid * 2 * (size_t)n * 4, s));
+    CK(dev_alloc((void **)&dmap, (size_t)grid * (size_t)words * 4, s));
+    if (c.vis != kVisSmem) CK(dev_alloc((void **)&gmap, (size_t)grid * (size_t)words * 4, s));
+    CK(cudaMemcpyAsync(d_rows, rows.data(), (size_t)cnt * 4, cudaMemcpyHostToDevice, s));
+    unsigned long long *slots = h->dstats + kSlotDefer + 8;  // [0..3] stats, [4] row counter
+    CK(cudaMemsetAsync(slots, 0, 5 * sizeof(unsigned long long), s));
+    CK(cudaMemsetAsync(dmap, 0, (size_t)grid * (size_t)words * 4, s));
+    if (gmap) CK(cudaMemsetAsync(gmap, 0, (size_t)grid * (size_t)words * 4, s));
+    Fill2Params p;
+    p.n = n;
+    p.rp = h->rp;
+    p.ci = h->ci;
+    p.ell = h->ell;
+    p.descending = 1;
+    p.fill_count = fc;
+    p.rp_lu = nullptr;
+    p.ci_lu = nullptr;
+    p.gbitmap = gmap;
+    p.dbitmap = dmap;
+    p.gbitmap_stride = words;
+    p.gspill = spill;
+    p.spill_cap = n;
+    p.nw = c.smem_words;
+    p.lbw = c.lbw;
+    p.sw = (int32_t)((((int64_t)n + 31) / 32 + 31) / 32);
+    p.q = c.q;
+    p.wcap = c.q;
+    p.row_counter = slots + 4;
+    p.stats = slots;
+    p.row_list = d_rows;
+    p.list_len = cnt;
+    p.row_begin = p.row_end = 0;
+    p.stg = nullptr;
+    p.pool = nullptr;
+    p.pool_cap = 0;
+    p.row_off = nullptr;
+    p.pool_cursor = nullptr;
+    p.unstaged = nullptr;
+    p.unstaged_cnt = nullptr;
+    p.row_prof = nullptr;
+    p.kloc = c.occ <= LUSYM_KLOC_OCC ? LUSYM_KLOC : 0;
+    p.defer_win = 64;
+    p.defer_from = 0;
+    CK(fill2_launch(p, c.nt, h->w, kCount, c.vis, grid, c.smem, s));
+    h->launches += 1;
+    unsigned long long st[kStatCount] = {};
+    CK(cudaMemcpyAsync(st, slots, sizeof(st), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    for (void *b : {(void *)d_rows, (void *)fc, (void *)spill, (void *)dmap, (void *)gmap})
+        dev_free(b, s);
+    *mean_sv = (double)st[kStatVerts] / cnt;
+    return LU_OK;
+}
+
 lu_status plan(lu_sym *h)
 {
     int sms = 0, smem_optin = 0;
@@ -309,8 +409,9 @@ lu_status plan(lu_sym *h)
     const int nw32 = (nw + 31) / 32 * 32;  // whole swizzle groups
     if (h->opts.threads_per_row > 0 && h->opts.threads_per_row != 128 &&
         h->opts.threads_per_row != 256 && h->opts.threads_per_row != 512 &&
-        h->opts.threads_per_row != 1024 && h->opts.threads_per_row != 1025)
-        return fail(LU_ERR_ARG, "threads_per_row must be 128, 256, 512, 1024 or 1025 (got %d)",
+        h->opts.threads_per_row != 1024 && h->opts.threads_per_row != 1025 &&
+        h->opts.threads_per_row != 64)
+        return fail(LU_ERR_ARG, "threads_per_row must be 64, 128, 256, 512, 1024 or 1025 (got %d)",
                     h->opts.threads_per_row);
     // top class: the whole visited map in shared memory, else in HBM
     Cfg cur;
@@ -372,8 +473,6 @@ lu_status plan(lu_sym *h)
         h->classes.push_back(RowClass{0, hi, vis, sw_words, vis == kVisGlobal ? 0 : sw_words,
                                       cur.nt, cur.q, cur.occ, cur.smem});
     }
-    // HBM budget: per row in flight, frontier spill (2 x cap) + L staging (cap) + done map
-    // (+ the HBM visited slot); cap = rows of the class (a row's frontier and L part lie below i)
     size_t free_b = 0, total_b = 0;
     CK(cudaMemGetInfo(&free_b, &total_b));
     const uint64_t budget = h->opts.scratch_budget_bytes ? h->opts.scratch_budget_bytes
@@ -381,6 +480,38 @@ lu_status plan(lu_sym *h)
     h->budget = budget;
     h->staging = !(h->opts.flags & LU_F_TWO_PASS);
     h->gb_stride = nw32;
+    // Sparse rows (reading G9): where a class holds few rows per SM because its shared visited
+    // map is large, but the rows visit only a small part of it (a sample's mean SV < n/16 —
+    // ND-ordered circuits scan ~3K of 10^6 vertices per row, natural-order grids ~i), the
+    // whole range is better served by HBM visited slots (L2-resident) and 64-thread CTAs at
+    // 32 rows per SM: latency is hidden by rows in flight instead of threads per row (cfg3:
+    // 1/2/4/8 rows per SM in four shared-map classes 630 ms, 16 rows of 128 threads 195 ms,
+    // 32 rows of 64 threads 159 ms, scripts/exp_plan.py).
+    h->sparse_sv = -1;
+    if (!(h->opts.flags & (LU_F_ONE_CLASS | LU_F_GLOBAL_BITMAP | LU_F_FORCE_CLASSES |
+                           LU_F_NO_SPARSE)) &&
+        h->opts.threads_per_row == 0 && h->opts.queue_capacity == 0) {
+        Cfg g;
+        if ((st = best_cfg(h, 0, kVisGlobal, smem_optin, &g, 64, 256)) != LU_OK) return st;
+        size_t kc = 0;
+        while (g.key >= 0 && kc < h->classes.size() && h->classes[kc].occ < g.occ) ++kc;
+        const bool force = getenv("LUSYM_FORCE_SPARSE") != nullptr;  // test knob
+        if (force && g.key >= 0) kc = h->classes.size();
+        if (kc > 0) {
+            double sv = -1;
+            const int32_t lo = h->classes[kc - 1].lo;
+            if ((st = sample_mean_sv(h, h->classes[0], lo, n, 256, sms, &sv)) != LU_OK) return st;
+            if (force) sv = 0;
+            h->sparse_sv = sv;
+            if (sv >= 0 && sv < (double)n / 16) {
+                h->classes.erase(h->classes.begin(), h->classes.begin() + (long)kc);
+                h->classes.insert(h->classes.begin(),
+                                  RowClass{lo, n, kVisGlobal, 0, 0, g.nt, g.q, g.occ, g.smem});
+            }
+        }
+    }
+    // HBM budget: per row in flight, frontier spill (2 x cap) + L staging (cap) + done map
+    // (+ the HBM visited slot); cap = rows of the class (a row's frontier and L part lie below i)
     const bool need_hbm_map = h->classes.front().vis != kVisSmem || h->classes.size() > 1;
     uint64_t need_spill = 0, need_stg = 0, need_map = 0;
     int max_grid = 0;
@@ -419,6 +550,15 @@ lu_status plan(lu_sym *h)
     if (h->staging) {
         if ((st = salloc(h, &h->stg, need_stg)) != LU_OK) return st;
         if ((st = salloc(h, &h->row_off, (size_t)n)) != LU_OK) return st;
+        if ((st = salloc(h, &h->ucut, (size_t)n)) != LU_OK) return st;
+    }
+    // deferred rows (reading G8)
+    {
+        const int dw = h->opts.defer_windows, dm = h->opts.defer_max;
+        h->defer_win = (h->opts.flags & LU_F_NO_DEFER) || dw < 0 ? 0 : (dw > 0 ? dw : 4096);
+        h->defer_max = dm > 0 ? std::min(dm, (int)kMergeSortMax) : 1024;
+        if (const char *e = getenv("LUSYM_DEFER_WINDOWS")) h->defer_win = atoi(e);
+        if (!h->staging) h->defer_win = 0;
     }
     if (getenv("LUSYM_DEBUG_PLAN")) {
         for (auto &c : h->classes)
@@ -459,7 +599,7 @@ void ev_end(lu_sym *h, int k, cudaStream_t s)
 lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_count,
                    const int64_t *rp_lu, int32_t *ci_lu, cudaStream_t s,
                    const int32_t *row_list = nullptr, int32_t list_len = 0, int set = 0,
-                   bool reset_stats = true)
+                   bool reset_stats = true, const unsigned long long *list_len_dev = nullptr)
 {
     const bool emit = mode == kEmit;
     unsigned long long *st = h->dstats + (emit ? 5 : 1);
@@ -494,6 +634,15 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     p.unstaged = h->unstaged;
     p.unstaged_cnt = h->dstats + kSlotUnstaged;
     p.row_prof = h->row_prof;
+    p.ucut = h->ucut;
+    p.list_len_dev = list_len_dev;
+    if (mode == kStage && h->defer_active && !row_list) {
+        p.defer_win = h->defer_win;
+        p.defer_from = h->defer_from;
+        p.defer_max = h->defer_max;
+        p.defer_list = h->defer_list;
+        p.defer_cnt = h->dstats + kSlotDefer;
+    }
     // classes run concurrently: the top class on s, the others on their own streams forked
     // from s, so lower-class CTAs take over SMs as soon as top-class CTAs drain
     bool forked = false;
@@ -502,7 +651,7 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
         // a row list (rows that did not fit the staging pool) runs in the top class only
         if (row_list && k > 0) break;
         const int32_t lo = row_list ? 0 : std::max(rb, c.lo), hi = row_list ? 0 : std::min(re, c.hi);
-        const int rows = row_list ? list_len : hi - lo;
+        const int rows = row_list ? (list_len_dev ? c.grid : list_len) : hi - lo;
         if (rows <= 0) continue;
         cudaStream_t cs = s;
         if (k > 0) {
@@ -630,6 +779,103 @@ lu_status ensure_pool(lu_sym *h)
     h->pool_cap = cap;
     h->scratch_bytes += cap * (int64_t)sizeof(int32_t);
     return LU_OK;
+}
+
+// Scratch of the row-merge tail (reading G8), allocated on the first count that may defer
+// rows: the deferred / failed row lists and, per tail CTA, a frontier spill (2 x n entries), a
+// wait list (defer_max) and, when n/8 bytes do not fit shared memory, an HBM visited slot.
+// One 1024-thread CTA per SM, fewer if the scratch budget is short (none: deferral is off).
+lu_status ensure_merge(lu_sym *h)
+{
+    if (h->defer_list || h->defer_win <= 0) return LU_OK;
+    int sms = 0, smem_optin = 0;
+    CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device));
+    CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->device));
+    const int n = h->n;
+    h->merge_smem_bm = merge_smem_bytes(n, true, h->merge_q) <= (size_t)smem_optin &&
+                       !getenv("LUSYM_MERGE_HBM_BITMAP");  // test knob: the HBM-slot variant
+    h->merge_smem = merge_smem_bytes(n, h->merge_smem_bm, h->merge_q);
+    if (h->merge_smem > (size_t)smem_optin) {
+        h->defer_win = 0;
+        return LU_OK;
+    }
+    const int64_t words = ((int64_t)n + 31) / 32;
+    const uint64_t per_cta = (uint64_t)(2 * (int64_t)n + h->defer_max) * 4 +
+                             (h->merge_smem_bm ? 0 : (uint64_t)words * 4);
+    const uint64_t lists = (uint64_t)2 * h->defer_max * 4;
+    const uint64_t left = h->budget > (uint64_t)h->scratch_bytes + lists
+                              ? h->budget - (uint64_t)h->scratch_bytes - lists : 0;
+    int64_t grid = std::min<int64_t>(sms, h->defer_max);
+    grid = std::min<int64_t>(grid, (int64_t)(left / per_cta));
+    if (grid < 1) {
+        h->defer_win = 0;
+        return LU_OK;
+    }
+    CK(merge_configure(h->merge_smem));
+    h->merge_grid = (int)grid;
+    lu_status st;
+    if ((st = salloc(h, &h->defer_list, (size_t)h->defer_max)) != LU_OK) return st;
+    if ((st = salloc(h, &h->fail_list, (size_t)h->defer_max)) != LU_OK) return st;
+    if ((st = salloc(h, &h->mspill, (size_t)grid * 2 * (size_t)n)) != LU_OK) return st;
+    if ((st = salloc(h, &h->mwait, (size_t)grid * (size_t)h->defer_max)) != LU_OK) return st;
+    if (!h->merge_smem_bm) {
+        if ((st = salloc(h, &h->mgbitmap, (size_t)grid * (size_t)words)) != LU_OK) return st;
+        CK(cudaMemsetAsync(h->mgbitmap, 0, (size_t)grid * (size_t)words * 4, h->stream));
+    }
+    return LU_OK;
+}
+
+// [0, row_end) covered by the staged ranges (every row a deferred row may need is staged)
+bool staged_below(const lu_sym *h, int32_t row_end)
+{
+    std::vector<std::pair<int32_t, int32_t>> r = h->staged;
+    std::sort(r.begin(), r.end());
+    int32_t reach = 0;
+    for (auto &x : r) {
+        if (x.first > reach) break;
+        reach = std::max(reach, x.second);
+    }
+    return reach >= row_end;
+}
+
+// The row-merge tail after a pass that deferred rows: sort the deferred list, finish the rows
+// by closure over the staged rows (k_merge_rows), then let fill2 finish (stage) whatever the
+// tail could not — its list length is read on the device, so no host round trip.
+lu_status run_tail(lu_sym *h, int32_t *fill_count, cudaStream_t s)
+{
+    ev_begin(h, kEvTail, s);
+    unsigned long long *slots = h->dstats + kSlotDefer;
+    CK(merge_sort_list(h->defer_list, slots, h->defer_max, s));
+    MergeParams mp;
+    mp.n = h->n;
+    mp.rp = h->rp;
+    mp.ci = h->ci;
+    mp.pool = h->pool;
+    mp.pool_cap = h->pool_cap;
+    mp.pool_cursor = h->dstats + kSlotPoolCursor;
+    mp.row_off = h->row_off;
+    mp.ucut = h->ucut;
+    mp.fill_count = fill_count;
+    mp.list = h->defer_list;
+    mp.list_cnt = slots;
+    mp.list_max = h->defer_max;
+    mp.counter = slots + 1;
+    mp.gbitmap = h->mgbitmap;
+    mp.gb_stride = ((int64_t)h->n + 31) / 32;
+    mp.spill = h->mspill;
+    mp.spill_cap = h->n;
+    mp.wait = h->mwait;
+    mp.fail_list = h->fail_list;
+    mp.fail_cnt = slots + 2;
+    mp.stats = slots + 3;
+    mp.q = h->merge_q;
+    CK(merge_launch(mp, h->merge_smem_bm, h->merge_grid, h->merge_smem, s));
+    h->launches += 2;
+    lu_status st = run_pass(h, kStage, 0, h->n, fill_count, nullptr, nullptr, s, h->fail_list, 0,
+                            0, false, slots + 2);
+    ev_end(h, kEvTail, s);
+    h->tail_ran = true;
+    return st;
 }
 
 }  // namespace
@@ -768,7 +1014,10 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
     h->stream = s;
     ev_begin(h, kEvCount, s);
     int mode = kCount;
+    bool defer = false;
+    h->tail_ran = false;
     if (h->staging) {
+        if ((st = ensure_merge(h)) != LU_OK) return st;
         st = ensure_pool(h);
         if (st != LU_OK) return st;
         if (h->pool) {
@@ -783,9 +1032,16 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
                                    s));
             }
             h->staged.emplace_back(row_begin, row_end);
+            // deferred rows need every row below them staged (reading G8)
+            defer = h->defer_win > 0 && h->defer_list && staged_below(h, row_end);
         }
     }
+    if (defer) CK(cudaMemsetAsync(h->dstats + kSlotDefer, 0, 6 * sizeof(unsigned long long), s));
+    h->defer_active = defer;
+    h->defer_from = row_begin;
     st = run_pass(h, mode, row_begin, row_end, d_fill_count, nullptr, nullptr, s);
+    h->defer_active = false;
+    if (st == LU_OK && defer) st = run_tail(h, d_fill_count, s);
     ev_end(h, kEvCount, s);
     return st;
 }
@@ -910,6 +1166,7 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
         nchunks = std::max(1, std::min(16, n / 4096));
     if (nchunks > n) nchunks = n > 0 ? n : 1;
     if (h->staging) {
+        if ((st = ensure_merge(h)) != LU_OK) return st;
         if ((st = ensure_pool(h)) != LU_OK) return st;
     }
     if (!h->staging || !h->pool || n == 0 || nchunks == 1) {
@@ -977,6 +1234,11 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
     CK(cudaMemsetAsync(h->dstats + kSlotPoolCursor, 0, 2 * sizeof(unsigned long long), s));
     CK(cudaMemsetAsync(h->dstats + 1, 0, sizeof(unsigned long long) * kStatCount, s));
     CK(cudaMemsetAsync(d_row_ptr_lu, 0, sizeof(int64_t), s));
+    // rows of the last chunk may be deferred to the row-merge tail (reading G8): it runs once
+    // every chunk is traversed, and only the last chunk's scan waits for it
+    const bool defer = h->defer_win > 0 && h->defer_list != nullptr;
+    h->tail_ran = false;
+    if (defer) CK(cudaMemsetAsync(h->dstats + kSlotDefer, 0, 6 * sizeof(unsigned long long), s));
     CK(cudaEventRecord(ev_count[kMaxChunks], s));
     for (cudaStream_t x : {cs[1], cs[2], sp, sc})
         CK(cudaStreamWaitEvent(x, ev_count[kMaxChunks], 0));
@@ -988,14 +1250,21 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
     for (int pos = 0; pos < nchunks; ++pos) {
         const int k = hl ? (pos == 0 ? nchunks - 1 : pos - 1) : pos;
         const int set = set_of(k);
-        if (b[k] < b[k + 1] &&
-            (st = run_pass(h, kStage, b[k], b[k + 1], d_fill_count, nullptr, nullptr, cs[set],
-                           nullptr, 0, set, false)) != LU_OK)
-            return st;
+        h->defer_active = defer && k == nchunks - 1;
+        h->defer_from = b[k];
+        st = b[k] < b[k + 1] ? run_pass(h, kStage, b[k], b[k + 1], d_fill_count, nullptr, nullptr,
+                                        cs[set], nullptr, 0, set, false)
+                             : LU_OK;
+        h->defer_active = false;
+        if (st != LU_OK) return st;
         CK(cudaEventRecord(ev_count[k], cs[set]));
     }
     for (int k = nchunks - 1; k >= 0 && k >= nchunks - 3; --k)  // the last chunk of each set
         CK(cudaStreamWaitEvent(s, ev_count[k], 0));
+    if (defer) {  // s follows every chunk's traversal: finish the deferred rows
+        if ((st = run_tail(h, d_fill_count, s)) != LU_OK) return st;
+        CK(cudaEventRecord(ev_count[nchunks - 1], s));
+    }
     CK(cudaEventRecord(h->ev[kEvCount][1], s));  // s now follows every chunk's traversal
     h->ev_used[kEvCount] = true;
     // per chunk, behind its traversal: chained prefix sum, placement (symbolic_2 of staged
@@ -1199,7 +1468,7 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
     if (!hc || !out) return fail(LU_ERR_ARG, "null pointer");
     lu_sym *h = const_cast<lu_sym *>(hc);
     double *ms[kEvN] = {&h->stats.ms_count, &h->stats.ms_scan, &h->stats.ms_emit,
-                        &h->stats.ms_levelize};
+                        &h->stats.ms_levelize, &h->stats.ms_tail};
     for (int k = 0; k < kEvN; ++k) {
         if (!h->ev_used[k]) continue;
         if (cudaEventSynchronize(h->ev[k][1]) != cudaSuccess) continue;
@@ -1215,6 +1484,20 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
             h->stats.vertices_scanned_emit = (int64_t)st[5 + kStatVerts];
             h->stats.spills = (int64_t)(st[1 + kStatSpills] + st[5 + kStatSpills]);
         }
+        unsigned long long dt[6] = {};
+        if (h->tail_ran && cudaMemcpy(dt, h->dstats + kSlotDefer, sizeof(dt),
+                                      cudaMemcpyDeviceToHost) == cudaSuccess) {
+            h->stats.rows_deferred = (int64_t)std::min<unsigned long long>(dt[0], h->defer_max);
+            h->stats.rows_merge_failed = (int64_t)dt[2];
+            h->stats.merge_entries_read = (int64_t)dt[3];
+            h->stats.merge_rounds = (int64_t)dt[4];
+            h->stats.merge_waits = (int64_t)dt[5];
+        } else {
+            h->stats.merge_rounds = h->stats.merge_waits = 0;
+            h->stats.rows_deferred = h->stats.rows_merge_failed = 0;
+            h->stats.merge_entries_read = 0;
+            h->stats.ms_tail = 0;
+        }
     }
     h->stats.scratch_bytes = h->scratch_bytes;
     h->stats.rows_in_flight = h->grid;
@@ -1226,6 +1509,7 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
     h->stats.queue_capacity = h->q;
     h->stats.kernel_launches = h->launches;
     h->stats.pool_bytes = h->pool ? h->pool_cap * (int64_t)sizeof(int32_t) : 0;
+    h->stats.sample_mean_sv = h->sparse_sv;
     *out = h->stats;
     return LU_OK;
 }

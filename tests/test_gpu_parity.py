@@ -327,67 +327,46 @@ def test_cfg2_full_bench_launch_config():
 
 
 @pytest.mark.slow
-def test_cfg3_sampled_rows_and_levels():
+def test_cfg3_full():
+    """cfg3 (circuit, n = 2^20, hubs last; rows deferred to the row-merge tail and the sparse
+    planner class on by default): counts, row_ptr and col_idx of EVERY row against the full
+    oracle, and both rules' levels of the GPU pattern against the oracle's Kahn."""
     rp, ci = gen.circuit(1024, 1)
-    n = len(rp) - 1
+    ref = oracle.fill2(rp, ci)
     g = gpu_run(rp, ci, rules=("u", "glu3"))
-    rng = np.random.default_rng(3)
-    rows = np.unique(np.concatenate([rng.choice(n, 1500, replace=False),
-                                     np.arange(n - 300, n)])).astype(np.int32)
-    ref = oracle.fill2(rp, ci, rows=rows)
-    for k, i in enumerate(rows):
-        a, b = ref["row_ptr"][k], ref["row_ptr"][k + 1]
-        got = g["col_idx"][g["row_ptr"][i]:g["row_ptr"][i + 1]]
-        assert np.array_equal(got, ref["col_idx"][a:b]), f"row {i}"
-    assert np.array_equal(np.diff(g["row_ptr"]), g["counts"])
-    # levels of the GPU pattern vs the oracle's Kahn on the same pattern (bit-exact)
+    assert np.array_equal(g["counts"], ref["counts"])
+    assert np.array_equal(g["row_ptr"], ref["row_ptr"])
+    assert np.array_equal(g["col_idx"], ref["col_idx"])
+    assert g["stats"]["rows_deferred"] > 0          # the hubs went through the tail
     for r in ("u", "glu3"):
-        lv, nl = oracle.levels(g["row_ptr"], g["col_idx"], r)
+        lv, nl = oracle.levels(ref["row_ptr"], ref["col_idx"], r)
         assert np.array_equal(g["levels"][r][0], lv) and g["levels"][r][1] == nl
-
-
-def _closed_form_counts_2d(k):
-    n = k * k
-    i = np.arange(n)
-    y, x = i // k, i % k
-    L = np.where(y >= 1, k, np.where(x >= 1, 1, 0))
-    U = np.where(y == k - 1, n - i, np.where(y >= 1, k + 1, 1 + (x < k - 1) + x + 1))
-    return (L + U).astype(np.int64)
-
-
-def _closed_form_counts_3d(k):
-    n = k ** 3
-    k2 = k * k
-    i = np.arange(n)
-    z, p = i // k2, i % k2
-    c2 = _closed_form_counts_2d(k)[p] + (p + 1)         # plane-0 rows gain [k^2, k^2+p]
-    cz = np.where(z == k - 1, k2 + (n - i), 2 * k2 + 1)
-    return np.where(z == 0, c2, cz).astype(np.int64)
 
 
 @pytest.mark.slow
 @pytest.mark.parametrize("cfg", [4, 5])
 def test_cfg45_closed_forms(cfg):
-    """cfg4/cfg5 (2.1e9 entries): every count vs the closed form, sampled rows vs the closed
-    form rows and the oracle, levels == arange(n) (chains), checked on the device."""
+    """cfg4/cfg5 (2.1e9 entries): EVERY row (counts, row_ptr, col_idx) against the closed form,
+    expanded on the device chunk by chunk (tests/closed_forms.py); sampled rows also against
+    the oracle; levels == arange(n) (chains)."""
+    from tests import closed_forms
     name, rp, ci = gen.config(cfg)
     n = len(rp) - 1
-    k = 1024 if cfg == 4 else 64
+    k, kind = (1024, "2d") if cfg == 4 else (64, "3d")
     d = dev()
     h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
     fc, rp_lu, ci_lu = h.run()
-    expect = _closed_form_counts_2d(k) if cfg == 4 else _closed_form_counts_3d(k)
-    assert np.array_equal(fc.cpu().numpy().astype(np.int64), expect)
     nnz = pins.nnz_2d(k) if cfg == 4 else pins.nnz_3d(k)
     assert int(rp_lu[-1]) == nnz
+    assert torch.equal(fc.to(torch.int64), closed_forms.counts(kind, k, torch, d))
+    assert closed_forms.check_device(kind, k, rp_lu, ci_lu) == nnz
     rng = np.random.default_rng(cfg)
-    rows = np.unique(np.concatenate([rng.choice(n, 200, replace=False), [0, 1, n - 2, n - 1]]))
+    rows = np.unique(np.concatenate([rng.choice(n, 64, replace=False), [0, 1, n - 2, n - 1]]))
     rpl = rp_lu.cpu().numpy()
     ref = oracle.fill2(rp, ci, rows=rows.astype(np.int32))
     for kk, i in enumerate(rows):
         got = ci_lu[int(rpl[i]):int(rpl[i + 1])].cpu().numpy()
         assert np.array_equal(got, ref["col_idx"][ref["row_ptr"][kk]:ref["row_ptr"][kk + 1]])
-    # every row sorted and inside [0, n): checked on the device in chunks
     lv, nl = h.levelize(rp_lu, ci_lu, "u")
     assert nl == n
     assert torch.equal(lv, torch.arange(n, dtype=torch.int32, device=d))
@@ -485,3 +464,108 @@ def test_symbolic_distributed_single_rank():
     assert nl == nref and np.array_equal(lv.cpu().numpy(), lref)
     fc, rp_lu, ci_lu, lv, nl = lu.symbolic_distributed(*args, output="local_rows")
     assert lv is None and np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+
+
+# ---------------------------------------------------------------- deferred rows (reading G8)
+def _hub_matrix(n=3000, hubs=6, deg=900, seed=70_001):
+    """Random pattern whose last rows are hubs (degree >> mean): the rows fill2 serialises on."""
+    rp0, ci0 = gen.random_pattern(n, 1.5, seed=seed)
+    R = [np.repeat(np.arange(n), np.diff(rp0))]
+    C = [ci0.astype(np.int64)]
+    for hub in range(n - hubs, n):
+        nb = np.random.default_rng(hub).choice(n, deg, replace=False)
+        R += [np.full(nb.size, hub), nb]
+        C += [nb, np.full(nb.size, hub)]
+    return gen.csr_from_edges(n, np.concatenate(R), np.concatenate(C))
+
+
+DEFER_KNOBS = [
+    dict(defer_windows=1),                          # nearly every row with a threshold defers
+    dict(defer_windows=2, defer_max=5),             # the cap: the rest finish by traversal
+    dict(defer_windows=1, defer_max=4096),
+    dict(defer_windows=1, pool_bytes=300_000),      # pool too small: tail rows fail -> fill2
+    dict(defer_windows=3, queue_capacity=32),       # tail frontiers spill to HBM
+    dict(defer_windows=1, flags=lu.F_FORCE_CLASSES),
+    dict(defer_windows=1, flags=lu.F_ASCENDING),
+    dict(defer_windows=2, rows_in_flight=3),
+]
+
+
+@pytest.mark.parametrize("knob", DEFER_KNOBS, ids=[str(k) for k in DEFER_KNOBS])
+def test_deferred_rows_row_merge_tail(knob):
+    """Rows abandoned by fill2 and finished by the row-merge closure over staged rows are
+    bit-exact; chains of deferred rows (a row waiting for a deferred row below it) included."""
+    for rp, ci in (_hub_matrix(), gen.circuit(48, 3), gen.lap3d(9), gen.lap2d(24),
+                   gen.random_pattern(900, 2.5, seed=12), gen.arrow_first(300)):
+        g = check(rp, ci, tag=str(knob), **knob)
+        st = g["stats"]
+        if knob.get("defer_windows") == 1 and "pool_bytes" not in knob:
+            assert st["rows_deferred"] > 0 or len(rp) < 400, st
+
+
+def test_deferred_rows_hbm_bitmap_variant(monkeypatch):
+    monkeypatch.setenv("LUSYM_MERGE_HBM_BITMAP", "1")
+    for rp, ci in (_hub_matrix(), gen.circuit(40, 2)):
+        g = check(rp, ci, tag="merge-hbm", defer_windows=1)
+        assert g["stats"]["rows_deferred"] > 0
+
+
+def test_deferred_rows_stats_and_row_ranges():
+    """The tail only runs when every row below is staged by the handle: a count over [0, n)
+    defers, a count over an upper block alone does not; both are exact."""
+    rp, ci = _hub_matrix(n=4000, hubs=8, deg=1500, seed=3)
+    n = len(rp) - 1
+    ref = oracle.fill2(rp, ci)
+    d = dev()
+    h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d), defer_windows=2)
+    fc = torch.zeros(n, dtype=torch.int32, device=d)
+    h.count(2000, n, fc)                       # rows below 2000 are not staged: no deferral
+    assert h.stats()["rows_deferred"] == 0
+    assert np.array_equal(fc.cpu().numpy()[2000:], ref["counts"][2000:])
+    fc = h.count()
+    st = h.stats()
+    assert st["rows_deferred"] > 0 and st["rows_merge_failed"] == 0
+    assert st["merge_entries_read"] > 0 and st["ms_tail"] > 0
+    assert np.array_equal(fc.cpu().numpy(), ref["counts"])
+    rp_lu, nnz = h.scan(fc)
+    ci_lu = h.emit(rp_lu)
+    assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+    assert h.stats()["rows_retraversed"] == 0
+    # two calls covering [0, n) in increasing order: the second may defer
+    h.count(0, 2000, fc)
+    h.count(2000, n, fc)
+    assert np.array_equal(fc.cpu().numpy(), ref["counts"])
+    rp_lu, nnz = h.scan(fc)
+    assert np.array_equal(h.emit(rp_lu).cpu().numpy(), ref["col_idx"])
+    h.close()
+
+
+@pytest.mark.parametrize("nchunks", [3, 8])
+def test_deferred_rows_run_host(nchunks):
+    d = dev()
+    for rp, ci in (_hub_matrix(), gen.circuit(48, 5)):
+        ref = oracle.fill2(rp, ci)
+        nnz = int(ref["row_ptr"][-1])
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d), defer_windows=1)
+        for _ in range(2):
+            hr = torch.full((len(rp),), -7, dtype=torch.int64).pin_memory()
+            hc = torch.full((nnz,), -7, dtype=torch.int32).pin_memory()
+            fc, rp_lu, ci_lu = h.run_host(nnz, hr, hc, nchunks=nchunks)
+            torch.cuda.synchronize()
+            assert np.array_equal(fc.cpu().numpy(), ref["counts"])
+            assert np.array_equal(hr.numpy(), ref["row_ptr"])
+            assert np.array_equal(hc.numpy(), ref["col_idx"])
+        h.close()
+
+
+@pytest.mark.parametrize("knob", [dict(), dict(defer_windows=1), dict(queue_capacity=0, rows_in_flight=5),
+                                  dict(flags=lu.F_TWO_PASS)], ids=str)
+def test_sparse_class_forced(monkeypatch, knob):
+    """The planner's sparse class (reading G9: HBM visited slots, 128-thread CTAs) replacing
+    every shared-memory class, forced on small inputs; bit-exact."""
+    monkeypatch.setenv("LUSYM_FORCE_SPARSE", "1")
+    for rp, ci in (gen.lap3d(9), gen.circuit(48, 2), _hub_matrix(), gen.lap2d(20),
+                   gen.random_pattern(700, 2.5, seed=9)):
+        g = check(rp, ci, tag=f"sparse {knob}", **knob)
+        assert g["stats"]["visited_in_smem"] == 0 and g["stats"]["row_classes"] == 1
+        assert g["stats"]["sample_mean_sv"] == 0.0

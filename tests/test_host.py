@@ -30,7 +30,7 @@ def test_library_exports_every_declared_symbol():
     for name in names:
         assert hasattr(lib, name), name
     assert set(names) == set(lu.EXPORTED)
-    assert lib.lu_sym_abi_version() == 1
+    assert lib.lu_sym_abi_version() == lu.ABI_VERSION
 
 
 def test_status_strings_and_opts_layout():

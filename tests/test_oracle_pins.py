@@ -132,6 +132,35 @@ def test_closed_form_3d(k):
     assert np.array_equal(r["sv"], np.arange(len(rp) - 1))
 
 
+@pytest.mark.parametrize("kind,k", [("2d", k) for k in (1, 2, 3, 5, 8, 17, 40)] +
+                         [("3d", k) for k in (1, 2, 3, 4, 7, 9)])
+def test_interval_closed_forms_expand_to_pinned_rows(kind, k):
+    """tests/closed_forms.py (the O(nnz) checker used on cfg4/cfg5 at full size, on the device)
+    expands to exactly the pinned closed-form rows and to the oracle's CSR, whole and in row
+    blocks, with numpy and with torch."""
+    import torch
+    from tests import closed_forms
+    rows = [[0]] if k == 1 else (pins.closed_form_2d(k) if kind == "2d" else pins.closed_form_3d(k))
+    flat = np.concatenate([np.array(r, dtype=np.int64) for r in rows])
+    n = len(rows)
+    assert np.array_equal(closed_forms.expand_rows(kind, k, 0, n), flat)
+    assert np.array_equal(closed_forms.counts(kind, k), [len(r) for r in rows])
+    rp, ci = gen.lap2d(k) if kind == "2d" else gen.lap3d(k)
+    ref = oracle.fill2(rp, ci)
+    assert np.array_equal(ref["col_idx"], flat)
+    for a, b in ((0, n // 2), (n // 3, n), (n - 1, n)):
+        if a < b:
+            got = closed_forms.expand_rows(kind, k, a, b, torch, "cpu").numpy()
+            assert np.array_equal(got, ref["col_idx"][ref["row_ptr"][a]:ref["row_ptr"][b]])
+    # the device checker itself, run here on CPU tensors: accepts the truth, rejects a flip
+    trp, tci = torch.from_numpy(ref["row_ptr"]), torch.from_numpy(ref["col_idx"].copy())
+    assert closed_forms.check_device(kind, k, trp, tci, chunk_entries=97) == flat.size
+    if flat.size > 3:
+        tci[flat.size // 2] += 1
+        with pytest.raises(AssertionError):
+            closed_forms.check_device(kind, k, trp, tci, chunk_entries=97)
+
+
 def test_closed_form_counts_cfg2():
     """cfg2 (3D 40^3): nnz(L+U) = 2k^5-2k^4+3k^3-2k^2+2k-2 = 199,868,878 (counts only)."""
     rp, ci = gen.lap3d(40)
