@@ -92,12 +92,15 @@ struct MergeParams {
     unsigned long long *stats;         // [0] U entries read, [1] rounds, [2] waits
     int32_t q;                         // shared frontier capacity per buffer
 };
-size_t merge_smem_bytes(int n, bool smem_bitmap, int q);
+// mode 0: one CTA per row, bitmap in shared memory; 1: one CTA, bitmap in an HBM slot;
+// 2: a cluster of g CTAs per row, bitmap sliced over their shared memories (DSMEM)
+size_t merge_smem_bytes(int n, int mode, int g, int q);
 cudaError_t merge_configure(size_t smem);
+cudaError_t merge_max_clusters(int g, size_t smem, int *clusters);
 // sort list[0..min(*cnt, max)) ascending (one CTA; max <= 4096)
 cudaError_t merge_sort_list(int32_t *list, const unsigned long long *cnt, int32_t max,
                             cudaStream_t s);
-cudaError_t merge_launch(const MergeParams &p, bool smem_bitmap, int grid, size_t smem,
+cudaError_t merge_launch(const MergeParams &p, int mode, int g, int grid, size_t smem,
                          cudaStream_t s);
 constexpr int kMergeNT = 1024;
 constexpr int kMergeSortMax = 4096;

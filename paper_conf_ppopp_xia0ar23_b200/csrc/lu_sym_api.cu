@@ -152,7 +152,7 @@ struct lu_sym {
     int32_t *defer_list = nullptr, *fail_list = nullptr;  // [defer_max] each
     int32_t *mspill = nullptr, *mwait = nullptr;
     uint32_t *mgbitmap = nullptr;
-    int merge_grid = 0, merge_q = 2048;
+    int merge_grid = 0, merge_q = 2048, merge_mode = 0, merge_g = 1;
     bool merge_smem_bm = true;
     size_t merge_smem = 0;
     bool tail_ran = false;
@@ -792,9 +792,32 @@ lu_status ensure_merge(lu_sym *h)
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, h->device));
     CK(cudaDeviceGetAttribute(&smem_optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, h->device));
     const int n = h->n;
-    h->merge_smem_bm = merge_smem_bytes(n, true, h->merge_q) <= (size_t)smem_optin &&
-                       !getenv("LUSYM_MERGE_HBM_BITMAP");  // test knob: the HBM-slot variant
-    h->merge_smem = merge_smem_bytes(n, h->merge_smem_bm, h->merge_q);
+    // a cluster of G CTAs per deferred row (bitmap sliced over their shared memories), else
+    // one CTA with the bitmap in shared memory, else in an HBM slot
+    int g = 4;
+    if (const char *e = getenv("LUSYM_MERGE_CLUSTER")) g = atoi(e);  // A/B knob; 1 = no cluster
+    h->merge_mode = -1;
+    int max_rows = std::min(sms, h->defer_max);
+    if (g > 1 && !getenv("LUSYM_MERGE_HBM_BITMAP")) {
+        const size_t sm = merge_smem_bytes(n, 2, g, h->merge_q);
+        int clusters = 0;
+        if (sm <= (size_t)smem_optin && merge_configure(sm) == cudaSuccess &&
+            merge_max_clusters(g, sm, &clusters) == cudaSuccess && clusters > 0) {
+            h->merge_mode = 2;
+            h->merge_g = g;
+            h->merge_smem = sm;
+            max_rows = std::min(clusters, h->defer_max);
+        }
+        cudaGetLastError();
+    }
+    if (h->merge_mode < 0) {
+        h->merge_g = 1;
+        const bool sb = merge_smem_bytes(n, 0, 1, h->merge_q) <= (size_t)smem_optin &&
+                        !getenv("LUSYM_MERGE_HBM_BITMAP");  // test knob: the HBM-slot variant
+        h->merge_mode = sb ? 0 : 1;
+        h->merge_smem = merge_smem_bytes(n, h->merge_mode, 1, h->merge_q);
+    }
+    h->merge_smem_bm = h->merge_mode != 1;
     if (h->merge_smem > (size_t)smem_optin) {
         h->defer_win = 0;
         return LU_OK;
@@ -805,12 +828,12 @@ lu_status ensure_merge(lu_sym *h)
     const uint64_t lists = (uint64_t)2 * h->defer_max * 4;
     const uint64_t left = h->budget > (uint64_t)h->scratch_bytes + lists
                               ? h->budget - (uint64_t)h->scratch_bytes - lists : 0;
-    int64_t grid = std::min<int64_t>(sms, h->defer_max);
-    grid = std::min<int64_t>(grid, (int64_t)(left / per_cta));
-    if (grid < 1) {
+    int64_t rows = std::min<int64_t>(max_rows, (int64_t)(left / per_cta) / h->merge_g);
+    if (rows < 1) {
         h->defer_win = 0;
         return LU_OK;
     }
+    const int64_t grid = rows * h->merge_g;  // CTAs
     CK(merge_configure(h->merge_smem));
     h->merge_grid = (int)grid;
     lu_status st;
@@ -869,7 +892,7 @@ lu_status run_tail(lu_sym *h, int32_t *fill_count, cudaStream_t s)
     mp.fail_cnt = slots + 2;
     mp.stats = slots + 3;
     mp.q = h->merge_q;
-    CK(merge_launch(mp, h->merge_smem_bm, h->merge_grid, h->merge_smem, s));
+    CK(merge_launch(mp, h->merge_mode, h->merge_g, h->merge_grid, h->merge_smem, s));
     h->launches += 2;
     lu_status st = run_pass(h, kStage, 0, h->n, fill_count, nullptr, nullptr, s, h->fail_list, 0,
                             0, false, slots + 2);

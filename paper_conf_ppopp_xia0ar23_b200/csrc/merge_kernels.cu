@@ -6,32 +6,43 @@
 //     (i,j) in P  iff  A(i,j) != 0  or  (i,t) in P and (t,j) in P for some t < min(i,j).
 // Row i of L+U is therefore the least set S with S ⊇ A(i,:) and S ⊇ U_t = {j > t : (t,j) in P}
 // for every t in S with t < i (the diagonal comes from A only, reading R7).  A least fixed
-// point does not depend on the order its members are expanded in, so one CTA expands a whole
-// frontier of new members t < i at once: there is no serial chain of increasing thresholds
+// point does not depend on the order its members are expanded in, so a whole frontier of new
+// members t < i is expanded at once: there is no serial chain of increasing thresholds
 // (Alg. 1), which on circuit matrices with hubs ordered last makes a single row cost
 // 10^5 dependent threshold windows.  Rows t are read from the staging pool the count pass
 // filled (their strict-U part starts ucut[t] entries into the row).
 //
+// One row is processed by a cluster of G CTAs (kMergeCluster) whose shared memories hold the
+// row's visited bitmap in G slices (distributed shared memory, test-and-set by DSMEM atomics),
+// or by one CTA with the whole bitmap in shared memory or in an HBM slot.  Each CTA expands
+// the members it discovered itself; cluster barriers end a round.
+//
 // Rows are claimed in increasing order.  A member t that is itself a deferred row still in
-// progress is set aside until its CTA publishes it (row_off[t] >= 0, release/acquire); the
+// progress is set aside until its cluster publishes it (row_off[t] >= 0, release/acquire); the
 // smallest unfinished claimed row never waits, so the resident grid always progresses.  A row
 // that cannot be finished (a row it needs is unstaged, or the pool is full) is listed for the
 // fill2 fallback launch that follows.
 #include "internal.h"
 
 #include <climits>
+#include <cooperative_groups.h>
+
+namespace cg = cooperative_groups;
 
 namespace lusym {
 namespace {
 
 constexpr int NT = kMergeNT;
 constexpr int NW = NT / 32;
-constexpr int kU = 4;  // pool loads in flight per thread
+constexpr int kU = 4;      // pool loads in flight per thread
+constexpr int kSent = 64;  // sentinel starts past the last segment
 
 struct MHdr {
     int row, diag, fail, nwait;
     int cnt[2];
+    int tn, tw, tf, tdiag;  // cluster totals of the round (thread 0 -> block)
     long long off;
+    long long part_c, part_lo;
     long long red[2][NW];
     long long scan[NW];
 };
@@ -76,6 +87,28 @@ __device__ __forceinline__ long long scan_excl(long long x, MHdr &h, long long *
     return r;
 }
 
+// block sums of two 64-bit values (valid in every thread)
+__device__ __forceinline__ void block_sum2(long long &a, long long &b, MHdr &h)
+{
+#pragma unroll
+    for (int o = 16; o; o >>= 1) {
+        a += __shfl_xor_sync(0xffffffffu, a, o);
+        b += __shfl_xor_sync(0xffffffffu, b, o);
+    }
+    if ((threadIdx.x & 31) == 0) {
+        h.red[0][threadIdx.x >> 5] = a;
+        h.red[1][threadIdx.x >> 5] = b;
+    }
+    __syncthreads();
+    a = b = 0;
+#pragma unroll
+    for (int k = 0; k < NW; ++k) {
+        a += h.red[0][k];
+        b += h.red[1][k];
+    }
+    __syncthreads();
+}
+
 // frontier entry k of buffer b (shared up to q entries, then the CTA's HBM spill half b)
 __device__ __forceinline__ int32_t q_get(const int32_t *sq, const int32_t *gq, int q, int64_t k)
 {
@@ -97,70 +130,142 @@ __device__ __forceinline__ void q_push(bool pred, int32_t w, int *cnt, int32_t *
     }
 }
 
-// test-and-set of bit v; true iff this call set it
-__device__ __forceinline__ bool tas(uint32_t *bm, int v)
+// The row's visited bitmap: whole in this CTA (shared memory or HBM slot), or sliced over the
+// cluster, word w in rank w >> sh at local index w & (wpc - 1).
+template <bool CL>
+struct Bits {
+    uint32_t *w;  // local words
+    int sh;       // log2(words per CTA) (cluster)
+    int rank, g;  // cluster rank and size (1 / 0 without a cluster)
+    int lo, hi;   // local word range [lo, hi) in global word numbering
+
+    __device__ __forceinline__ uint32_t *word(int gw) const
+    {
+        if constexpr (!CL) return w + gw;
+        const int r = gw >> sh;
+        uint32_t *base = w + (gw & ((1 << sh) - 1));
+        return r == rank ? base : cg::this_cluster().map_shared_rank(base, r);
+    }
+    // test-and-set of bit v; true iff this call set it
+    __device__ __forceinline__ bool tas(int v) const
+    {
+        const uint32_t b = 1u << (v & 31);
+        uint32_t *p = word(v >> 5);
+        if (*p & b) return false;
+        return !(atomicOr(p, b) & b);
+    }
+};
+
+__device__ __forceinline__ void csync_impl(bool cl)
 {
-    const uint32_t b = 1u << (v & 31);
-    if (bm[v >> 5] & b) return false;
-    return !(atomicOr(bm + (v >> 5), b) & b);
+    if (cl) cg::this_cluster().sync(); else __syncthreads();
 }
 
-template <bool SB>
-__global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p)
+// MODE: 0 = one CTA, bitmap in shared memory; 1 = one CTA, bitmap in an HBM slot;
+//       2 = a cluster of G CTAs, bitmap sliced over their shared memories
+template <int MODE>
+__global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int sh)
 {
+    constexpr bool CL = MODE == 2;
     extern __shared__ __align__(16) unsigned char smem[];
     MHdr &h = *reinterpret_cast<MHdr *>(smem);
-    long long *s_off = reinterpret_cast<long long *>(smem + kHdrBytes);   // [NT]
-    long long *s_start = s_off + NT;                                       // [NT]
-    int32_t *sq = reinterpret_cast<int32_t *>(s_start + NT);              // 2 x q
+    // compacted frontier segments of one block of members: pool offset and flat start
+    long long *c_off = reinterpret_cast<long long *>(smem + kHdrBytes);    // [NT]
+    long long *c_start = c_off + NT;                                        // [NT + kSent]
+    int32_t *sq = reinterpret_cast<int32_t *>(c_start + NT + kSent);       // 2 x q
     const int nw = (p.n + 31) >> 5;
-    uint32_t *bm = SB ? reinterpret_cast<uint32_t *>(sq + 2 * p.q)
-                      : p.gbitmap + (size_t)blockIdx.x * p.gb_stride;
+    Bits<CL> bm;
+    bm.sh = sh;
+    if constexpr (CL) {
+        bm.rank = (int)cg::this_cluster().block_rank();
+        bm.g = (int)cg::this_cluster().num_blocks();
+        bm.w = reinterpret_cast<uint32_t *>(sq + 2 * p.q);
+        bm.lo = min(nw, bm.rank << sh);
+        bm.hi = min(nw, (bm.rank + 1) << sh);
+    } else {
+        bm.rank = 0;
+        bm.g = 1;
+        bm.w = MODE == 0 ? reinterpret_cast<uint32_t *>(sq + 2 * p.q)
+                         : p.gbitmap + (size_t)blockIdx.x * p.gb_stride;
+        bm.lo = 0;
+        bm.hi = nw;
+    }
+    uint32_t *lw = CL ? bm.w - bm.lo : bm.w;  // local words by global word index
     int32_t *gq0 = p.spill + (size_t)blockIdx.x * 2 * p.spill_cap;
     int32_t *wait = p.wait + (size_t)blockIdx.x * p.list_max;
     const int tid = threadIdx.x;
     const int nlist = (int)min(*p.list_cnt, (unsigned long long)p.list_max);
-    if (SB)
-        for (int w = tid; w < nw; w += NT) bm[w] = 0;
-    unsigned long long n_read = 0, n_rounds = 0, n_waits = 0;  // thread 0
+    if (MODE != 1)
+        for (int w = bm.lo + tid; w < bm.hi; w += NT) lw[w] = 0;
+    unsigned long long n_read = 0, n_rounds = 0, n_waits = 0;  // thread 0 of rank 0
     for (;;) {
         if (tid == 0) {
-            const unsigned long long c = atomicAdd(p.counter, 1ull);
-            h.row = c < (unsigned long long)nlist ? p.list[c] : -1;
             h.diag = 0;
             h.fail = 0;
             h.nwait = 0;
             h.cnt[0] = h.cnt[1] = 0;
+            if (bm.rank == 0) {
+                const unsigned long long c = atomicAdd(p.counter, 1ull);
+                h.row = c < (unsigned long long)nlist ? p.list[c] : -1;
+            }
         }
-        __syncthreads();
+        csync_impl(CL);
+        if constexpr (CL) {
+            if (tid == 0 && bm.rank != 0) h.row = cg::this_cluster().map_shared_rank(&h, 0)->row;
+            __syncthreads();
+        }
         const int i = h.row;
         if (i < 0) break;
-        // ---- seed: S = A(i,:); members t < i form the first frontier
-        if (tid == 0) atomicOr(bm + (i >> 5), 1u << (i & 31));
-        __syncthreads();
+        // ---- seed: S = A(i,:); members t < i form the first frontier (entries split by rank)
+        if (tid == 0 && bm.rank == 0) atomicOr(bm.word(i >> 5), 1u << (i & 31));
+        csync_impl(CL);
         {
             const int64_t rb = p.rp[i], re = p.rp[i + 1];
-            for (int64_t b0 = rb; b0 < re; b0 += NT) {
+            for (int64_t b0 = rb + (int64_t)bm.rank * NT; b0 < re; b0 += (int64_t)bm.g * NT) {
                 const int64_t e = b0 + tid;
                 int v = -1;
                 bool fr = false;
                 if (e < re) {
                     v = __ldg(p.ci + e);
                     if (v == i) h.diag = 1;
-                    else if (tas(bm, v)) fr = v < i;
+                    else if (bm.tas(v)) fr = v < i;
                 }
                 q_push(fr, v, &h.cnt[0], sq, gq0, p.q);
             }
         }
         __syncthreads();
         int cur = 0;
+        int diag = 0, fail = 0;
         for (;;) {
-            const int fsize = h.cnt[cur];
-            if (fsize == 0) {
-                const int nwt = h.nwait;
-                if (nwt == 0) break;
+            // cluster totals of the frontier in buffer cur, the wait lists and failures
+            csync_impl(CL);
+            if (tid == 0) {
+                int tn = h.cnt[cur], tw = h.nwait, tf = h.fail, td = h.diag;
+                if constexpr (CL)
+                    for (int r = 0; r < bm.g; ++r)
+                        if (r != bm.rank) {
+                            const MHdr *o = cg::this_cluster().map_shared_rank(&h, r);
+                            tn += o->cnt[cur];
+                            tw += o->nwait;
+                            tf |= o->fail;
+                            td |= o->diag;
+                        }
+                h.tn = tn;
+                h.tw = tw;
+                h.tf = tf;
+                h.tdiag = td;
+            }
+            __syncthreads();
+            const int tn = h.tn, tw = h.tw;
+            fail = h.tf;
+            diag = h.tdiag;
+            if constexpr (CL) cg::this_cluster().sync();  // everyone has read the counters
+            if (fail) break;
+            if (tn == 0) {
+                if (tw == 0) break;
                 // every member left is a deferred row still in progress: wait for them (each
-                // was claimed before row i by a running CTA), then expand them
+                // was claimed before row i by a running cluster), then expand them
+                const int nwt = h.nwait;
                 for (int k = tid; k < nwt; k += NT) {
                     const int t = wait[k];
                     while (ld_acquire(p.row_off + t) == kRowDeferred) __nanosleep(200);
@@ -176,10 +281,10 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p)
                     h.cnt[cur] = nwt;
                     h.nwait = 0;
                 }
-                __syncthreads();
                 continue;
             }
             const int nxt = cur ^ 1;
+            const int fsize = h.cnt[cur];
             const int32_t *fq = sq + cur * p.q, *gfq = gq0 + (size_t)cur * p.spill_cap;
             int32_t *nq = sq + nxt * p.q, *gnq = gq0 + (size_t)nxt * p.spill_cap;
             for (int base = 0; base < fsize; base += NT) {
@@ -198,33 +303,55 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p)
                         len = (long long)__ldcg(p.fill_count + t) - uc;
                     }
                 }
+                // compact the non-empty segments (strictly increasing starts): one scan of
+                // (len << 11 | nonempty)
                 long long total;
-                const long long st = scan_excl(len, h, &total);
-                s_off[tid] = off;
-                s_start[tid] = st;  // non-decreasing; an empty segment shares its successor's start
+                const long long st = scan_excl((len << 11) | (len > 0 ? 1 : 0), h, &total);
+                const int nsrc = (int)(total & 2047);
+                const long long E = total >> 11;
+                if (len > 0) {
+                    c_start[st & 2047] = st >> 11;
+                    c_off[st & 2047] = off;
+                }
+                if (tid < kSent) c_start[nsrc + tid] = LLONG_MAX;
                 __syncthreads();
-                if (tid == 0) n_read += (unsigned long long)total;
-                // the member owning flat position pos: the last k with s_start[k] <= pos (never an
-                // empty segment, and never one past the frontier: those start at total)
-                for (long long p0 = 0; p0 < total; p0 += (long long)NT * kU) {
-                    int jv[kU];
+                if (tid == 0) n_read += (unsigned long long)E;
+                // each warp expands a contiguous chunk of the E flat positions, 32 at a time: one
+                // binary search for the chunk's first owner, then the owner of lane l of a window
+                // [p, p+32) is that window's owner plus the segments starting in (p, p+l]
+                // (one OR-reduction of 32 start bits, no per-entry search)
+                const int wid = tid >> 5, lane = tid & 31;
+                const long long C = ((E + NW - 1) / NW + 31) & ~31ll;
+                long long pw = (long long)wid * C;
+                const long long pend = min(E, pw + C);
+                if (pw < pend) {
+                    int src = 0;
 #pragma unroll
-                    for (int u = 0; u < kU; ++u) {
-                        const long long pos = p0 + (long long)u * NT + tid;
-                        jv[u] = -1;
-                        if (pos < total) {
-                            int lo = 0;
+                    for (int step = NT / 2; step >= 1; step >>= 1)
+                        if (src + step < nsrc && c_start[src + step] <= pw) src += step;
+                    while (pw < pend) {
+                        int jv[kU];
 #pragma unroll
-                            for (int step = NT / 2; step >= 1; step >>= 1)
-                                if (s_start[lo + step] <= pos) lo += step;
-                            jv[u] = __ldcg(p.pool + s_off[lo] + (pos - s_start[lo]));
+                        for (int u = 0; u < kU; ++u) {
+                            jv[u] = -1;
+                            if (pw < pend) {
+                                const long long sn = c_start[src + 1 + lane];
+                                const unsigned bit = sn < pw + 32 ? 1u << (int)(sn - pw) : 0u;
+                                const unsigned mask = __reduce_or_sync(0xffffffffu, bit);
+                                const int my = src + __popc(mask & ((2u << lane) - 1u));
+                                if (pw + lane < pend)
+                                    jv[u] = p.pool[c_off[my] + (pw + lane - c_start[my])];
+                                const int last = __shfl_sync(0xffffffffu, my, 31);
+                                src = last + (c_start[last + 1] == pw + 32 ? 1 : 0);
+                                pw += 32;
+                            }
                         }
-                    }
 #pragma unroll
-                    for (int u = 0; u < kU; ++u) {
-                        const int j = jv[u];
-                        const bool fr = j >= 0 && tas(bm, j) && j < i;
-                        q_push(fr, j, &h.cnt[nxt], nq, gnq, p.q);
+                        for (int u = 0; u < kU; ++u) {
+                            const int j = jv[u];
+                            const bool fr = j >= 0 && bm.tas(j) && j < i;
+                            q_push(fr, j, &h.cnt[nxt], nq, gnq, p.q);
+                        }
                     }
                 }
                 __syncthreads();
@@ -234,77 +361,83 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p)
                 ++n_rounds;
             }
             __syncthreads();
-            if (h.fail) break;
             cur = nxt;
         }
-        // ---- output: the set bits, ascending, into the pool; publish the row
-        if (!h.fail) {
-            if (tid == 0 && !h.diag) atomicAnd(bm + (i >> 5), ~(1u << (i & 31)));
+        // ---- output: the set bits, ascending, into the pool; publish the row.  Each rank
+        // writes its own word slice at the offset of the slices before it.
+        if (!fail) {
+            if (tid == 0 && !diag && (i >> 5) >= bm.lo && (i >> 5) < bm.hi)
+                atomicAnd(lw + (i >> 5), ~(1u << (i & 31)));
             __syncthreads();
             long long c = 0, lo = 0;
-            for (int w = tid; w < nw; w += NT) {
-                const uint32_t x = bm[w];
+            for (int w = bm.lo + tid; w < bm.hi; w += NT) {
+                const uint32_t x = lw[w];
                 const int pc = __popc(x);
                 c += pc;
                 if (w < (i >> 5)) lo += pc;
                 else if (w == (i >> 5)) lo += __popc(x & ((i & 31) == 31 ? 0xffffffffu
                                                                            : ((2u << (i & 31)) - 1u)));
             }
-#pragma unroll
-            for (int o = 16; o; o >>= 1) {
-                c += __shfl_xor_sync(0xffffffffu, c, o);
-                lo += __shfl_xor_sync(0xffffffffu, lo, o);
-            }
-            if ((tid & 31) == 0) {
-                h.red[0][tid >> 5] = c;
-                h.red[1][tid >> 5] = lo;
-            }
-            __syncthreads();
-            if (tid == 0) {
-                long long cc = 0, ll = 0;
-                for (int k = 0; k < NW; ++k) {
-                    cc += h.red[0][k];
-                    ll += h.red[1][k];
+            block_sum2(c, lo, h);
+            long long before = 0;
+            if constexpr (CL) {
+                if (tid == 0) {
+                    h.part_c = c;
+                    h.part_lo = lo;
                 }
-                const unsigned long long o = atomicAdd(p.pool_cursor, (unsigned long long)cc);
-                const bool fits = o + (unsigned long long)cc <= (unsigned long long)p.pool_cap;
+                cg::this_cluster().sync();
+                long long tc = 0, tl = 0;
+                for (int r = 0; r < bm.g; ++r) {
+                    const MHdr *o = cg::this_cluster().map_shared_rank(&h, r);
+                    if (r < bm.rank) before += o->part_c;
+                    tc += o->part_c;
+                    tl += o->part_lo;
+                }
+                c = tc;
+                lo = tl;
+            }
+            if (tid == 0 && bm.rank == 0) {
+                const unsigned long long o = atomicAdd(p.pool_cursor, (unsigned long long)c);
+                const bool fits = o + (unsigned long long)c <= (unsigned long long)p.pool_cap;
                 h.off = fits ? (long long)o : -1ll;
                 if (fits) {
-                    p.fill_count[i] = (int32_t)cc;
-                    p.ucut[i] = (int32_t)ll;
-                } else {
-                    h.fail = 1;
+                    p.fill_count[i] = (int32_t)c;
+                    p.ucut[i] = (int32_t)lo;
                 }
             }
-            __syncthreads();
-            if (!h.fail) {
-                int32_t *dst = p.pool + h.off;
+            csync_impl(CL);
+            long long off = h.off;
+            if constexpr (CL) off = cg::this_cluster().map_shared_rank(&h, 0)->off;
+            if (off < 0) {
+                fail = 1;
+            } else {
+                int32_t *dst = p.pool + off + before;
                 long long run = 0;
-                for (int w0 = 0; w0 < nw; w0 += NT) {
+                for (int w0 = bm.lo; w0 < bm.hi; w0 += NT) {
                     const int w = w0 + tid;
-                    uint32_t x = w < nw ? bm[w] : 0u;
+                    uint32_t x = w < bm.hi ? lw[w] : 0u;
                     long long tot;
                     long long pos = run + scan_excl(__popc(x), h, &tot);
                     for (; x; x &= x - 1, ++pos) dst[pos] = (w << 5) + __ffs(x) - 1;
                     run += tot;
                 }
                 __threadfence();
-                __syncthreads();
-                if (tid == 0) st_release(p.row_off + i, h.off);
+                csync_impl(CL);
+                if (tid == 0 && bm.rank == 0) st_release(p.row_off + i, off);
             }
         }
-        if (h.fail && tid == 0) {
+        if (fail && tid == 0 && bm.rank == 0) {
             p.fail_list[atomicAdd(p.fail_cnt, 1ull)] = i;
             st_release(p.row_off + i, -1);
         }
         // ---- fill(:) = 0 for the next row (L115)
         __syncthreads();
-        for (int w = tid; w < nw; w += NT) bm[w] = 0;
-        __syncthreads();
+        for (int w = bm.lo + tid; w < bm.hi; w += NT) lw[w] = 0;
+        // (the next claim's cluster barrier orders this before any rank's next seed)
     }
     if (tid == 0 && p.stats) {
         atomicAdd(p.stats + 0, n_read);
-        atomicAdd(p.stats + 1, n_rounds);
+        atomicAdd(p.stats + 1, bm.rank == 0 ? n_rounds : 0ull);
         atomicAdd(p.stats + 2, n_waits);
     }
 }
@@ -338,22 +471,53 @@ __global__ void __launch_bounds__(1024) k_sort_list(int32_t *list, const unsigne
     for (int k = threadIdx.x; k < m; k += blockDim.x) list[k] = a[k];
 }
 
+int cluster_shift(int n, int g)
+{
+    const int nw = (n + 31) / 32;
+    const int per = (nw + g - 1) / g;
+    int sh = 0;
+    while ((1 << sh) < per) ++sh;
+    return sh;
+}
+
 }  // namespace
 
-size_t merge_smem_bytes(int n, bool smem_bitmap, int q)
+size_t merge_smem_bytes(int n, int mode, int g, int q)
 {
-    size_t b = kHdrBytes + 2 * (size_t)NT * sizeof(long long) + 2 * (size_t)q * sizeof(int32_t);
-    if (smem_bitmap) b += (size_t)((n + 31) / 32) * sizeof(uint32_t);
+    size_t b = kHdrBytes + (2 * (size_t)NT + kSent) * sizeof(long long) +
+               2 * (size_t)q * sizeof(int32_t);
+    if (mode == 0) b += (size_t)((n + 31) / 32) * sizeof(uint32_t);
+    if (mode == 2) b += ((size_t)1 << cluster_shift(n, g)) * sizeof(uint32_t);
     return (b + 15) & ~(size_t)15;
 }
 
 cudaError_t merge_configure(size_t smem)
 {
-    cudaError_t e = cudaFuncSetAttribute(k_merge_rows<true>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-    return cudaFuncSetAttribute(k_merge_rows<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                (int)smem);
+    const void *fns[3] = {(const void *)k_merge_rows<0>, (const void *)k_merge_rows<1>,
+                          (const void *)k_merge_rows<2>};
+    for (const void *f : fns) {
+        cudaError_t e = cudaFuncSetAttribute(f, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                             (int)smem);
+        if (e != cudaSuccess) return e;
+    }
+    return cudaFuncSetAttribute((const void *)k_merge_rows<2>,
+                                cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+}
+
+cudaError_t merge_max_clusters(int g, size_t smem, int *clusters)
+{
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(g * 64, 1, 1);
+    cfg.blockDim = dim3(NT, 1, 1);
+    cfg.dynamicSmemBytes = smem;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = g;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaOccupancyMaxActiveClusters(clusters, (const void *)k_merge_rows<2>, &cfg);
 }
 
 cudaError_t merge_sort_list(int32_t *list, const unsigned long long *cnt, int32_t max,
@@ -363,14 +527,30 @@ cudaError_t merge_sort_list(int32_t *list, const unsigned long long *cnt, int32_
     return cudaGetLastError();
 }
 
-cudaError_t merge_launch(const MergeParams &p, bool smem_bitmap, int grid, size_t smem,
+cudaError_t merge_launch(const MergeParams &p, int mode, int g, int grid, size_t smem,
                          cudaStream_t s)
 {
     static_assert(sizeof(MHdr) <= kHdrBytes, "merge header too large");
-    if (smem_bitmap)
-        k_merge_rows<true><<<grid, NT, smem, s>>>(p);
-    else
-        k_merge_rows<false><<<grid, NT, smem, s>>>(p);
+    if (mode == 0) {
+        k_merge_rows<0><<<grid, NT, smem, s>>>(p, 0);
+    } else if (mode == 1) {
+        k_merge_rows<1><<<grid, NT, smem, s>>>(p, 0);
+    } else {
+        cudaLaunchConfig_t cfg = {};
+        cfg.gridDim = dim3(grid, 1, 1);  // CTAs: a multiple of g
+        cfg.blockDim = dim3(NT, 1, 1);
+        cfg.dynamicSmemBytes = smem;
+        cfg.stream = s;
+        cudaLaunchAttribute attr[1];
+        attr[0].id = cudaLaunchAttributeClusterDimension;
+        attr[0].val.clusterDim.x = g;
+        attr[0].val.clusterDim.y = 1;
+        attr[0].val.clusterDim.z = 1;
+        cfg.attrs = attr;
+        cfg.numAttrs = 1;
+        const int sh = cluster_shift(p.n, g);
+        return cudaLaunchKernelEx(&cfg, k_merge_rows<2>, p, sh);
+    }
     return cudaGetLastError();
 }
 

@@ -503,11 +503,18 @@ def test_deferred_rows_row_merge_tail(knob):
             assert st["rows_deferred"] > 0 or len(rp) < 400, st
 
 
-def test_deferred_rows_hbm_bitmap_variant(monkeypatch):
-    monkeypatch.setenv("LUSYM_MERGE_HBM_BITMAP", "1")
-    for rp, ci in (_hub_matrix(), gen.circuit(40, 2)):
-        g = check(rp, ci, tag="merge-hbm", defer_windows=1)
-        assert g["stats"]["rows_deferred"] > 0
+@pytest.mark.parametrize("variant", [("LUSYM_MERGE_HBM_BITMAP", "1"), ("LUSYM_MERGE_CLUSTER", "1"),
+                                     ("LUSYM_MERGE_CLUSTER", "2"), ("LUSYM_MERGE_CLUSTER", "8"),
+                                     ("LUSYM_MERGE_CLUSTER", "16")], ids=str)
+def test_deferred_rows_tail_variants(monkeypatch, variant):
+    """The tail's bitmap placements: one CTA per row with an HBM slot or a shared-memory
+    bitmap, and clusters of 2/8/16 CTAs with the bitmap sliced over distributed shared memory
+    (the default is 4)."""
+    monkeypatch.setenv(*variant)
+    for rp, ci in (_hub_matrix(), gen.circuit(40, 2), gen.lap2d(24)):
+        for knob in (dict(defer_windows=1), dict(defer_windows=2, queue_capacity=32)):
+            g = check(rp, ci, tag=f"merge {variant} {knob}", **knob)
+            assert g["stats"]["rows_deferred"] > 0
 
 
 def test_deferred_rows_stats_and_row_ranges():
