@@ -7,11 +7,15 @@ levelize) on synthetic BASELINE.json workloads.
 One step = one pass of the whole hot path (SURVEY §8(a) S1-S9 minus the create-time S1/S2,
 which are timed in the e2e number) over the workload, inputs resident in HBM.  For N > 1 the
 script runs under torchrun, one rank per GPU, rows sharded (strong scaling of one matrix):
-count own rows, all-reduce counts, scan, emit own rows, allgatherv the pattern, levelize.
+count own rows, all-reduce counts, scan, emit own rows, all-gather the pattern, levelize.
 Timed with CUDA events on the launching stream, K steps bracketed by barrier + synchronize,
 max over ranks.  L2 is flushed (256 MiB write) between timed steps, outside the events.
+Every timed output is checked bit-exactly (full oracle for cfg1-3, the pinned closed form of
+every row for cfg4/cfg5), outside the events.
 
-Prints ONE JSON line (rank 0).  metric = fill entries/s = nnz(L+U) / step time.
+Prints ONE JSON line (rank 0).  metric = fill entries/s = nnz(L+U) / step time of the
+headline config (--config, default cfg2 = BASELINE.json configs[1]); `per_config` carries the
+same record for the other configs (3 timed steps each).
 --impl reference times the CPU oracle (the only reference this tier has), bounded samples.
 """
 from __future__ import annotations
@@ -47,10 +51,17 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
-    ap.add_argument("--e2e-mode", default="pipelined", choices=["pipelined", "plain"],
-                    help="pipelined: lu_sym_run_host (pattern copied to the host behind the "
-                         "traversal, 1 GPU); plain: count/scan/emit then copies")
-    ap.add_argument("--e2e-chunks", type=int, default=0, help="lu_sym_run_host chunks (0 = the library default, 16)")
+    ap.add_argument("--e2e-host", default="pinned", choices=["pinned", "pageable"],
+                    help="host output buffers of the e2e run (allocated inside the timed region)")
+    ap.add_argument("--per-config", default="1,2,3,4,5",
+                    help="configs measured after the headline one (N=1 line's per_config block); "
+                         "'' = none")
+    ap.add_argument("--per-config-steps", type=int, default=3)
+    ap.add_argument("--per-config-warmup", type=int, default=3)
+    ap.add_argument("--no-verify", action="store_true",
+                    help="skip the parity check of every timed output (never for reported runs)")
+    ap.add_argument("--apriori-partition", action="store_true",
+                    help="N>1: keep the a-priori row_ptr[i+1] cost partition (no measured pass)")
     ap.add_argument("--cpu-sample-stride", type=int, default=0,
                     help="oracle sample: every s-th row (0 = auto, ~10-30 s of CPU work)")
     ap.add_argument("--profile", action="store_true", help="short run for ncu (no extras)")
@@ -302,10 +313,9 @@ def run_reference(args, rank, world):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": t_step * 1e3,
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
         "data": "synthetic",
-        "config": {"workload": f"cfg{args.config} {name}", "n": n, "nnz_a": int(rp[-1]),
-                   "nnz_lu": nnz},
+        "config": config_key(args.config, n, int(rp[-1]), nnz, args.rule),
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": entries["threads"],
-                         "kind": "oracle",
+                         "kind": "oracle", "host": host_cpu(),
                          "sample": f"fill2 count+emit on every {stride}-th row "
                                    f"({len(entries['rows'])} rows, descending), extrapolated by "
                                    f"exact TE share x{entries['scale']:.2f}; Kahn on the full "
@@ -315,26 +325,141 @@ def run_reference(args, rank, world):
     print(json.dumps(out), flush=True)
 
 
+# --------------------------------------------------------------------------- verification
+class Verifier:
+    """Parity of every timed output ("Parity check ... on every measured run's
+    output"), on the device, outside the timed region.
+
+    cfg1-3: the full oracle (oracle/, Alg. 1 + Alg. 5 on the host cores, computed once per run)
+            -> counts, row_ptr, col_idx and levels compared element by element.
+    cfg4/5: every row against the pinned closed form of the natural-ordered grid
+            (tests/closed_forms.py, expanded on the device chunk by chunk), levels == arange(n).
+    """
+
+    def __init__(self, cfg, rp, ci, rule, dev, rank=0):
+        import torch
+        self.cfg, self.rule, self.dev = cfg, rule, dev
+        self.active = rank == 0
+        self.t_build = 0.0
+        if not self.active:
+            return
+        t0 = time.perf_counter()
+        n = len(rp) - 1
+        if cfg in (1, 2, 3):
+            import oracle
+            ref = oracle.fill2(rp, ci, threads=os.cpu_count() or 1)
+            lv, nl = oracle.levels(ref["row_ptr"], ref["col_idx"], rule)
+            self.ref = {k: torch.from_numpy(np.ascontiguousarray(v)).to(dev) for k, v in
+                        (("counts", ref["counts"]), ("row_ptr", ref["row_ptr"]),
+                         ("col_idx", ref["col_idx"]), ("level", lv))}
+            self.nl = nl
+            self.what = (f"bit-exact vs the full oracle: counts, row_ptr, col_idx ({ref['row_ptr'][-1]} "
+                         f"entries) and {rule}-rule levels, every timed step")
+        else:
+            from tests import closed_forms
+            self.cf = closed_forms
+            self.kind, self.k = ("2d", 1024) if cfg == 4 else ("3d", 64)
+            if n != (self.k ** 2 if self.kind == "2d" else self.k ** 3):
+                raise ValueError("closed-form check needs the cfg4/cfg5 grid")
+            self.counts = closed_forms.counts(self.kind, self.k, torch, dev).to(torch.int32)
+            self.nl = n
+            self.what = ("bit-exact vs the closed form of the natural-ordered grid (tests/closed_forms.py,"
+                         " pinned to the oracle): every row's count and columns, levels == arange(n), "
+                         "every timed step")
+        self.t_build = time.perf_counter() - t0
+        self.checked = 0
+
+    def __call__(self, fc, rp_lu, ci_lu, level, nl):
+        import torch
+        if not self.active:
+            return
+        if self.cfg in (1, 2, 3):
+            ok = (torch.equal(fc, self.ref["counts"]) and torch.equal(rp_lu, self.ref["row_ptr"])
+                  and torch.equal(ci_lu, self.ref["col_idx"]) and nl == self.nl
+                  and torch.equal(level, self.ref["level"]))
+        else:
+            ok = torch.equal(fc, self.counts) and nl == self.nl
+            ok = ok and self.cf.check_device(self.kind, self.k, rp_lu, ci_lu) == int(rp_lu[-1])
+            ok = ok and torch.equal(level, torch.arange(nl, dtype=torch.int32, device=self.dev))
+        if not ok:
+            raise AssertionError(f"cfg{self.cfg}: GPU output differs from the reference")
+        self.checked += 1
+
+    def host(self, rp_h, ci_h, lv_h):
+        """The e2e host copies (numpy) against the same reference."""
+        import torch
+        if not self.active:
+            return
+        if self.cfg in (1, 2, 3):
+            ok = (np.array_equal(rp_h, self.ref["row_ptr"].cpu().numpy())
+                  and np.array_equal(ci_h, self.ref["col_idx"].cpu().numpy())
+                  and np.array_equal(lv_h, self.ref["level"].cpu().numpy()))
+        else:
+            rp_t = torch.from_numpy(rp_h).to(self.dev)
+            ci_t = torch.from_numpy(ci_h).to(self.dev)
+            ok = self.cf.check_device(self.kind, self.k, rp_t, ci_t) == int(rp_h[-1])
+            ok = ok and np.array_equal(lv_h, np.arange(len(lv_h), dtype=np.int32))
+        if not ok:
+            raise AssertionError(f"cfg{self.cfg}: e2e host copy differs from the reference")
+        self.checked += 1
+
+
+def ncu_profile(cfg):
+    """Per-kernel ncu figures of this config (profiles/r02/ncu_summary.json, written by
+    scripts/summarize_ncu.py from `ncu --set full` captures of scripts/prof_count.py)."""
+    try:
+        return json.load(open(os.path.join(ROOT, "profiles", "r02", "ncu_summary.json"))).get(
+            f"cfg{cfg}")
+    except Exception:
+        return None
+
+
+def host_cpu():
+    """lscpu model / sockets / cores / threads of this host (the oracle arm's machine)."""
+    info = {"logical_cpus": os.cpu_count()}
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            k, _, v = line.partition(":")
+            k, v = k.strip(), v.strip()
+            if k in ("Model name", "Socket(s)", "Core(s) per socket", "Thread(s) per core"):
+                info[k] = v
+    except Exception:
+        pass
+    return info
+
+
 # --------------------------------------------------------------------------- our arm
-def run_ours(args, rank, world, local_rank):
+def peak_hbm():
+    try:
+        return float(json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))["hbm_gbs"]), \
+            "MEASURED_PEAKS.json hbm_gbs (of measured)"
+    except Exception:
+        return 6650.0, "B200_PROFILING.md fallback 6.65 TB/s (of fallback)"
+
+
+def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
+    """Time `steps` hot-path steps of config `cfg` (after `warmup`), verify every timed output,
+    return the per-config record.  One step: count (S3, + the row-merge tail) -> [all-reduce
+    counts] -> scan (S4) -> allocate (S5) -> emit (S6) -> [all-gather pattern] -> levelize (S8+S9)."""
     import torch
     import torch.distributed as dist
     import paper_conf_ppopp_xia0ar23_b200 as lu
 
     dev = torch.device("cuda", local_rank)
-    torch.cuda.set_device(dev)
     stream = torch.cuda.current_stream()
-    name, rp_np, ci_np = gen.config(args.config)
+    name, rp_np, ci_np = gen.config(cfg)
     n = len(rp_np) - 1
-    te, sv = work_units(rp_np, args.config)
+    te, sv = work_units(rp_np, cfg)
+    verify = None if args.no_verify else Verifier(cfg, rp_np, ci_np, args.rule, dev, rank)
     rp = torch.from_numpy(rp_np).to(dev)
     ci = torch.from_numpy(ci_np).to(dev)
     sym_opts = dict(flags=args.flags, threads_per_row=args.threads_per_row,
                     queue_capacity=args.queue_capacity)
     h = lu.Symbolic(rp, ci, **sym_opts)
+    ms_create = h.stats()["ms_create"]
     cost = lu.row_cost_upper_bound(rp_np)
     bounds = lu.partition_rows(cost, world)
-    rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
     flush = torch.empty(L2_FLUSH_BYTES // 4, dtype=torch.int32, device=dev)
 
     def barrier():
@@ -343,7 +468,7 @@ def run_ours(args, rank, world, local_rank):
 
     state = {}
 
-    def step():
+    def step(rb, re_):
         state.clear()  # let the allocator reuse the previous step's output blocks
         fc = torch.zeros(n, dtype=torch.int32, device=dev)
         h.count(rb, re_, fc)                                     # S3 (symbolic_1)
@@ -357,24 +482,36 @@ def run_ours(args, rank, world, local_rank):
         level, nl = h.levelize(rp_lu, ci_lu, args.rule)          # S8 + S9
         state.update(nnz=nnz, nl=nl, rp_lu=rp_lu, ci_lu=ci_lu, level=level, fc=fc)
 
-    for _ in range(args.warmup):
-        step()
+    rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
+    for _ in range(warmup):
+        step(rb, re_)
     torch.cuda.synchronize()
+    if world > 1 and not args.apriori_partition:
+        # rows are independent (L100), but their cost is not known a priori outside the grids:
+        # re-partition by the per-row cycles measured in one profiled pass of this matrix
+        cyc = lu.measured_row_cost(h, rb, re_, torch.zeros(n, dtype=torch.int32, device=dev))
+        bounds = lu.partition_rows(cyc, world)
+        rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
+        step(rb, re_)
+        torch.cuda.synchronize()
     launches0 = h.stats()["kernel_launches"]
     ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True))
-          for _ in range(args.steps)]
-    k_ms = {"count": [], "scan": [], "emit": [], "levelize": []}
+          for _ in range(steps)]
+    keys = ("count", "tail", "scan", "emit", "levelize")
+    k_ms = {k: [] for k in keys}
     barrier()
     torch.cuda.synchronize()
     with ClockSampler(local_rank) as clk:
-        for k in range(args.steps):
+        for k in range(steps):
             flush.fill_(k)                                   # L2 flush, outside the events
             ev[k][0].record(stream)
-            step()
+            step(rb, re_)
             ev[k][1].record(stream)
             st = h.stats()
-            for key in k_ms:
+            for key in keys:
                 k_ms[key].append(st["ms_" + key])
+            if verify is not None:                           # outside the events
+                verify(state["fc"], state["rp_lu"], state["ci_lu"], state["level"], state["nl"])
         barrier()
         torch.cuda.synchronize()
     launches = h.stats()["kernel_launches"] - launches0
@@ -382,129 +519,179 @@ def run_ours(args, rank, world, local_rank):
     tot = torch.tensor([sum(step_ms)], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(tot, op=dist.ReduceOp.MAX)
-    ms_per_step = float(tot.item()) / args.steps
+    ms_per_step = float(tot.item()) / steps
     nnz = state["nnz"]
-    value = nnz / (ms_per_step / 1e3)
     stats = h.stats()
-    if args.profile:
-        if rank == 0:
-            print(json.dumps({"profile": True, "ms_per_step": ms_per_step, "stats": stats}))
-        return
-
-    # ---- roofline of the dominant kernel (fill2 traversal; events around its launch)
     avg = {k: float(np.mean(v)) for k, v in k_ms.items()}
-    rows_mine = re_ - rb
+
+    # roofline of the dominant kernel: the count pass (fill2 traversal staging every row, plus
+    # the row-merge tail of deferred rows), CUDA events on the launching stream
     frac_rows = cost[rb:re_].sum() / max(cost.sum(), 1)
     te_mine, sv_mine = te * frac_rows, sv * frac_rows
-    # the count pass runs the traversal and stages every row (staged mode), so its algorithmic
-    # bytes are the traversal's plus the pattern it writes; emit is then a placement copy
     staged = stats["pool_bytes"] > 0
-    b_count = alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, staged)
-    b_emit = (8.0 * nnz * frac_rows + 8 * rows_mine) if staged else \
-        alg_bytes_per_pass(te_mine, sv_mine, rows_mine, nnz * frac_rows, True)
+    b_count = alg_bytes_per_pass(te_mine, sv_mine, re_ - rb, nnz * frac_rows, staged)
+    b_emit = (8.0 * nnz * frac_rows + 8 * (re_ - rb)) if staged else \
+        alg_bytes_per_pass(te_mine, sv_mine, re_ - rb, nnz * frac_rows, True)
     dom = "emit" if avg["emit"] >= avg["count"] else "count"
     b_dom = b_emit if dom == "emit" else b_count
-    kname = {"count": "stage" if staged else "count", "emit": "place" if staged else "emit"}[dom]
-    peaks = {}
-    try:
-        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-    except Exception:
-        pass
-    peak = float(peaks.get("hbm_gbs", 6650.0))
+    kname = {"count": "fill2_kernel<stage> (+ k_merge_rows tail)" if staged else
+             "fill2_kernel<count>", "emit": "k_place" if staged else "fill2_kernel<emit>"}[dom]
+    peak, peak_src = peak_hbm()
     achieved = b_dom / (avg[dom] / 1e3) / 1e9
-    traffic = None
-    try:
-        prof = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
-        traffic = prof.get(f"cfg{args.config}", {}).get(
-            f"fill2_{kname}" if kname in ("stage", "count", "emit") else "k_place")
-    except Exception:
-        pass
-    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
-                "frac": achieved / peak, "traffic": traffic,
-                "kernel": f"fill2_kernel<{kname}>" if kname != "place" else "k_place",
-                "peak_source": "MEASURED_PEAKS.json hbm_gbs" if peaks else "fallback",
-                "alg_bytes_per_launch": b_dom, "ms_per_launch": avg[dom]}
+    prof = ncu_profile(cfg) or {}
+    kp = prof.get("fill2_stage" if dom == "count" else "k_place") or {}
+    roofline = {
+        "bound": "issue/LSU",
+        "bound_note": "gathers of A's L2-resident adjacency + shared-memory bit test-and-set: "
+                      "instruction issue and the L1/LSU pipe bind, not DRAM (DESIGN.md §4); "
+                      "frac = algorithmic bytes at ANY cache level (SURVEY 8(d2)) / the HBM copy "
+                      "peak, as the contract defines it",
+        "achieved": achieved, "peak": peak, "unit": "GB/s", "frac": achieved / peak,
+        "peak_source": peak_src, "kernel": kname, "alg_bytes_per_launch": b_dom,
+        "ms_per_launch": avg[dom],
+        "traffic": kp.get("dram_bytes"),
+        "traffic_source": prof.get("_source") if kp else None,
+        "hbm_gbs": (kp["dram_bytes"] / (kp["time_ns"] / 1e9) / 1e9) if kp else None,
+        "hbm_frac": (kp["dram_bytes"] / (kp["time_ns"] / 1e9) / 1e9 / peak) if kp else None,
+        "l2_frac": kp.get("l2_pct") / 100 if kp.get("l2_pct") is not None else None,
+        "sm_issue_frac": kp.get("issue_pct") / 100 if kp.get("issue_pct") is not None else None,
+        "warp_inst_per_sv": (kp["inst_executed"] / kp["sv"]) if kp.get("sv") else None,
+    }
+    rec = {
+        "workload": f"cfg{cfg} {name}", "n": n, "nnz_a": int(rp_np[-1]), "nnz_lu": nnz,
+        "num_levels": state["nl"], "ms_per_step": ms_per_step, "steps": steps, "warmup": warmup,
+        "fill_entries_per_s": nnz / (ms_per_step / 1e3),
+        "symbolic_s": (avg["count"] + avg["scan"] + avg["emit"]) / 1e3,
+        "levelize_s": avg["levelize"] / 1e3,
+        "teps": te / ((avg["count"] + avg["scan"] + avg["emit"]) / 1e3),
+        "traversed_edges_per_pass": te, "scanned_vertices_per_pass": sv,
+        "phases_ms": avg, "ms_create": ms_create,
+        "parity": (verify.what + f" ({verify.checked} checked)") if verify and verify.active
+        else ("rank 0 verifies" if verify else "not verified (--no-verify)"),
+        "roofline": roofline, "gpu_launches": int(launches), "clocks": clk.summary(),
+        "plan": {k: stats[k] for k in ("rows_in_flight", "threads_per_row", "smem_bytes_per_row",
+                                        "visited_in_smem", "ell_width", "queue_capacity",
+                                        "row_classes", "pool_bytes", "rows_retraversed",
+                                        "rows_deferred", "rows_merge_failed", "sample_mean_sv",
+                                        "levelize_wide_levels", "levelize_narrow_levels",
+                                        "spills")},
+    }
+    if world > 1:
+        rec["partition"] = {"bounds": [int(b) for b in bounds],
+                            "by": "a-priori bound row_ptr[i+1]" if args.apriori_partition
+                            else "per-row cycles measured in a profiled pass"}
+    if headline and not args.no_e2e:
+        rec["e2e"] = e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank,
+                         bounds, verify)
+    rec["_state"] = state
+    h.close()
+    return rec
 
-    # ---- e2e through the public API with host buffers
-    e2e = None
-    if not args.no_e2e:
-        rp_h = torch.from_numpy(rp_np).pin_memory()
-        ci_h = torch.from_numpy(ci_np).pin_memory()
-        out_rp = torch.empty(n + 1, dtype=torch.int64).pin_memory()
-        out_ci = torch.empty(nnz, dtype=torch.int32).pin_memory()
-        out_lv = torch.empty(n, dtype=torch.int32).pin_memory()
-        e_ms = []
-        e_phase = {}
-        pipelined = args.e2e_mode == "pipelined" and world == 1
-        for k in range(args.e2e_steps + 1):
-            barrier()
-            torch.cuda.synchronize()
-            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            marks = []
 
-            def mark(tag):
-                ev_ = torch.cuda.Event(enable_timing=True)
-                ev_.record(stream)
-                marks.append((tag, ev_))
-
-            a.record(stream)
-            rpd = rp_h.to(dev, non_blocking=True)
-            cid = ci_h.to(dev, non_blocking=True)
-            mark("h2d")
-            he = lu.Symbolic(rpd, cid, **sym_opts)             # S1 + S2 (validate, plan)
-            mark("create")
-            if pipelined:
-                # S3-S6 with the pattern streamed to pinned host memory behind the traversal
-                fc, rp_lu, ci_lu = he.run_host(nnz, out_rp, out_ci, nchunks=args.e2e_chunks)
-                mark("count+scan+emit+d2h(pattern)")
-                level, _ = he.levelize(rp_lu, ci_lu, args.rule)
-                mark("levelize")
-                out_lv.copy_(level, non_blocking=True)
-            else:
-                fc = torch.zeros(n, dtype=torch.int32, device=dev)
-                he.count(rb, re_, fc)
-                if world > 1:
-                    lu.assemble_counts(fc)
-                mark("count")
-                rp_lu, nz = he.scan(fc)
-                ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)
-                mark("scan+alloc")
-                he.emit(rp_lu, ci_lu, rb, re_)
-                if world > 1:
-                    lu.assemble_pattern(ci_lu, rp_lu, bounds)
-                mark("emit")
-                level, _ = he.levelize(rp_lu, ci_lu, args.rule)
-                mark("levelize")
-                if rank == 0:
-                    out_rp.copy_(rp_lu, non_blocking=True)
-                    out_ci.copy_(ci_lu, non_blocking=True)
-                    out_lv.copy_(level, non_blocking=True)
-            b.record(stream)
-            torch.cuda.synchronize()
-            he.close()
-            if k > 0:
-                e_ms.append(a.elapsed_time(b))
-                prev = a
-                for tag, ev_ in marks + [("d2h", b)]:
-                    e_phase.setdefault(tag, []).append(prev.elapsed_time(ev_))
-                    prev = ev_
-        t = torch.tensor([float(np.mean(e_ms))], dtype=torch.float64, device=dev)
+def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds, verify):
+    """The same metric through the public API with HOST buffers: H2D of A from pinned memory,
+    create (validate, adjacency, plan), count, scan (nnz is now known), allocate the device
+    pattern and the host output buffers, emit, levelize, D2H of row_ptr / col_idx / level.
+    Everything, allocations included, is inside the events; the host result is verified."""
+    import torch
+    import torch.distributed as dist
+    n = len(rp_np) - 1
+    rp_h = torch.from_numpy(rp_np).pin_memory()      # the caller's input, in pinned memory
+    ci_h = torch.from_numpy(ci_np).pin_memory()
+    pinned = args.e2e_host == "pinned"
+    rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
+    e_ms, phases = [], {}
+    for k in range(args.e2e_steps + 1):
         if world > 1:
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e = {"value": nnz / (float(t.item()) / 1e3), "unit": UNIT,
-               "h2d_bytes_per_step": int(rp_np.nbytes + ci_np.nbytes),
-               "d2h_bytes_per_step": int((n + 1) * 8 + nnz * 4 + n * 4) if rank == 0 else 0,
-               "ms_per_step": float(t.item()),
-               "phases_ms": {k: float(np.mean(v)) for k, v in e_phase.items()},
-               "mode": "lu_sym_run_host (chunked count/scan/place, pattern D2H behind the "
-                       "traversal)" if pipelined else "count, scan, alloc, emit, then copies",
-               "includes": "H2D of A, create (validate+adjacency+plan), count, scan, alloc, "
-                           "emit, levelize, D2H of row_ptr/col_idx/level"}
+            dist.barrier()
+        torch.cuda.synchronize()
+        a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        marks = []
 
+        def mark(tag):
+            e_ = torch.cuda.Event(enable_timing=True)
+            e_.record(stream)
+            marks.append((tag, e_))
+
+        a.record(stream)
+        rpd = rp_h.to(dev, non_blocking=True)
+        cid = ci_h.to(dev, non_blocking=True)
+        mark("h2d")
+        he = lu.Symbolic(rpd, cid, **sym_opts)                 # S1 + S2
+        mark("create")
+        fc = torch.zeros(n, dtype=torch.int32, device=dev)
+        he.count(rb, re_, fc)                                  # S3 (+ tail)
+        if world > 1:
+            lu.assemble_counts(fc)
+        rp_lu, nz = he.scan(fc)                                # S4: nnz known on the host
+        mark("count+scan")
+        ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)  # S5
+        out_rp = torch.empty(n + 1, dtype=torch.int64, pin_memory=pinned)
+        out_ci = torch.empty(nz, dtype=torch.int32, pin_memory=pinned)
+        out_lv = torch.empty(n, dtype=torch.int32, pin_memory=pinned)
+        mark("alloc (device + host outputs)")
+        out_rp.copy_(rp_lu, non_blocking=pinned)
+        he.emit(rp_lu, ci_lu, rb, re_)                         # S6
+        if world > 1:
+            lu.assemble_pattern(ci_lu, rp_lu, bounds)
+        mark("emit")
+        out_ci.copy_(ci_lu, non_blocking=pinned)
+        mark("d2h(pattern)")
+        level, _ = he.levelize(rp_lu, ci_lu, args.rule)        # S8 + S9
+        out_lv.copy_(level, non_blocking=pinned)
+        b.record(stream)
+        torch.cuda.synchronize()
+        he.close()
+        if k > 0:
+            e_ms.append(a.elapsed_time(b))
+            prev = a
+            for tag, e_ in marks + [("levelize+d2h(levels)", b)]:
+                phases.setdefault(tag, []).append(prev.elapsed_time(e_))
+                prev = e_
+            if verify is not None:
+                verify.host(out_rp.numpy(), out_ci.numpy(), out_lv.numpy())
+        del out_rp, out_ci, out_lv, ci_lu, rp_lu, fc
+    t = torch.tensor([float(np.mean(e_ms))], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return {"value": nnz / (float(t.item()) / 1e3), "unit": UNIT,
+            "h2d_bytes_per_step": int(rp_np.nbytes + ci_np.nbytes),
+            "d2h_bytes_per_step": int((n + 1) * 8 + nnz * 4 + n * 4) if rank == 0 else 0,
+            "ms_per_step": float(t.item()),
+            "phases_ms": {k: float(np.mean(v)) for k, v in phases.items()},
+            "host_buffers": ("pinned, allocated inside the timed region once nnz is known"
+                             if pinned else "pageable, allocated inside the timed region"),
+            "mode": "two-call protocol: count + scan -> nnz -> allocate -> emit -> copies",
+            "parity": "host copies verified against the reference every step" if verify else None}
+
+
+def run_ours(args, rank, world, local_rank):
+    import torch
+    dev = torch.device("cuda", local_rank)
+    torch.cuda.set_device(dev)
+    head = measure(args, args.config, args.steps, args.warmup, world, rank, local_rank, True)
+    if args.profile:
+        if rank == 0:
+            print(json.dumps({"profile": True, "ms_per_step": head["ms_per_step"]}))
+        return
+    per = {}
+    others = [int(c) for c in args.per_config.split(",") if c.strip()] if args.per_config else []
+    for c in others:
+        if c == args.config:
+            continue
+        r = measure(args, c, args.per_config_steps, args.per_config_warmup, world, rank,
+                    local_rank, False)
+        r.pop("_state")
+        per[f"cfg{c}"] = r
+    state = head.pop("_state")
     if rank != 0:
         return
+    nnz = head["nnz_lu"]
+    n = head["n"]
     cpu = None
     if world == 1 and not args.no_cpu_baseline:
+        name, rp_np, ci_np = gen.config(args.config)
+        te = head["traversed_edges_per_pass"]
         stride = args.cpu_sample_stride or auto_stride(n, te)
         s = cpu_oracle_sample(rp_np, ci_np, stride, te_total=te)
         one = cpu_one_core_rate(rp_np, ci_np, te)
@@ -516,38 +703,41 @@ def run_ours(args, rank, world, local_rank):
         t_lev = time.perf_counter() - t0
         t_cpu = s["t_sym_full"] + t_lev
         cpu = {"value": nnz / t_cpu, "unit": UNIT, "cores": s["threads"], "kind": "oracle",
+               "host": host_cpu(),
                "sample": f"fill2 count+emit on every {stride}-th row ({len(s['rows'])} rows) in "
-                         f"{s['t_sample']:.2f} s, extrapolated by exact TE share "
-                         f"x{s['scale']:.2f}; Kahn levels on the full pattern {t_lev:.2f} s "
+                         f"{s['t_sample']:.2f} s on {s['threads']} threads, extrapolated by exact "
+                         f"TE share x{s['scale']:.2f}; Kahn levels on the full pattern {t_lev:.2f} s "
                          f"(1 thread)",
                "one_core": {"traversed_edges_per_s": one["te_per_s"], "rows": one["rows"],
                             "note": "oracle on 1 thread, count+emit (2 traversals per row)"}}
     out = {
-        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-        "scaling": "strong", "vs_baseline": None, "dtype": "int32", "data": "synthetic",
-        "config": {"workload": f"cfg{args.config} {name}", "n": n, "nnz_a": int(rp_np[-1]),
-                   "nnz_lu": nnz, "num_levels": state["nl"], "rule": args.rule,
-                   "parallelism": f"rows sharded over {world} GPU(s)" if world > 1 else "1 GPU",
-                   "l2": "flushed between timed steps (256 MiB write, outside the events)"},
-        "phases_ms": avg,
-        "symbolic_s": (avg["count"] + avg["scan"] + avg["emit"]) / 1e3,
-        "levelize_s": avg["levelize"] / 1e3,
-        "teps": te / ((avg["count"] + avg["scan"] + avg["emit"]) / 1e3),
-        "traversed_edges_per_pass": te, "scanned_vertices_per_pass": sv,
-        "roofline": roofline,
-        "cpu_baseline": cpu,
-        "e2e": e2e,
-        "gpu_launches": int(launches),
-        "clocks": clk.summary(),
+        "metric": METRIC, "value": head["fill_entries_per_s"], "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": head["ms_per_step"],
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "int32",
+        "data": "synthetic (seeded generators, inputs/gen.py; SURVEY 8(d1))",
+        "config": config_key(args.config, head["n"], head["nnz_a"], nnz, args.rule),
+        "parallelism": f"rows sharded over {world} GPUs (strong scaling)" if world > 1 else "1 GPU",
+        "l2": "flushed between timed steps (256 MiB write, outside the events)",
+        "num_levels": head["num_levels"], "parity": head["parity"],
+        "phases_ms": head["phases_ms"], "ms_create": head["ms_create"],
+        "symbolic_s": head["symbolic_s"], "levelize_s": head["levelize_s"], "teps": head["teps"],
+        "traversed_edges_per_pass": head["traversed_edges_per_pass"],
+        "scanned_vertices_per_pass": head["scanned_vertices_per_pass"],
+        "roofline": head["roofline"], "cpu_baseline": cpu, "e2e": head.get("e2e"),
+        "gpu_launches": head["gpu_launches"], "clocks": head["clocks"], "plan": head["plan"],
+        "per_config": per,
         "numeric": None if (world > 1 or args.no_numeric) else numeric_side(),
-        "plan": {k: stats[k] for k in ("rows_in_flight", "threads_per_row", "smem_bytes_per_row",
-                                        "visited_in_smem", "ell_width", "queue_capacity",
-                                        "row_classes", "pool_bytes", "rows_retraversed",
-                                        "levelize_wide_levels", "levelize_narrow_levels",
-                                        "spills")},
     }
+    if "partition" in head:
+        out["partition"] = head["partition"]
     print(json.dumps(out), flush=True)
+
+
+def config_key(cfg, n, nnz_a, nnz_lu, rule):
+    """The `config` object, identical in both arms."""
+    name = gen.CONFIGS[cfg][0]
+    return {"workload": f"cfg{cfg} {name}", "n": n, "nnz_a": nnz_a, "nnz_lu": nnz_lu,
+            "rule": rule}
 
 
 def main():
@@ -555,8 +745,8 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
-    # test hook: run every rank on one GPU over gloo (exercises the N>1 path where only one GPU
-    # exists); never used for a reported number
+    # test hook: run every rank on one GPU (exercises the N>1 path where only one GPU exists);
+    # never used for a reported number
     if os.environ.get("LUSYM_BENCH_ONE_GPU"):
         local_rank = 0
     if args.impl == "reference":

@@ -23,12 +23,12 @@ from dataclasses import dataclass
 import numpy as np
 import torch
 
-from .parallel import (assemble_counts, assemble_pattern, partition_rows,  # noqa: F401
-                       row_cost_upper_bound)
+from .parallel import (assemble_counts, assemble_pattern, measured_row_cost,  # noqa: F401
+                       partition_rows, row_cost_upper_bound)
 
 __all__ = ["Symbolic", "LuSymError", "levelize", "level_schedule", "load_library", "library_path",
            "partition_rows", "assemble_counts", "assemble_pattern", "symbolic_distributed",
-           "row_cost_upper_bound", "DEP_U", "DEP_GLU3", "numeric_scatter", "numeric_factor",
+           "row_cost_upper_bound", "measured_row_cost", "DEP_U", "DEP_GLU3", "numeric_scatter", "numeric_factor",
            "factorize"]
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
@@ -377,11 +377,17 @@ def numeric_scatter(row_ptr: torch.Tensor, col_idx: torch.Tensor, val: torch.Ten
     fill entries (lu_numeric_scatter).  Returns val_lu float32[nnz_lu] on the device."""
     n = int(row_ptr_lu.numel()) - 1
     nnz_lu = int(col_idx_lu.numel())
+    nnz_a = int(col_idx.numel())
+    if int(row_ptr.numel()) != n + 1:
+        raise ValueError("row_ptr and row_ptr_lu must describe the same n")
+    if int(val.numel()) != nnz_a:
+        raise ValueError(f"val has {val.numel()} entries, A has {nnz_a}")
     val_lu = torch.empty(max(nnz_lu, 1), dtype=torch.float32, device=row_ptr_lu.device)[:nnz_lu]
-    opt = lambda t: ctypes.c_void_p(t.data_ptr()) if t.numel() else None  # noqa: E731
+    opt = lambda t, dt, name: _dev(t, dt, name) if t.numel() else None  # noqa: E731
     _check(load_library().lu_numeric_scatter(
-        n, _dev(row_ptr, torch.int64, "row_ptr"), opt(col_idx), opt(val),
-        _dev(row_ptr_lu, torch.int64, "row_ptr_lu"), opt(col_idx_lu), nnz_lu, opt(val_lu),
+        n, _dev(row_ptr, torch.int64, "row_ptr"), opt(col_idx, torch.int32, "col_idx"),
+        opt(val, torch.float32, "val"), _dev(row_ptr_lu, torch.int64, "row_ptr_lu"),
+        opt(col_idx_lu, torch.int32, "col_idx_lu"), nnz_lu, opt(val_lu, torch.float32, "val_lu"),
         _stream_ptr(stream)))
     return val_lu
 
@@ -394,13 +400,16 @@ def numeric_factor(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, level_ptr
     n = int(row_ptr_lu.numel()) - 1
     if val_lu.dtype != torch.float32 or not val_lu.is_cuda or not val_lu.is_contiguous():
         raise TypeError("val_lu must be a contiguous CUDA float32 tensor")
+    if int(val_lu.numel()) != int(col_idx_lu.numel()):
+        raise ValueError("val_lu and col_idx_lu must have one entry per pattern entry")
+    if int(level_cols.numel()) != n:
+        raise ValueError("level_cols must list the n columns")
     nl = int(level_ptr.numel()) - 1
+    opt = lambda t, dt, name: _dev(t, dt, name) if t.numel() else None  # noqa: E731
     _check(load_library().lu_numeric_factor(
-        n, _dev(row_ptr_lu, torch.int64, "row_ptr_lu"),
-        ctypes.c_void_p(col_idx_lu.data_ptr()) if col_idx_lu.numel() else None,
-        _dev(level_ptr, torch.int64, "level_ptr"),
-        ctypes.c_void_p(level_cols.data_ptr()) if level_cols.numel() else None, nl,
-        ctypes.c_void_p(val_lu.data_ptr()) if val_lu.numel() else None, _stream_ptr(stream)))
+        n, _dev(row_ptr_lu, torch.int64, "row_ptr_lu"), opt(col_idx_lu, torch.int32, "col_idx_lu"),
+        _dev(level_ptr, torch.int64, "level_ptr"), opt(level_cols, torch.int32, "level_cols"), nl,
+        opt(val_lu, torch.float32, "val_lu"), _stream_ptr(stream)))
     return val_lu
 
 

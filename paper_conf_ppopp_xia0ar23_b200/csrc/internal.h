@@ -159,7 +159,12 @@ cudaError_t level_types(int32_t n, const int64_t *rp, const int32_t *ci, const i
                         int32_t num_levels, int32_t min_cols, int32_t max_sub_a, int32_t *type,
                         int64_t *sub, cudaStream_t s);
 cudaError_t level_schedule(int32_t n, const int32_t *level, int32_t num_levels,
-                           int64_t *level_ptr, int32_t *level_cols, cudaStream_t s);
+                           int64_t *level_ptr, int32_t *level_cols, int *h_bad, cudaStream_t s);
+// a level schedule (level_ptr / cols) is a permutation of [0, n) under which every strict entry
+// (i,j) of the pattern has level(min(i,j)) < level(max(i,j)) (the GLU3 rule); *h_bad = 1 if not
+cudaError_t validate_schedule(int32_t n, const int64_t *rp, const int32_t *ci,
+                              const int64_t *level_ptr, int32_t num_levels, const int32_t *cols,
+                              int *h_bad, cudaStream_t s);
 
 // numeric_kernels.cu — Algorithm 2 (numeric LU) on the L+U pattern, SURVEY 8(f4)
 cudaError_t numeric_scatter(int32_t n, const int64_t *rpa, const int32_t *cia, const float *va,

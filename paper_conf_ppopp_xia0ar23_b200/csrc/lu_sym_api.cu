@@ -494,7 +494,10 @@ lu_status plan(lu_sym *h)
         Cfg g;
         if ((st = best_cfg(h, 0, kVisGlobal, smem_optin, &g, 64, 256)) != LU_OK) return st;
         size_t kc = 0;
-        while (g.key >= 0 && kc < h->classes.size() && h->classes[kc].occ < g.occ) ++kc;
+        // candidates: the classes whose shared map holds them below 8 rows per SM
+        while (g.key >= 0 && kc < h->classes.size() && h->classes[kc].occ < 8 &&
+               h->classes[kc].occ < g.occ)
+            ++kc;
         const bool force = getenv("LUSYM_FORCE_SPARSE") != nullptr;  // test knob
         if (force && g.key >= 0) kc = h->classes.size();
         if (kc > 0) {
@@ -510,25 +513,40 @@ lu_status plan(lu_sym *h)
             }
         }
     }
-    // HBM budget: per row in flight, frontier spill (2 x cap) + L staging (cap) + done map
-    // (+ the HBM visited slot); cap = rows of the class (a row's frontier and L part lie below i)
+    // HBM budget: everything the handle allocates stays within scratch_budget_bytes.
+    // Per row in flight: frontier spill (2 x cap) + L staging (cap) + done map (+ the HBM
+    // visited slot); cap = rows of the class (a row's frontier and L part lie below i).  Every
+    // class gets one row in flight, then the rest of the budget goes to the classes in order,
+    // top (heaviest rows) first; classes run concurrently on disjoint regions.
     const bool need_hbm_map = h->classes.front().vis != kVisSmem || h->classes.size() > 1;
+    const uint64_t fixed = (uint64_t)n * 4 + (h->staging ? (uint64_t)n * 12 : 0);
+    std::vector<uint64_t> per_row(h->classes.size());
+    uint64_t min_total = fixed;
+    for (size_t k = 0; k < h->classes.size(); ++k) {
+        RowClass &c = h->classes[k];
+        c.cap = c.hi > 0 ? c.hi : 1;
+        per_row[k] = (uint64_t)(h->staging ? 3 : 2) * c.cap * 4 +
+                     (uint64_t)(need_hbm_map ? 2 : 1) * h->gb_stride * 4;
+        min_total += per_row[k];
+    }
+    const uint64_t used = (uint64_t)h->scratch_bytes;
+    if (budget < used + min_total)
+        return fail(LU_ERR_NOMEM, "scratch budget %llu B < %llu B (adjacency and statistics "
+                    "%llu B + one row in flight per row class %llu B)",
+                    (unsigned long long)budget, (unsigned long long)(used + min_total),
+                    (unsigned long long)used, (unsigned long long)min_total);
+    uint64_t have = budget - used - min_total;
     uint64_t need_spill = 0, need_stg = 0, need_map = 0;
     int max_grid = 0;
-    for (auto &c : h->classes) {
-        const int64_t cap = c.hi > 0 ? c.hi : 1;
-        c.cap = cap;
-        const uint64_t per_row = (uint64_t)(h->staging ? 3 : 2) * cap * 4 +
-                                 (uint64_t)(need_hbm_map ? 2 : 1) * h->gb_stride * 4;
-        const uint64_t fit = budget / per_row;
-        if (fit < 1)
-            return fail(LU_ERR_NOMEM, "scratch budget %llu B < one row's scratch %llu B",
-                        (unsigned long long)budget, (unsigned long long)per_row);
+    for (size_t k = 0; k < h->classes.size(); ++k) {
+        RowClass &c = h->classes[k];
         int64_t grid = (int64_t)sms * c.occ;
         if (h->opts.rows_in_flight > 0 && h->opts.rows_in_flight < grid)
             grid = h->opts.rows_in_flight;
-        if ((uint64_t)grid > fit) grid = (int64_t)fit;
-        c.grid = (int)(grid < 1 ? 1 : grid);
+        const int64_t extra = std::min<int64_t>(grid - 1, (int64_t)(have / per_row[k]));
+        c.grid = (int)(1 + std::max<int64_t>(extra, 0));
+        have -= (uint64_t)(c.grid - 1) * per_row[k];
+        const int64_t cap = c.cap;
         c.spill_off = (int64_t)need_spill;
         c.stg_off = (int64_t)need_stg;
         c.map_off = (int64_t)need_map;
@@ -714,13 +732,22 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
 
 // Extra traversal scratch sets 1..kSets-1 (same sizes as set 0), their class streams and the
 // pipeline's streams; allocated on the first pipelined lu_sym_run_host call.
-lu_status ensure_sets(lu_sym *h)
+lu_status ensure_sets(lu_sym *h, bool *fits)
 {
+    *fits = true;
     if (h->dbitmapS[kSets - 1]) return LU_OK;
     int64_t need_spill = 0, need_stg = 0;
     for (auto &c : h->classes) {
         need_spill = std::max<int64_t>(need_spill, c.spill_off + 2 * c.cap * (int64_t)c.grid);
         need_stg = std::max<int64_t>(need_stg, c.stg_off + c.cap * (int64_t)c.grid);
+    }
+    // the two extra sets must fit the budget too (else lu_sym_run_host runs unpipelined)
+    const uint64_t extra = (uint64_t)(kSets - 1) *
+                           ((uint64_t)need_spill * 4 + (h->staging ? (uint64_t)need_stg * 4 : 0) +
+                            (uint64_t)h->map_words * 4 * (h->gbitmap ? 2 : 1));
+    if ((uint64_t)h->scratch_bytes + extra > h->budget) {
+        *fits = false;
+        return LU_OK;
     }
     lu_status st;
     for (int k = 1; k < kSets; ++k) {
@@ -1188,11 +1215,18 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
     if (nchunks == 0)  // 16 chunks, but none under 4096 rows (each chunk costs a host sync)
         nchunks = std::max(1, std::min(16, n / 4096));
     if (nchunks > n) nchunks = n > 0 ? n : 1;
+    bool sets_fit = true;
     if (h->staging) {
         if ((st = ensure_merge(h)) != LU_OK) return st;
+        if (h->opts.pool_bytes == 0 && !h->pool && h->pool_cap >= 0 && nchunks > 1) {
+            // leave room for the pipeline's two extra scratch sets before the pool takes the rest
+            if ((st = ensure_sets(h, &sets_fit)) != LU_OK) return st;
+        }
         if ((st = ensure_pool(h)) != LU_OK) return st;
     }
-    if (!h->staging || !h->pool || n == 0 || nchunks == 1) {
+    if (sets_fit && h->staging && h->pool && n > 0 && nchunks > 1)
+        if ((st = ensure_sets(h, &sets_fit)) != LU_OK) return st;
+    if (!h->staging || !h->pool || n == 0 || nchunks == 1 || !sets_fit) {
         // one chunk, two-pass mode or no pool: the plain calls, then the copies
         int64_t nnz = 0;
         if ((st = lu_sym_run(h, d_fill_count, d_row_ptr_lu, nullptr, 0, &nnz, stream)) != LU_OK)
@@ -1212,7 +1246,6 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
         CK(cudaStreamSynchronize(s));
         return LU_OK;
     }
-    if ((st = ensure_sets(h)) != LU_OK) return st;
     // row chunks of equal a-priori traversal cost (row_ptr[i+1]: the TE bound of row i, exact on
     // the grids); offsets are chained in increasing row order
     if ((int)h->chunk_bounds.size() != nchunks + 1) {
@@ -1412,7 +1445,9 @@ lu_status lu_level_schedule(int32_t n, const int32_t *d_level, int32_t num_level
         return fail(LU_ERR_ARG, "null pointer");
     if (n > 0 && num_levels < 1) return fail(LU_ERR_ARG, "num_levels must be >= 1 when n > 0");
     cudaStream_t s = (cudaStream_t)stream;
-    CK(level_schedule(n, d_level, num_levels, d_level_ptr, d_level_cols, s));
+    int bad = 0;
+    CK(level_schedule(n, d_level, num_levels, d_level_ptr, d_level_cols, &bad, s));
+    if (bad) return fail(LU_ERR_ARG, "a level is outside [0, num_levels)");
     CK(cudaStreamSynchronize(s));
     return LU_OK;
 }
@@ -1448,6 +1483,17 @@ lu_status lu_numeric_scatter(int32_t n, const int64_t *d_row_ptr_a, const int32_
     if (n < 0 || nnz_lu < 0) return fail(LU_ERR_ARG, "negative size");
     if (n > 0 && (!d_row_ptr_a || !d_row_ptr_lu || (nnz_lu > 0 && (!d_col_idx_lu || !d_val_lu))))
         return fail(LU_ERR_ARG, "null pointer");
+    if (n > 0) {
+        int64_t nnz_a = 0, nnz_p = 0;
+        CK(cudaMemcpyAsync(&nnz_a, d_row_ptr_a + n, sizeof(int64_t), cudaMemcpyDeviceToHost,
+                           (cudaStream_t)stream));
+        CK(cudaMemcpyAsync(&nnz_p, d_row_ptr_lu + n, sizeof(int64_t), cudaMemcpyDeviceToHost,
+                           (cudaStream_t)stream));
+        CK(cudaStreamSynchronize((cudaStream_t)stream));
+        if (nnz_a > 0 && (!d_col_idx_a || !d_val_a)) return fail(LU_ERR_ARG, "null pointer (A)");
+        if (nnz_p != nnz_lu) return fail(LU_ERR_ARG, "nnz_lu %lld != row_ptr_lu[n] %lld",
+                                          (long long)nnz_lu, (long long)nnz_p);
+    }
     int err = 0;
     CK(numeric_scatter(n, d_row_ptr_a, d_col_idx_a, d_val_a, d_row_ptr_lu, d_col_idx_lu, nnz_lu,
                        d_val_lu, &err, (cudaStream_t)stream));
@@ -1473,6 +1519,17 @@ lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_
     if (lp[0] != 0 || lp[num_levels] != n) return fail(LU_ERR_ARG, "level_ptr does not cover n");
     for (int32_t l = 0; l < num_levels; ++l)
         if (lp[l + 1] < lp[l]) return fail(LU_ERR_ARG, "level_ptr not monotone");
+    {
+        // the schedule must be a permutation of the columns under which every GLU3-rule
+        // dependency goes to a later level (a U-rule schedule would race; O(nnz) check)
+        int bad = 0;
+        CK(validate_schedule(n, d_row_ptr_lu, d_col_idx_lu, d_level_ptr, num_levels,
+                             d_level_cols, &bad, s));
+        if (bad)
+            return fail(LU_ERR_ARG, "the level schedule is not a GLU3-rule schedule of this "
+                                    "pattern (a column repeated or out of range, or a strict "
+                                    "entry (i,j) with level(min(i,j)) >= level(max(i,j)))");
+    }
     int dev = 0, sms = 0;
     CK(cudaGetDevice(&dev));
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));

@@ -61,7 +61,79 @@ __global__ void k_level_type(int32_t num_levels, const unsigned long long *lsub,
     if (sub_out) sub_out[l] = sb;
 }
 
+// every level value inside [0, num_levels)
+__global__ void k_check_levels(int32_t n, const int32_t *level, int32_t num_levels, int *bad)
+{
+    const int j = blockIdx.x * blockDim.x + threadIdx.x;
+    if (j < n && (level[j] < 0 || level[j] >= num_levels)) atomicOr(bad, 1);
+}
+
+// schedule -> level of each column; a column listed twice or out of [0, n) is flagged
+__global__ void k_sched_levels(int32_t n, const int64_t *level_ptr, int32_t num_levels,
+                               const int32_t *cols, int32_t *lvl, int *bad)
+{
+    const int64_t q = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (q >= n) return;
+    int lo = 0, hi = num_levels;  // last l with level_ptr[l] <= q
+    while (hi - lo > 1) {
+        const int mid = (lo + hi) >> 1;
+        if (level_ptr[mid] <= q) lo = mid; else hi = mid;
+    }
+    const int c = cols[q];
+    if (c < 0 || c >= n) {
+        atomicOr(bad, 1);
+        return;
+    }
+    if (atomicExch(&lvl[c], lo) != -1) atomicOr(bad, 1);
+}
+
+// every strict entry (i,j) of L+U makes min(i,j) a GLU3-rule predecessor of max(i,j): its
+// level must be lower (one warp per row)
+__global__ void k_sched_edges(int32_t n, const int64_t *rp, const int32_t *ci, const int32_t *lvl,
+                              int *bad)
+{
+    const int64_t w = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+    const int lane = threadIdx.x & 31;
+    if (w >= n) return;
+    const int i = (int)w;
+    const int li = lvl[i];
+    bool ok = li >= 0;
+    for (int64_t p = rp[i] + lane; ok && p < rp[i + 1]; p += 32) {
+        const int j = ci[p];
+        if (j < 0 || j >= n) { ok = false; break; }
+        if (j == i) continue;
+        const int lj = lvl[j];
+        ok = j < i ? lj < li : li < lj;
+    }
+    if (!ok) atomicOr(bad, 1);
+}
+
 }  // namespace
+
+cudaError_t validate_schedule(int32_t n, const int64_t *rp, const int32_t *ci,
+                              const int64_t *level_ptr, int32_t num_levels, const int32_t *cols,
+                              int *h_bad, cudaStream_t s)
+{
+    *h_bad = 0;
+    if (n <= 0) return cudaSuccess;
+    int32_t *lvl = nullptr;
+    int *bad = nullptr;
+    cudaError_t e;
+    if ((e = dev_alloc((void **)&lvl, sizeof(int32_t) * n, s)) != cudaSuccess) return e;
+    if ((e = dev_alloc((void **)&bad, sizeof(int), s)) != cudaSuccess) goto out;
+    if ((e = cudaMemsetAsync(lvl, 0xff, sizeof(int32_t) * n, s)) != cudaSuccess) goto out;
+    if ((e = cudaMemsetAsync(bad, 0, sizeof(int), s)) != cudaSuccess) goto out;
+    k_sched_levels<<<(n + 255) / 256, 256, 0, s>>>(n, level_ptr, num_levels, cols, lvl, bad);
+    k_sched_edges<<<(int)(((int64_t)n * 32 + 255) / 256), 256, 0, s>>>(n, rp, ci, lvl, bad);
+    if ((e = cudaGetLastError()) != cudaSuccess) goto out;
+    if ((e = cudaMemcpyAsync(h_bad, bad, sizeof(int), cudaMemcpyDeviceToHost, s)) != cudaSuccess)
+        goto out;
+    e = cudaStreamSynchronize(s);
+out:
+    dev_free(lvl, s);
+    dev_free(bad, s);
+    return e;
+}
 
 cudaError_t level_types(int32_t n, const int64_t *rp, const int32_t *ci, const int32_t *level,
                         int32_t num_levels, int32_t min_cols, int32_t max_sub_a, int32_t *type,
@@ -90,9 +162,21 @@ out:
 }
 
 cudaError_t level_schedule(int32_t n, const int32_t *level, int32_t num_levels,
-                           int64_t *level_ptr, int32_t *level_cols, cudaStream_t s)
+                           int64_t *level_ptr, int32_t *level_cols, int *h_bad, cudaStream_t s)
 {
+    *h_bad = 0;
     if (n <= 0) return cudaMemsetAsync(level_ptr, 0, sizeof(int64_t) * (num_levels + 1), s);
+    {
+        int *bad = nullptr;
+        cudaError_t e0 = dev_alloc((void **)&bad, sizeof(int), s);
+        if (e0 != cudaSuccess) return e0;
+        cudaMemsetAsync(bad, 0, sizeof(int), s);
+        k_check_levels<<<(n + 255) / 256, 256, 0, s>>>(n, level, num_levels, bad);
+        e0 = cudaMemcpyAsync(h_bad, bad, sizeof(int), cudaMemcpyDeviceToHost, s);
+        if (e0 == cudaSuccess) e0 = cudaStreamSynchronize(s);
+        dev_free(bad, s);
+        if (e0 != cudaSuccess || *h_bad) return e0;
+    }
     int32_t *keys_out = nullptr, *vals_in = nullptr;
     void *tmp = nullptr;
     size_t tmp_bytes = 0;

@@ -176,3 +176,43 @@ def test_coop_without_pair_table(monkeypatch):
     for k, (rp, ci) in enumerate([gen.lap2d(20), gen.circuit(32, 2),
                                   gen.random_pattern(150, 3.0, seed=5, zero_free_diag=True)]):
         check_case(rp, ci, 30 + k, tag=f"no-table {k}")
+
+
+def test_argument_checks():
+    """Bad arguments fail loudly instead of computing garbage or faulting: float64 values, host
+    tensors, wrong lengths, a level schedule that is not a GLU3-rule schedule of the pattern
+    (here the U-rule schedule of an unsymmetric pattern), a repeated column, a level outside
+    [0, num_levels)."""
+    rp, ci = gen.random_pattern(300, 2.5, seed=21, sym_frac=0.2)
+    val = gen.dominant_values(rp, ci, 5, dtype=np.float32)
+    h = lu.Symbolic(t(rp), t(ci))
+    _, rp_lu, ci_lu = h.run()
+    lv_u, nl_u = h.levelize(rp_lu, ci_lu, "u")
+    lv_g, nl_g = h.levelize(rp_lu, ci_lu, "glu3")
+    h.close()
+    with pytest.raises(TypeError):
+        lu.numeric_scatter(t(rp), t(ci), t(val.astype(np.float64)), rp_lu, ci_lu)
+    with pytest.raises(TypeError):
+        lu.numeric_scatter(t(rp), t(ci), torch.from_numpy(val), rp_lu, ci_lu)
+    with pytest.raises(ValueError):
+        lu.numeric_scatter(t(rp), t(ci), t(val[:-1]), rp_lu, ci_lu)
+    v = lu.numeric_scatter(t(rp), t(ci), t(val), rp_lu, ci_lu)
+    ptr_u, cols_u = lu.level_schedule(lv_u, nl_u)
+    ref_u = oracle.levels(rp_lu.cpu().numpy(), ci_lu.cpu().numpy(), "u")
+    ref_g = oracle.levels(rp_lu.cpu().numpy(), ci_lu.cpu().numpy(), "glu3")
+    assert ref_u[1] != ref_g[1] or not np.array_equal(ref_u[0], ref_g[0])
+    with pytest.raises(lu.LuSymError) as e:
+        lu.numeric_factor(rp_lu, ci_lu, ptr_u, cols_u, v.clone())
+    assert e.value.status == lu.LU_ERR_ARG
+    ptr_g, cols_g = lu.level_schedule(lv_g, nl_g)
+    bad = cols_g.clone()
+    bad[1] = bad[0]
+    with pytest.raises(lu.LuSymError) as e:
+        lu.numeric_factor(rp_lu, ci_lu, ptr_g, bad, v.clone())
+    assert e.value.status == lu.LU_ERR_ARG
+    lu.numeric_factor(rp_lu, ci_lu, ptr_g, cols_g, v)    # the GLU3 schedule is accepted
+    lvb = lv_g.clone()
+    lvb[3] = nl_g
+    with pytest.raises(lu.LuSymError) as e:
+        lu.level_schedule(lvb, nl_g)
+    assert e.value.status == lu.LU_ERR_ARG

@@ -576,3 +576,25 @@ def test_sparse_class_forced(monkeypatch, knob):
         g = check(rp, ci, tag=f"sparse {knob}", **knob)
         assert g["stats"]["visited_in_smem"] == 0 and g["stats"]["row_classes"] == 1
         assert g["stats"]["sample_mean_sv"] == 0.0
+
+
+@pytest.mark.parametrize("budget", [2_500_000, 6_000_000, 40_000_000])
+def test_scratch_budget_is_enforced(budget):
+    """Every allocation of the handle (row classes running concurrently, the staging pool, the
+    row-merge tail, lu_sym_run_host's extra scratch sets) stays within scratch_budget_bytes
+    (ADVICE r1); results stay exact."""
+    d = dev()
+    for rp, ci in (gen.lap3d(20), gen.circuit(64, 2), _hub_matrix()):
+        ref = oracle.fill2(rp, ci)
+        nnz = int(ref["row_ptr"][-1])
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d),
+                        scratch_budget_bytes=budget, flags=lu.F_FORCE_CLASSES)
+        fc, rp_lu, ci_lu = h.run()
+        assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
+        hc = torch.empty(nnz, dtype=torch.int32).pin_memory()
+        fc, rp_lu, ci_lu = h.run_host(nnz, None, hc, nchunks=4)
+        torch.cuda.synchronize()
+        assert np.array_equal(hc.numpy(), ref["col_idx"])
+        st = h.stats()
+        assert st["scratch_bytes"] <= budget, (budget, st["scratch_bytes"])
+        h.close()
