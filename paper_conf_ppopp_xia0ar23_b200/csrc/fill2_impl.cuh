@@ -42,6 +42,9 @@ namespace f2 {
 #ifndef LUSYM_VPT  // frontier vertices per thread per round in plain BFS levels (1: scan_level)
 #define LUSYM_VPT 1
 #endif
+#ifndef LUSYM_PRED_TAS  // test_and_mark as predicated straight-line code (shared bitmaps)
+#define LUSYM_PRED_TAS 0
+#endif
 #ifndef LUSYM_TAM  // test_and_mark with one shared bit mask (0: visited() then mark())
 #define LUSYM_TAM 1
 #endif
@@ -203,6 +206,31 @@ __device__ __forceinline__ bool mark(const VisMap<VIS> &m, uint32_t *sm, int v)
 template <int VIS>
 __device__ __forceinline__ bool test_and_mark(const VisMap<VIS> &m, uint32_t *sm, int v)
 {
+#if LUSYM_PRED_TAS
+    if constexpr (VIS == kVisSmem) {
+        // straight-line: a plain shared load (the compiler may batch the W loads of a vertex),
+        // then the atomic and the summary update as predicated instructions — no branch and
+        // no reconvergence barrier per neighbour
+        const uint32_t b = 1u << (v & 31);
+        const int w = v >> 5;
+        const uint32_t a = (uint32_t)phys<VIS>(w) * 4u;
+        uint32_t word;
+        asm("ld.shared.u32 %0, [%1+%2];" : "=r"(word) : "r"(a), "n"(kBmShared));
+        uint32_t old;
+        asm volatile(
+            "{\n\t.reg .pred p, q;\n\t"
+            "setp.eq.u32 p, %2, 0;\n\t"
+            "mov.u32 %0, %3;\n\t"
+            "@p atom.shared.or.b32 %0, [%1+%4], %3;\n\t"
+            "setp.eq.and.u32 q, %0, 0, p;\n\t"
+            "@q red.shared.or.b32 [%5], %6;\n\t}"
+            : "=&r"(old)
+            : "r"(a), "r"(word & b), "r"(b), "n"(kBmShared),
+              "r"(summary_saddr(m) + (uint32_t)(v >> 10) * 4u), "r"(1u << (w & 31))
+            : "memory");
+        return !(old & b);  // visited: old = b
+    }
+#endif
 #if LUSYM_TAM
     const uint32_t b = 1u << (v & 31);
     const int w = v >> 5;

@@ -431,6 +431,16 @@ lu_status plan(lu_sym *h)
                         h->opts.queue_capacity);
         lbw = nw32;  // for splitting below: start from the full map
     }
+    if (const char *e = getenv("LUSYM_TOP_LBW")) {  // A/B knob: split the top class itself
+        const int want = (atoi(e) + 31) / 32 * 32;
+        Cfg c;
+        if (want > 0 && want < nw32 &&
+            (st = best_cfg(h, want, kVisSplit, smem_optin, &c)) == LU_OK && c.key >= 0) {
+            cur = c;
+            vis = kVisSplit;
+            lbw = want;
+        }
+    }
     // lower row classes (Alg. 4): halve the shared part while that adds rows in flight
     h->classes.clear();
     int hi = n;
@@ -1083,7 +1093,9 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
             }
             h->staged.emplace_back(row_begin, row_end);
             // deferred rows need every row below them staged (reading G8)
-            defer = h->defer_win > 0 && h->defer_list && staged_below(h, row_end);
+            // (a row has at most i thresholds, so rows below defer_win cannot be deferred)
+            defer = h->defer_win > 0 && h->defer_list && row_end > h->defer_win &&
+                    staged_below(h, row_end);
         }
     }
     if (defer) CK(cudaMemsetAsync(h->dstats + kSlotDefer, 0, 6 * sizeof(unsigned long long), s));
@@ -1292,7 +1304,7 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
     CK(cudaMemsetAsync(d_row_ptr_lu, 0, sizeof(int64_t), s));
     // rows of the last chunk may be deferred to the row-merge tail (reading G8): it runs once
     // every chunk is traversed, and only the last chunk's scan waits for it
-    const bool defer = h->defer_win > 0 && h->defer_list != nullptr;
+    const bool defer = h->defer_win > 0 && h->defer_list != nullptr && n > h->defer_win;
     h->tail_ran = false;
     if (defer) CK(cudaMemsetAsync(h->dstats + kSlotDefer, 0, 6 * sizeof(unsigned long long), s));
     CK(cudaEventRecord(ev_count[kMaxChunks], s));
