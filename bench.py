@@ -454,8 +454,9 @@ def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
     verify = None if args.no_verify else Verifier(cfg, rp_np, ci_np, args.rule, dev, rank)
     rp = torch.from_numpy(rp_np).to(dev)
     ci = torch.from_numpy(ci_np).to(dev)
-    sym_opts = dict(flags=args.flags, threads_per_row=args.threads_per_row,
-                    queue_capacity=args.queue_capacity)
+    # N > 1: rows deferred on any rank are finished after the pattern exchange (reading G8)
+    sym_opts = dict(flags=args.flags | (lu.F_DEFER_GLOBAL if world > 1 else 0),
+                    threads_per_row=args.threads_per_row, queue_capacity=args.queue_capacity)
     h = lu.Symbolic(rp, ci, **sym_opts)
     ms_create = h.stats()["ms_create"]
     cost = lu.row_cost_upper_bound(rp_np)
@@ -470,16 +471,18 @@ def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
 
     def step(rb, re_):
         state.clear()  # let the allocator reuse the previous step's output blocks
-        fc = torch.zeros(n, dtype=torch.int32, device=dev)
-        h.count(rb, re_, fc)                                     # S3 (symbolic_1)
         if world > 1:
-            lu.assemble_counts(fc)                               # S7 (counts)
-        rp_lu, nnz = h.scan(fc)                                  # S4
-        ci_lu = torch.empty(nnz, dtype=torch.int32, device=dev)  # S5
-        h.emit(rp_lu, ci_lu, rb, re_)                            # S6 (symbolic_2)
-        if world > 1:
-            lu.assemble_pattern(ci_lu, rp_lu, bounds)            # S7 (pattern)
-        level, nl = h.levelize(rp_lu, ci_lu, args.rule)          # S8 + S9
+            # S3 count own rows, S7 all-reduce counts + deferred flags, S4 scan, S5 allocate,
+            # S6 emit own rows, S7 all-gather the pattern, row-merge tail of deferred rows
+            fc, rp_lu, ci_lu = lu.sharded_pass(h, rb, re_, bounds)
+            nnz = int(ci_lu.numel())
+        else:
+            fc = torch.zeros(n, dtype=torch.int32, device=dev)
+            h.count(rb, re_, fc)                                     # S3 (symbolic_1)
+            rp_lu, nnz = h.scan(fc)                                  # S4
+            ci_lu = torch.empty(nnz, dtype=torch.int32, device=dev)  # S5
+            h.emit(rp_lu, ci_lu, rb, re_)                            # S6 (symbolic_2)
+        level, nl = h.levelize(rp_lu, ci_lu, args.rule)              # S8 + S9
         state.update(nnz=nnz, nl=nl, rp_lu=rp_lu, ci_lu=ci_lu, level=level, fc=fc)
 
     rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
@@ -619,22 +622,28 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
         mark("h2d")
         he = lu.Symbolic(rpd, cid, **sym_opts)                 # S1 + S2
         mark("create")
-        fc = torch.zeros(n, dtype=torch.int32, device=dev)
-        he.count(rb, re_, fc)                                  # S3 (+ tail)
         if world > 1:
-            lu.assemble_counts(fc)
-        rp_lu, nz = he.scan(fc)                                # S4: nnz known on the host
-        mark("count+scan")
-        ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)  # S5
-        out_rp = torch.empty(n + 1, dtype=torch.int64, pin_memory=pinned)
-        out_ci = torch.empty(nz, dtype=torch.int32, pin_memory=pinned)
-        out_lv = torch.empty(n, dtype=torch.int32, pin_memory=pinned)
-        mark("alloc (device + host outputs)")
-        out_rp.copy_(rp_lu, non_blocking=pinned)
-        he.emit(rp_lu, ci_lu, rb, re_)                         # S6
-        if world > 1:
-            lu.assemble_pattern(ci_lu, rp_lu, bounds)
-        mark("emit")
+            fc, rp_lu, ci_lu = lu.sharded_pass(he, rb, re_, bounds)
+            nz = int(ci_lu.numel())
+            mark("count+scan+emit+exchange")
+            out_rp = torch.empty(n + 1, dtype=torch.int64, pin_memory=pinned)
+            out_ci = torch.empty(nz, dtype=torch.int32, pin_memory=pinned)
+            out_lv = torch.empty(n, dtype=torch.int32, pin_memory=pinned)
+            mark("alloc (host outputs)")
+            out_rp.copy_(rp_lu, non_blocking=pinned)
+        else:
+            fc = torch.zeros(n, dtype=torch.int32, device=dev)
+            he.count(rb, re_, fc)                                  # S3 (+ tail)
+            rp_lu, nz = he.scan(fc)                                # S4: nnz known on the host
+            mark("count+scan")
+            ci_lu = torch.empty(nz, dtype=torch.int32, device=dev)  # S5
+            out_rp = torch.empty(n + 1, dtype=torch.int64, pin_memory=pinned)
+            out_ci = torch.empty(nz, dtype=torch.int32, pin_memory=pinned)
+            out_lv = torch.empty(n, dtype=torch.int32, pin_memory=pinned)
+            mark("alloc (device + host outputs)")
+            out_rp.copy_(rp_lu, non_blocking=pinned)
+            he.emit(rp_lu, ci_lu, rb, re_)                         # S6
+            mark("emit")
         out_ci.copy_(ci_lu, non_blocking=pinned)
         mark("d2h(pattern)")
         level, _ = he.levelize(rp_lu, ci_lu, args.rule)        # S8 + S9

@@ -97,10 +97,16 @@ enum {
                                     this GPU) + cudaMemPrefetchAsync after each allocation    */
     LU_F_NO_DEFER = 1 << 14,     /* no deferred rows: every row is finished by its fill2
                                     traversal (see lu_sym_opts.defer_windows)                 */
-    LU_F_NO_SPARSE = 1 << 15     /* planner: never replace shared-memory row classes by the
+    LU_F_NO_SPARSE = 1 << 15,    /* planner: never replace shared-memory row classes by the
                                     sparse class (HBM visited slots, 16 rows per SM) that a
                                     create-time sample of rows selects when they visit < n/16
                                     vertices on average (reading G9)              */
+    LU_F_DEFER_GLOBAL = 1 << 16  /* row sharding (reading G8 across GPUs): lu_sym_count may
+                                    defer rows even when the rows below them are counted on
+                                    other GPUs; it then runs no tail: the deferred rows keep
+                                    fill_count 0, lu_sym_deferred_flags reports them, and
+                                    lu_sym_merge_deferred finishes them once the pattern of
+                                    the other rows is assembled                              */
 };
 
 typedef struct {
@@ -141,7 +147,8 @@ typedef struct {
     int32_t rows_in_flight;       /* CTAs (= rows processed concurrently)                    */
     int32_t threads_per_row;
     int32_t smem_bytes_per_row;
-    int32_t visited_in_smem;      /* 1: visited bitmap in shared memory, 0: HBM slots        */
+    int32_t visited_in_smem;      /* top row class: 1 visited bitmap in shared memory, 0 in
+                                     HBM slots, 2 split (part in shared memory, part in HBM) */
     int32_t ell_width;
     int32_t queue_capacity;
     int32_t num_levels;           /* after lu_levelize with this handle                      */
@@ -315,6 +322,28 @@ lu_status lu_numeric_scatter(int32_t n, const int64_t *d_row_ptr_a, const int32_
 lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
                             const int64_t *d_level_ptr, const int32_t *d_level_cols,
                             int32_t num_levels, float *d_val_lu, void *stream);
+
+/*
+ * Row sharding with deferred rows (LU_F_DEFER_GLOBAL; reading G8).
+ *
+ * lu_sym_deferred_flags: d_flags[i] = 1 (int32[n], other entries untouched) for every row the
+ *   last lu_sym_count call on this handle deferred.  The ranks' flags are OR-ed (all-reduced)
+ *   by the caller.
+ *
+ * lu_sym_merge_deferred: finish the flagged rows (d_flags[i] != 0, ascending) by the row-merge
+ *   closure over the complete pattern of every other row, given as the assembled CSR
+ *   d_row_ptr_lu / d_col_idx_lu (rows sorted; flagged rows empty; d_fill_count[i] = their row
+ *   lengths, 0 for flagged rows).  On return d_fill_count[i] holds every row's count,
+ *   d_row_ptr_lu the final offsets and *nnz_lu (host) the final nnz; the handle's staging pool
+ *   holds every row, so a following lu_sym_emit(h, 0, n, d_row_ptr_lu, new array, cap) writes
+ *   the final CSR (the caller allocates it with the new nnz).  Every rank may run it on the
+ *   same inputs: the result is identical.  LU_ERR_NOMEM if the staging pool cannot hold the
+ *   assembled pattern plus n entries per flagged row.  Synchronises.
+ */
+lu_status lu_sym_deferred_flags(lu_sym *h, int32_t *d_flags, void *stream);
+lu_status lu_sym_merge_deferred(lu_sym *h, const int32_t *d_flags, int32_t *d_fill_count,
+                                int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
+                                int64_t *nnz_lu, void *stream);
 
 /* Copy the handle's statistics to *out (host). */
 lu_status lu_sym_get_stats(const lu_sym *h, lu_sym_stats *out);

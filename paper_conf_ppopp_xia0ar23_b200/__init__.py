@@ -42,6 +42,7 @@ F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4
 F_NO_CONTRACT, F_TWO_PASS, F_ONE_CLASS, F_FORCE_CLASSES = 32, 64, 128, 256
 F_SELF_CONT, F_NO_SELF_CONT, F_PAPER_CHUNKS = 512, 1024, 2048
 F_MANAGED, F_MANAGED_PREFETCH, F_NO_DEFER, F_NO_SPARSE = 4096, 8192, 16384, 32768
+F_DEFER_GLOBAL = 65536
 
 
 class LuSymError(RuntimeError):
@@ -88,7 +89,7 @@ EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sy
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
             "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile",
             "lu_level_schedule", "lu_sym_run_host", "lu_level_types", "lu_numeric_scatter",
-            "lu_numeric_factor"]
+            "lu_numeric_factor", "lu_sym_deferred_flags", "lu_sym_merge_deferred"]
 
 
 def library_path() -> str:
@@ -126,6 +127,10 @@ def load_library():
     lib.lu_numeric_factor.argtypes = [I32, P, P, P, P, I32, P, P]
     lib.lu_numeric_factor.restype = I32
     lib.lu_sym_set_row_profile.restype = I32
+    lib.lu_sym_deferred_flags.argtypes = [P, P, P]
+    lib.lu_sym_deferred_flags.restype = I32
+    lib.lu_sym_merge_deferred.argtypes = [P, P, P, P, P, P, P]
+    lib.lu_sym_merge_deferred.restype = I32
     lib.lu_status_str.argtypes = [I32]
     lib.lu_status_str.restype = ctypes.c_char_p
     lib.lu_last_error.restype = ctypes.c_char_p
@@ -284,6 +289,29 @@ class Symbolic:
         self.nnz_lu = int(nnz.value)
         return fc, rp_lu, ci_lu[: self.nnz_lu]
 
+    # -- row sharding with deferred rows (F_DEFER_GLOBAL, reading G8 across GPUs)
+    def deferred_flags(self, flags=None, stream=None):
+        """int32[n] with 1 at the rows the last count deferred (OR-ed into `flags` if given)."""
+        if flags is None:
+            flags = torch.zeros(self.n, dtype=torch.int32, device=self.device)
+        _check(load_library().lu_sym_deferred_flags(
+            self._h, _dev(flags, torch.int32, "flags") if self.n else None, _stream_ptr(stream)))
+        return flags
+
+    def merge_deferred(self, flags, fill_count, row_ptr_lu, col_idx_lu, stream=None):
+        """Finish the flagged rows by row-merge over the assembled pattern of the others
+        (lu_sym_merge_deferred); fill_count and row_ptr_lu are updated in place.  Returns the
+        final nnz; then emit(row_ptr_lu, new array) writes the final CSR."""
+        nnz = ctypes.c_int64(0)
+        _check(load_library().lu_sym_merge_deferred(
+            self._h, _dev(flags, torch.int32, "flags") if self.n else None,
+            _dev(fill_count, torch.int32, "fill_count") if self.n else None,
+            _dev(row_ptr_lu, torch.int64, "row_ptr_lu"),
+            _dev(col_idx_lu, torch.int32, "col_idx_lu") if col_idx_lu.numel() else None,
+            ctypes.byref(nnz), _stream_ptr(stream)))
+        self.nnz_lu = int(nnz.value)
+        return self.nnz_lu
+
     def levelize(self, row_ptr_lu, col_idx_lu, rule: str = "u", level=None, stream=None):
         return levelize(row_ptr_lu, col_idx_lu, rule, level=level, handle=self, stream=stream)
 
@@ -438,33 +466,67 @@ def symbolic_distributed(row_ptr: torch.Tensor, col_idx: torch.Tensor, group=Non
 
     A is replicated; rank r runs fill2 count and emit on its contiguous, cost-balanced row block
     (rows are independent); per-row counts are all-reduced (disjoint supports),
-    every rank scans them, and the pattern blocks are broadcast from their owners (allgatherv),
-    so all ranks end with the identical CSR of L+U; levels are then computed replicated.
+    every rank scans them, and the pattern blocks are all-gathered, so all ranks end with the
+    identical CSR of L+U; levels are then computed replicated.  Rows whose threshold chain is
+    too long are deferred on whichever rank holds them and finished, after the pattern of the
+    other rows is assembled, by the row-merge tail on every rank (F_DEFER_GLOBAL, reading G8).
     output="local_rows" (SURVEY 8(b) LU_OUT_LOCAL_ROWS) skips the pattern exchange: col_idx_lu
     holds only this rank's rows [row_ptr_lu[rb], row_ptr_lu[re]) and no levels are computed
-    (level = num_levels = None; the DAG is global).
+    (level = num_levels = None; the DAG is global; rows are not deferred).
     Returns (fill_count, row_ptr_lu, col_idx_lu, level, num_levels)."""
     if output not in ("replicated", "local_rows"):
         raise ValueError(f"output must be 'replicated' or 'local_rows', got {output!r}")
     import torch.distributed as dist
     world = dist.get_world_size(group) if dist.is_initialized() else 1
     rank = dist.get_rank(group) if dist.is_initialized() else 0
-    h = handle if handle is not None else Symbolic(row_ptr, col_idx, options, stream=stream)
+    if handle is None:
+        options = options or Options()
+        if world > 1 and output == "replicated":
+            options = Options(**{**options.__dict__, "flags": options.flags | F_DEFER_GLOBAL})
+        h = Symbolic(row_ptr, col_idx, options, stream=stream)
+    else:
+        h = handle
     n = h.n
     if cost is None:
         cost = row_cost_upper_bound(row_ptr)
     bounds = partition_rows(cost, world)
     rb, re = int(bounds[rank]), int(bounds[rank + 1])
+    if output == "local_rows":
+        fc = torch.zeros(n, dtype=torch.int32, device=h.device)
+        h.count(rb, re, fc, stream=stream)
+        if world > 1:
+            fc = assemble_counts(fc, group)
+        rp_lu, nnz = h.scan(fc, stream=stream)
+        ci_lu = torch.empty(nnz, dtype=torch.int32, device=h.device)
+        h.emit(rp_lu, ci_lu, rb, re, stream=stream)
+        return fc, rp_lu, ci_lu, None, None
+    fc, rp_lu, ci_lu = sharded_pass(h, rb, re, bounds, group, stream=stream)
+    level, nl = levelize(rp_lu, ci_lu, rule, handle=h, stream=stream)
+    return fc, rp_lu, ci_lu, level, nl
+
+
+def sharded_pass(h: Symbolic, rb: int, re: int, bounds, group=None, stream=None):
+    """One symbolic pass over this rank's rows [rb, re) and the exchange that gives every rank
+    the whole CSR of L+U: count (S3), all-reduce of the counts and of the deferred-row flags
+    (S7), scan (S4), allocate (S5), emit of the own rows (S6), all-gather of the pattern (S7);
+    then, if any rank deferred rows, the row-merge tail over the assembled pattern (replicated
+    on every rank, identical), a rescan and the placement of the final CSR."""
+    import torch.distributed as dist
+    world = dist.get_world_size(group) if dist.is_initialized() else 1
+    n = h.n
     fc = torch.zeros(n, dtype=torch.int32, device=h.device)
     h.count(rb, re, fc, stream=stream)
+    flags = h.deferred_flags(stream=stream)
     if world > 1:
-        fc = assemble_counts(fc, group)
+        assemble_counts(fc, group)
+        assemble_counts(flags, group)
     rp_lu, nnz = h.scan(fc, stream=stream)
     ci_lu = torch.empty(nnz, dtype=torch.int32, device=h.device)
     h.emit(rp_lu, ci_lu, rb, re, stream=stream)
-    if output == "local_rows":
-        return fc, rp_lu, ci_lu, None, None
     if world > 1:
         assemble_pattern(ci_lu, rp_lu, bounds, group)
-    level, nl = levelize(rp_lu, ci_lu, rule, handle=h, stream=stream)
-    return fc, rp_lu, ci_lu, level, nl
+    if int(flags.sum()) > 0:
+        nnz = h.merge_deferred(flags, fc, rp_lu, ci_lu, stream=stream)
+        ci_lu = torch.empty(nnz, dtype=torch.int32, device=h.device)
+        h.emit(rp_lu, ci_lu, 0, n, stream=stream)
+    return fc, rp_lu, ci_lu

@@ -108,11 +108,12 @@ struct VisMap {
     uint32_t *g;  // HBM slot (word index = vertex >> 5)
     int lbw;      // words held in shared memory (kVisSplit)
     int nw;       // shared visited words (the level-1 summary follows them)
+    uint32_t ssum;  // shared address of the level-1 summary (from the runtime window base)
 };
 
 
 template <int VIS>
-__device__ __forceinline__ int phys(int w)
+__device__ __forceinline__ int phys(const VisMap<VIS> &m, int w)
 {
     if (!LUSYM_SWZ) return w;
     return w ^ ((w >> 5) & 31);
@@ -151,22 +152,25 @@ __device__ __forceinline__ uint32_t atom_or_bm(int pw, uint32_t b)
     return old;
 }
 
+// The host probes the window base once per device (fill2_smem_base_ok) and plans only
+// kVisGlobal classes when it is not kDynSmemBase, so this trap is a last-resort assertion.
 __device__ __forceinline__ void check_smem_base(const unsigned char *smem)
 {
     if (threadIdx.x == 0 && (uint32_t)__cvta_generic_to_shared(smem) != kDynSmemBase) __trap();
 }
 
-// shared byte address of the level-1 summary (right after the shared visited words)
+// shared byte address of the level-1 summary (taken from the actual window, so kVisGlobal
+// kernels do not depend on where the dynamic shared memory starts)
 template <int VIS>
 __device__ __forceinline__ uint32_t summary_saddr(const VisMap<VIS> &m)
 {
-    return VIS == kVisGlobal ? kBmShared : kBmShared + 4u * (uint32_t)m.nw;
+    return m.ssum;
 }
 
 template <int VIS>
 __device__ __forceinline__ uint32_t bm_word(const VisMap<VIS> &m, int w)
 {
-    if (in_smem(m, w)) return lds_bm(phys<VIS>(w));
+    if (in_smem(m, w)) return lds_bm(phys<VIS>(m, w));
     return __ldcg(m.g + w);
 }
 
@@ -174,7 +178,7 @@ template <int VIS>
 __device__ __forceinline__ void bm_zero(const VisMap<VIS> &m, int w)
 {
     if (in_smem(m, w))
-        m.s[phys<VIS>(w)] = 0;
+        m.s[phys<VIS>(m, w)] = 0;
     else
         m.g[w] = 0;
 }
@@ -192,7 +196,7 @@ __device__ __forceinline__ bool mark(const VisMap<VIS> &m, uint32_t *sm, int v)
 {
     const uint32_t b = 1u << (v & 31);
     const int w = v >> 5;
-    const uint32_t old = in_smem(m, w) ? atom_or_bm(phys<VIS>(w), b) : atomicOr(m.g + w, b);
+    const uint32_t old = in_smem(m, w) ? atom_or_bm(phys<VIS>(m, w), b) : atomicOr(m.g + w, b);
     if (old == 0)
         asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(summary_saddr(m) + (uint32_t)(v >> 10) * 4u),
                      "r"(1u << (w & 31))
@@ -213,7 +217,7 @@ __device__ __forceinline__ bool test_and_mark(const VisMap<VIS> &m, uint32_t *sm
         // no reconvergence barrier per neighbour
         const uint32_t b = 1u << (v & 31);
         const int w = v >> 5;
-        const uint32_t a = (uint32_t)phys<VIS>(w) * 4u;
+        const uint32_t a = (uint32_t)phys<VIS>(m, w) * 4u;
         uint32_t word;
         asm("ld.shared.u32 %0, [%1+%2];" : "=r"(word) : "r"(a), "n"(kBmShared));
         uint32_t old;
@@ -235,9 +239,9 @@ __device__ __forceinline__ bool test_and_mark(const VisMap<VIS> &m, uint32_t *sm
     const uint32_t b = 1u << (v & 31);
     const int w = v >> 5;
     const bool sh = in_smem(m, w);
-    const uint32_t word = sh ? lds_bm(phys<VIS>(w)) : __ldcg(m.g + w);
+    const uint32_t word = sh ? lds_bm(phys<VIS>(m, w)) : __ldcg(m.g + w);
     if (word & b) return false;
-    const uint32_t old = sh ? atom_or_bm(phys<VIS>(w), b) : atomicOr(m.g + w, b);
+    const uint32_t old = sh ? atom_or_bm(phys<VIS>(m, w), b) : atomicOr(m.g + w, b);
     if (old == 0)
         asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(summary_saddr(m) + (uint32_t)(v >> 10) * 4u),
                      "r"(1u << (w & 31))
@@ -773,6 +777,7 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
         bm.s = reinterpret_cast<uint32_t *>(smem + kHdrBytes);
         sm = bm.s + p.nw;  // p.nw = shared visited words (whole swizzle groups)
     }
+    bm.ssum = (uint32_t)__cvta_generic_to_shared(sm);
     qA = reinterpret_cast<int32_t *>(sm + p.sw);
     qB = qA + p.q;
     const int tid = threadIdx.x, lane = tid & 31;

@@ -2,6 +2,8 @@
 // fill2_nt*.cu instantiate the kernels of fill2_impl.cuh).
 #include "internal.h"
 
+#include <cstdlib>
+
 namespace lusym {
 
 // header | visited words held in shared memory (smem_words, whole swizzle groups) | level-1
@@ -13,6 +15,39 @@ size_t fill2_smem_bytes(int n, int smem_words, int q)
     b += (words + 31) / 32 * sizeof(uint32_t);
     b += (size_t)smem_words * sizeof(uint32_t);
     return (b + 15) & ~(size_t)15;
+}
+
+namespace {
+__global__ void k_smem_base(unsigned *out)
+{
+    extern __shared__ __align__(16) unsigned char smem[];
+    if (threadIdx.x == 0) *out = (unsigned)__cvta_generic_to_shared(smem);
+}
+}  // namespace
+
+// The shared-memory fill2 variants address their visited words at the constant offset
+// 0x400 + kHdrBytes (fill2_impl.cuh kDynSmemBase): probe where a kernel's dynamic shared
+// memory actually starts on this device (once per device); false sends the planner to the
+// kVisGlobal variants, which take every shared address from the runtime window.
+bool fill2_smem_base_ok(int dev)
+{
+    static int cached[64];
+    static bool init[64];
+    if (dev < 0 || dev >= 64) return false;
+    if (getenv("LUSYM_ASSUME_SMEM_BASE_MISMATCH")) return false;  // test knob
+    if (init[dev]) return cached[dev] != 0;
+    unsigned *d = nullptr, h = 0;
+    bool ok = false;
+    if (cudaMalloc(&d, sizeof(unsigned)) == cudaSuccess) {
+        k_smem_base<<<1, 32, 16384>>>(d);
+        if (cudaMemcpy(&h, d, sizeof(unsigned), cudaMemcpyDeviceToHost) == cudaSuccess)
+            ok = h == 0x400u;
+        cudaFree(d);
+    }
+    cudaGetLastError();
+    cached[dev] = ok;
+    init[dev] = true;
+    return ok;
 }
 
 #define LUSYM_NT_SWITCH(FN, ...)                                                             \

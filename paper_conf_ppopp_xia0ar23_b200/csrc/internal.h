@@ -102,6 +102,16 @@ cudaError_t merge_sort_list(int32_t *list, const unsigned long long *cnt, int32_
                             cudaStream_t s);
 cudaError_t merge_launch(const MergeParams &p, int mode, int g, int grid, size_t smem,
                          cudaStream_t s);
+// row sharding with deferred rows (LU_F_DEFER_GLOBAL)
+cudaError_t zero_deferred_counts(const int32_t *list, const unsigned long long *cnt, int32_t max,
+                                 int32_t *fill_count, cudaStream_t s);
+cudaError_t deferred_to_flags(const int32_t *list, const unsigned long long *cnt, int32_t max,
+                              int32_t *flags, cudaStream_t s);
+// row_off / ucut of the assembled CSR (flagged rows: kRowDeferred); list[flag_pos[i]] = i for
+// flagged rows (flag_pos = exclusive prefix sum of flags: ascending)
+cudaError_t prep_merge(int32_t n, const int32_t *flags, const int64_t *rp, const int32_t *ci,
+                       int64_t *row_off, int32_t *ucut, const int64_t *flag_pos, int32_t *list,
+                       cudaStream_t s);
 constexpr int kMergeNT = 1024;
 constexpr int kMergeSortMax = 4096;
 
@@ -118,6 +128,7 @@ cudaError_t dev_alloc(void **p, size_t bytes, cudaStream_t s);
 void dev_free(void *p, cudaStream_t s);
 
 // fill2_kernels.cu (host dispatch; kernels instantiated in fill2_nt*.cu)
+bool fill2_smem_base_ok(int dev);
 size_t fill2_smem_bytes(int n, int smem_words, int q);
 cudaError_t fill2_configure(int nt, int w, int vis, size_t smem);
 cudaError_t fill2_occupancy(int nt, int w, int vis, size_t smem, int *occ);

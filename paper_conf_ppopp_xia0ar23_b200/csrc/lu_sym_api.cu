@@ -156,6 +156,7 @@ struct lu_sym {
     bool merge_smem_bm = true;
     size_t merge_smem = 0;
     bool tail_ran = false;
+    bool deferred_pending = false;  // LU_F_DEFER_GLOBAL count deferred rows, no tail yet
     double sparse_sv = -1;         // planner sample: mean SV per row (-1: not sampled)
 };
 
@@ -417,6 +418,8 @@ lu_status plan(lu_sym *h)
     Cfg cur;
     int vis = kVisGlobal, lbw = 0;
     lu_status st;
+    // the shared-memory variants need the dynamic window at its usual base (fill2_impl.cuh)
+    if (!fill2_smem_base_ok(h->device)) h->opts.flags |= LU_F_GLOBAL_BITMAP;
     if (!(h->opts.flags & LU_F_GLOBAL_BITMAP)) {
         if ((st = best_cfg(h, nw32, kVisSmem, smem_optin, &cur)) != LU_OK) return st;
         if (cur.key >= 0) {
@@ -501,6 +504,9 @@ lu_status plan(lu_sym *h)
     if (!(h->opts.flags & (LU_F_ONE_CLASS | LU_F_GLOBAL_BITMAP | LU_F_FORCE_CLASSES |
                            LU_F_NO_SPARSE)) &&
         h->opts.threads_per_row == 0 && h->opts.queue_capacity == 0) {
+        // (a shared window of 4-64 KB just below each row's own word, the rest in the HBM slot,
+        // measured slower on cfg3 than no shared visited words: 148/153/185 ms against 146 —
+        // the window costs rows per SM, profiles/r02/ab_window.log)
         Cfg g;
         if ((st = best_cfg(h, 0, kVisGlobal, smem_optin, &g, 64, 256)) != LU_OK) return st;
         size_t kc = 0;
@@ -901,11 +907,14 @@ bool staged_below(const lu_sym *h, int32_t row_end)
 // The row-merge tail after a pass that deferred rows: sort the deferred list, finish the rows
 // by closure over the staged rows (k_merge_rows), then let fill2 finish (stage) whatever the
 // tail could not — its list length is read on the device, so no host round trip.
-lu_status run_tail(lu_sym *h, int32_t *fill_count, cudaStream_t s)
+// The row-merge tail over `list` (ascending, *list_cnt rows on the device, at most list_max):
+// finish the rows by closure over the staged rows (k_merge_rows), then let fill2 finish
+// (stage) whatever the tail could not — its list length is read on the device, so no host
+// round trip.  wait / fail_list hold list_max entries (per tail CTA / in total).
+lu_status run_tail_list(lu_sym *h, int32_t *fill_count, const int32_t *list,
+                        unsigned long long *slots, int32_t list_max, int32_t *wait,
+                        int32_t *fail_list, cudaStream_t s)
 {
-    ev_begin(h, kEvTail, s);
-    unsigned long long *slots = h->dstats + kSlotDefer;
-    CK(merge_sort_list(h->defer_list, slots, h->defer_max, s));
     MergeParams mp;
     mp.n = h->n;
     mp.rp = h->rp;
@@ -916,25 +925,36 @@ lu_status run_tail(lu_sym *h, int32_t *fill_count, cudaStream_t s)
     mp.row_off = h->row_off;
     mp.ucut = h->ucut;
     mp.fill_count = fill_count;
-    mp.list = h->defer_list;
+    mp.list = list;
     mp.list_cnt = slots;
-    mp.list_max = h->defer_max;
+    mp.list_max = list_max;
     mp.counter = slots + 1;
     mp.gbitmap = h->mgbitmap;
     mp.gb_stride = ((int64_t)h->n + 31) / 32;
     mp.spill = h->mspill;
     mp.spill_cap = h->n;
-    mp.wait = h->mwait;
-    mp.fail_list = h->fail_list;
+    mp.wait = wait;
+    mp.fail_list = fail_list;
     mp.fail_cnt = slots + 2;
     mp.stats = slots + 3;
     mp.q = h->merge_q;
     CK(merge_launch(mp, h->merge_mode, h->merge_g, h->merge_grid, h->merge_smem, s));
     h->launches += 2;
-    lu_status st = run_pass(h, kStage, 0, h->n, fill_count, nullptr, nullptr, s, h->fail_list, 0,
+    lu_status st = run_pass(h, kStage, 0, h->n, fill_count, nullptr, nullptr, s, fail_list, 0,
                             0, false, slots + 2);
-    ev_end(h, kEvTail, s);
     h->tail_ran = true;
+    return st;
+}
+
+// The tail after a pass that deferred rows (its own list, sorted first).
+lu_status run_tail(lu_sym *h, int32_t *fill_count, cudaStream_t s)
+{
+    ev_begin(h, kEvTail, s);
+    unsigned long long *slots = h->dstats + kSlotDefer;
+    CK(merge_sort_list(h->defer_list, slots, h->defer_max, s));
+    lu_status st = run_tail_list(h, fill_count, h->defer_list, slots, h->defer_max, h->mwait,
+                                 h->fail_list, s);
+    ev_end(h, kEvTail, s);
     return st;
 }
 
@@ -1074,8 +1094,9 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
     h->stream = s;
     ev_begin(h, kEvCount, s);
     int mode = kCount;
-    bool defer = false;
+    bool defer = false, global_defer = false;
     h->tail_ran = false;
+    h->deferred_pending = false;
     if (h->staging) {
         if ((st = ensure_merge(h)) != LU_OK) return st;
         st = ensure_pool(h);
@@ -1092,10 +1113,12 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
                                    s));
             }
             h->staged.emplace_back(row_begin, row_end);
-            // deferred rows need every row below them staged (reading G8)
+            // deferred rows need every row below them staged (reading G8), or the pattern
+            // assembled across GPUs (LU_F_DEFER_GLOBAL: no tail here, lu_sym_merge_deferred)
             // (a row has at most i thresholds, so rows below defer_win cannot be deferred)
+            global_defer = (h->opts.flags & LU_F_DEFER_GLOBAL) != 0;
             defer = h->defer_win > 0 && h->defer_list && row_end > h->defer_win &&
-                    staged_below(h, row_end);
+                    (global_defer || staged_below(h, row_end));
         }
     }
     if (defer) CK(cudaMemsetAsync(h->dstats + kSlotDefer, 0, 6 * sizeof(unsigned long long), s));
@@ -1103,7 +1126,12 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
     h->defer_from = row_begin;
     st = run_pass(h, mode, row_begin, row_end, d_fill_count, nullptr, nullptr, s);
     h->defer_active = false;
-    if (st == LU_OK && defer) st = run_tail(h, d_fill_count, s);
+    if (st == LU_OK && defer && !global_defer) st = run_tail(h, d_fill_count, s);
+    if (defer && global_defer) {  // deferred rows keep count 0 until lu_sym_merge_deferred
+        h->deferred_pending = true;
+        CK(zero_deferred_counts(h->defer_list, h->dstats + kSlotDefer, h->defer_max,
+                                d_fill_count, s));
+    }
     ev_end(h, kEvCount, s);
     return st;
 }
@@ -1554,6 +1582,94 @@ lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_
     return LU_OK;
 }
 
+lu_status lu_sym_deferred_flags(lu_sym *h, int32_t *d_flags, void *stream)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    if (h->n > 0 && !d_flags) return fail(LU_ERR_ARG, "d_flags is NULL");
+    lu_status st = check_device(h);
+    if (st != LU_OK) return st;
+    if (!h->deferred_pending || !h->defer_list) return LU_OK;
+    cudaStream_t s = (cudaStream_t)stream;
+    CK(deferred_to_flags(h->defer_list, h->dstats + kSlotDefer, h->defer_max, d_flags, s));
+    h->launches += 1;
+    return LU_OK;
+}
+
+lu_status lu_sym_merge_deferred(lu_sym *h, const int32_t *d_flags, int32_t *d_fill_count,
+                                int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
+                                int64_t *nnz_lu, void *stream)
+{
+    g_err.clear();
+    if (!h) return fail(LU_ERR_ARG, "handle is NULL");
+    const int32_t n = h->n;
+    if (n > 0 && (!d_flags || !d_fill_count || !d_row_ptr_lu)) return fail(LU_ERR_ARG, "null pointer");
+    lu_status st = check_device(h);
+    if (st != LU_OK) return st;
+    if (!h->staging) return fail(LU_ERR_STATE, "row merge needs the staging pool (not TWO_PASS)");
+    cudaStream_t s = (cudaStream_t)stream;
+    h->stream = s;
+    if ((st = ensure_merge(h)) != LU_OK) return st;
+    if ((st = ensure_pool(h)) != LU_OK) return st;
+    if (!h->pool || !h->defer_list) return fail(LU_ERR_NOMEM, "no staging pool / tail scratch");
+    ev_begin(h, kEvTail, s);
+    int64_t nnz0 = 0;
+    CK(cudaMemcpyAsync(&nnz0, d_row_ptr_lu + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    int64_t *pos = nullptr;
+    int32_t *list = nullptr, *fails = nullptr, *wait = nullptr;
+    CK(dev_alloc((void **)&pos, sizeof(int64_t) * ((size_t)n + 1), s));
+    // flagged rows in ascending order: an exclusive prefix sum of the flags, then a scatter
+    CK(scan_counts(n, d_flags, pos, h->scan_blk, s));
+    int64_t nflag = 0;
+    CK(cudaMemcpyAsync(&nflag, pos + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+    CK(cudaStreamSynchronize(s));
+    if (nnz0 > 0 && !d_col_idx_lu) {
+        dev_free(pos, s);
+        return fail(LU_ERR_ARG, "d_col_idx_lu is NULL");
+    }
+    if ((double)nnz0 + (double)nflag * n > (double)h->pool_cap) {
+        dev_free(pos, s);
+        return fail(LU_ERR_NOMEM, "staging pool (%lld entries) < assembled pattern %lld + %lld "
+                    "deferred rows x n", (long long)h->pool_cap, (long long)nnz0,
+                    (long long)nflag);
+    }
+    const size_t lm = (size_t)std::max<int64_t>(nflag, 1);
+    CK(dev_alloc((void **)&list, sizeof(int32_t) * lm, s));
+    CK(dev_alloc((void **)&fails, sizeof(int32_t) * lm, s));
+    CK(dev_alloc((void **)&wait, sizeof(int32_t) * lm * (size_t)h->merge_grid, s));
+    // the assembled pattern becomes the pool: row t at its CSR offset, deferred rows appended
+    if (nnz0 > 0)
+        CK(cudaMemcpyAsync(h->pool, d_col_idx_lu, sizeof(int32_t) * (size_t)nnz0,
+                           cudaMemcpyDeviceToDevice, s));
+    CK(prep_merge(n, d_flags, d_row_ptr_lu, d_col_idx_lu, h->row_off, h->ucut, pos, list, s));
+    unsigned long long init[6] = {(unsigned long long)nflag, 0, 0, 0, 0, 0};
+    unsigned long long *slots = h->dstats + kSlotDefer;
+    CK(cudaMemcpyAsync(slots, init, sizeof(init), cudaMemcpyHostToDevice, s));
+    unsigned long long cursor = (unsigned long long)nnz0;
+    CK(cudaMemcpyAsync(h->dstats + kSlotPoolCursor, &cursor, sizeof(cursor),
+                       cudaMemcpyHostToDevice, s));
+    CK(cudaMemsetAsync(h->dstats + kSlotUnstaged, 0, sizeof(unsigned long long), s));
+    h->launches += 2;
+    if (nflag > 0)
+        st = run_tail_list(h, d_fill_count, list, slots, (int32_t)nflag, wait, fails, s);
+    if (st == LU_OK) {
+        CK(scan_counts(n, d_fill_count, d_row_ptr_lu, h->scan_blk, s));
+        h->launches += 3;
+        int64_t nnz = 0;
+        CK(cudaMemcpyAsync(&nnz, d_row_ptr_lu + n, sizeof(int64_t), cudaMemcpyDeviceToHost, s));
+        CK(cudaStreamSynchronize(s));
+        h->nnz_lu = nnz;
+        h->stats.nnz_lu = nnz;
+        h->scanned = true;
+        h->staged.assign(1, std::make_pair(0, n));  // the pool holds every row now
+        h->deferred_pending = false;
+        if (nnz_lu) *nnz_lu = nnz;
+    }
+    ev_end(h, kEvTail, s);
+    for (void *b : {(void *)pos, (void *)list, (void *)fails, (void *)wait}) dev_free(b, s);
+    return st;
+}
+
 lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
 {
     g_err.clear();
@@ -1595,7 +1711,7 @@ lu_status lu_sym_get_stats(const lu_sym *hc, lu_sym_stats *out)
     h->stats.rows_in_flight = h->grid;
     h->stats.threads_per_row = h->nt > 1024 ? 1024 : h->nt;
     h->stats.smem_bytes_per_row = (int32_t)h->smem;
-    h->stats.visited_in_smem = h->gb ? 0 : 1;
+    h->stats.visited_in_smem = h->gb ? 0 : (h->vis == kVisSmem ? 1 : 2);
     h->stats.row_classes = (int32_t)h->classes.size();
     h->stats.ell_width = h->w;
     h->stats.queue_capacity = h->q;

@@ -471,6 +471,44 @@ __global__ void __launch_bounds__(1024) k_sort_list(int32_t *list, const unsigne
     for (int k = threadIdx.x; k < m; k += blockDim.x) list[k] = a[k];
 }
 
+// ---- row sharding with deferred rows (LU_F_DEFER_GLOBAL)
+__global__ void k_list_to_flags(const int32_t *list, const unsigned long long *cnt, int32_t max,
+                                int32_t *flags, int32_t *fill_count, int32_t value)
+{
+    const int k = blockIdx.x * blockDim.x + threadIdx.x;
+    if (k >= (int)min(*cnt, (unsigned long long)max)) return;
+    if (flags) flags[list[k]] = value;
+    if (fill_count) fill_count[list[k]] = 0;
+}
+
+// the assembled CSR as the tail's pool: row_off = row_ptr (kRowDeferred for flagged rows),
+// ucut = entries <= i of row i (binary search in the sorted row)
+__global__ void k_prep_merge(int32_t n, const int32_t *flags, const int64_t *rp, const int32_t *ci,
+                             int64_t *row_off, int32_t *ucut)
+{
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i >= n) return;
+    if (flags[i]) {
+        row_off[i] = kRowDeferred;
+        return;
+    }
+    int64_t lo = rp[i], hi = rp[i + 1];
+    const int64_t b = lo;
+    while (lo < hi) {
+        const int64_t mid = (lo + hi) >> 1;
+        if (ci[mid] <= i) lo = mid + 1; else hi = mid;
+    }
+    row_off[i] = b;
+    ucut[i] = (int32_t)(lo - b);
+}
+
+__global__ void k_scatter_flagged(int32_t n, const int32_t *flags, const int64_t *pos,
+                                  int32_t *list)
+{
+    const int i = blockIdx.x * blockDim.x + threadIdx.x;
+    if (i < n && flags[i]) list[pos[i]] = i;
+}
+
 int cluster_shift(int n, int g)
 {
     const int nw = (n + 31) / 32;
@@ -518,6 +556,30 @@ cudaError_t merge_max_clusters(int g, size_t smem, int *clusters)
     cfg.attrs = attr;
     cfg.numAttrs = 1;
     return cudaOccupancyMaxActiveClusters(clusters, (const void *)k_merge_rows<2>, &cfg);
+}
+
+cudaError_t zero_deferred_counts(const int32_t *list, const unsigned long long *cnt, int32_t max,
+                                 int32_t *fill_count, cudaStream_t s)
+{
+    k_list_to_flags<<<(max + 255) / 256, 256, 0, s>>>(list, cnt, max, nullptr, fill_count, 0);
+    return cudaGetLastError();
+}
+
+cudaError_t deferred_to_flags(const int32_t *list, const unsigned long long *cnt, int32_t max,
+                              int32_t *flags, cudaStream_t s)
+{
+    k_list_to_flags<<<(max + 255) / 256, 256, 0, s>>>(list, cnt, max, flags, nullptr, 1);
+    return cudaGetLastError();
+}
+
+cudaError_t prep_merge(int32_t n, const int32_t *flags, const int64_t *rp, const int32_t *ci,
+                       int64_t *row_off, int32_t *ucut, const int64_t *flag_pos, int32_t *list,
+                       cudaStream_t s)
+{
+    if (n <= 0) return cudaSuccess;
+    k_prep_merge<<<(n + 255) / 256, 256, 0, s>>>(n, flags, rp, ci, row_off, ucut);
+    k_scatter_flagged<<<(n + 255) / 256, 256, 0, s>>>(n, flags, flag_pos, list);
+    return cudaGetLastError();
 }
 
 cudaError_t merge_sort_list(int32_t *list, const unsigned long long *cnt, int32_t max,

@@ -102,7 +102,8 @@ __global__ void k_collect_unstaged(int32_t rb, int32_t re, const int64_t *row_of
                                    int32_t *list, unsigned long long *cnt)
 {
     const int64_t r = rb + (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-    const bool un = r < re && row_off[r] < 0;
+    // (a row deferred across GPUs, kRowDeferred, is empty until lu_sym_merge_deferred)
+    const bool un = r < re && row_off[r] < 0 && row_off[r] != kRowDeferred;
     const unsigned b = __ballot_sync(0xffffffffu, un);
     if (!b) return;
     const int lane = threadIdx.x & 31, leader = __ffs(b) - 1;

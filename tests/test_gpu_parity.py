@@ -568,13 +568,14 @@ def test_deferred_rows_run_host(nchunks):
 @pytest.mark.parametrize("knob", [dict(), dict(defer_windows=1), dict(queue_capacity=0, rows_in_flight=5),
                                   dict(flags=lu.F_TWO_PASS)], ids=str)
 def test_sparse_class_forced(monkeypatch, knob):
-    """The planner's sparse class (reading G9: HBM visited slots, 128-thread CTAs) replacing
-    every shared-memory class, forced on small inputs; bit-exact."""
+    """The planner's sparse class (reading G9: 64-thread CTAs at 32 rows per SM, visited words
+    in an HBM slot) replacing every shared-memory class, forced on small inputs; bit-exact."""
     monkeypatch.setenv("LUSYM_FORCE_SPARSE", "1")
     for rp, ci in (gen.lap3d(9), gen.circuit(48, 2), _hub_matrix(), gen.lap2d(20),
                    gen.random_pattern(700, 2.5, seed=9)):
         g = check(rp, ci, tag=f"sparse {knob}", **knob)
-        assert g["stats"]["visited_in_smem"] == 0 and g["stats"]["row_classes"] == 1
+        assert g["stats"]["visited_in_smem"] == 0
+        assert g["stats"]["row_classes"] == 1
         assert g["stats"]["sample_mean_sv"] == 0.0
 
 
@@ -597,4 +598,59 @@ def test_scratch_budget_is_enforced(budget):
         assert np.array_equal(hc.numpy(), ref["col_idx"])
         st = h.stats()
         assert st["scratch_bytes"] <= budget, (budget, st["scratch_bytes"])
+        h.close()
+
+
+def test_smem_base_fallback(monkeypatch):
+    """If a kernel's dynamic shared memory did not start at the base the shared-bitmap kernels
+    assume, the planner falls back to the HBM-bitmap kernels (no trap); forced here."""
+    monkeypatch.setenv("LUSYM_ASSUME_SMEM_BASE_MISMATCH", "1")
+    for rp, ci in (gen.lap3d(9), gen.circuit(40, 2), _hub_matrix()):
+        g = check(rp, ci, tag="smem-base-fallback")
+        assert g["stats"]["visited_in_smem"] == 0
+
+
+@pytest.mark.parametrize("defer_windows", [1, 3, 0])
+def test_deferred_rows_across_shards(defer_windows):
+    """Reading G8 across GPUs (F_DEFER_GLOBAL), two "ranks" simulated by two handles in one
+    process: each counts its block deferring rows whose rows below live on the other handle,
+    counts and flags are summed (all-reduce), the pattern of the other rows is assembled, then
+    lu_sym_merge_deferred finishes the deferred rows on either handle; bit-exact."""
+    d = dev()
+    for rp, ci in (_hub_matrix(), _hub_matrix(n=4000, hubs=9, deg=1500, seed=3),
+                   gen.circuit(48, 3), gen.lap3d(9)):
+        ref = oracle.fill2(rp, ci)
+        n = len(rp) - 1
+        A = (torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+        hs = [lu.Symbolic(*A, flags=lu.F_DEFER_GLOBAL, defer_windows=defer_windows)
+              for _ in range(2)]
+        b = [0, n // 2, n]
+        fc = torch.zeros(n, dtype=torch.int32, device=d)
+        flags = torch.zeros(n, dtype=torch.int32, device=d)
+        for r in range(2):
+            part = torch.zeros(n, dtype=torch.int32, device=d)
+            hs[r].count(b[r], b[r + 1], part)
+            fc += part
+            flags |= hs[r].deferred_flags()
+        rp_lu, nnz = hs[0].scan(fc)
+        hs[1].scan(fc)
+        ci_lu = torch.zeros(nnz, dtype=torch.int32, device=d)
+        for r in range(2):
+            hs[r].emit(rp_lu, ci_lu, b[r], b[r + 1])
+        if defer_windows:
+            assert int(flags.sum()) > 0
+        for r in (1, 0):       # either handle finishes the same rows identically
+            fcr, rpr = fc.clone(), rp_lu.clone()
+            nnz2 = hs[r].merge_deferred(flags, fcr, rpr, ci_lu)
+            assert nnz2 == int(ref["row_ptr"][-1])
+            out = hs[r].emit(rpr, torch.empty(nnz2, dtype=torch.int32, device=d))
+            assert np.array_equal(fcr.cpu().numpy(), ref["counts"])
+            assert np.array_equal(rpr.cpu().numpy(), ref["row_ptr"])
+            assert np.array_equal(out.cpu().numpy(), ref["col_idx"])
+        for h in hs:
+            h.close()
+        # the one-process form of the same protocol
+        h = lu.Symbolic(*A, flags=lu.F_DEFER_GLOBAL, defer_windows=defer_windows)
+        fc, rp_lu, ci_lu = lu.sharded_pass(h, 0, n, [0, n])
+        assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
         h.close()
