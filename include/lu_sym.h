@@ -324,6 +324,24 @@ lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_
                             int32_t num_levels, float *d_val_lu, void *stream);
 
 /*
+ * lu_numeric_factor_ex: the same with the storage mode of As chosen (§3.4):
+ *   LU_NUMERIC_SPARSE: As(i,k) located in the sorted row by rank / binary search (Alg. 6) —
+ *                      what lu_numeric_factor does (one cooperative launch for all levels);
+ *   LU_NUMERIC_DENSE:  GLU3.0's dense format: the target row of each update expanded into a
+ *                      dense n-long position map, so As(i,k) is addressed directly; each
+ *                      concurrent CTA needs n ints, so at most M = L / (n sizeof) of them
+ *                      (L352), L = half the free HBM; one launch per level;
+ *   LU_NUMERIC_AUTO:   the paper's switch (L372): dense iff n <= L / (TB_max sizeof(float)),
+ *                      TB_max = SMs x resident CTAs per SM; else sparse.
+ * The results agree up to the float rounding order of the atomic updates.
+ */
+enum { LU_NUMERIC_AUTO = 0, LU_NUMERIC_DENSE = 1, LU_NUMERIC_SPARSE = 2 };
+lu_status lu_numeric_factor_ex(int32_t n, const int64_t *d_row_ptr_lu,
+                               const int32_t *d_col_idx_lu, const int64_t *d_level_ptr,
+                               const int32_t *d_level_cols, int32_t num_levels, int32_t mode,
+                               float *d_val_lu, void *stream);
+
+/*
  * Row sharding with deferred rows (LU_F_DEFER_GLOBAL; reading G8).
  *
  * lu_sym_deferred_flags: d_flags[i] = 1 (int32[n], other entries untouched) for every row the

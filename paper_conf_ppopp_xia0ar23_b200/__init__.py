@@ -89,7 +89,8 @@ EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sy
             "lu_sym_scan", "lu_sym_emit", "lu_sym_run", "lu_levelize", "lu_sym_get_stats",
             "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile",
             "lu_level_schedule", "lu_sym_run_host", "lu_level_types", "lu_numeric_scatter",
-            "lu_numeric_factor", "lu_sym_deferred_flags", "lu_sym_merge_deferred"]
+            "lu_numeric_factor", "lu_sym_deferred_flags", "lu_sym_merge_deferred",
+            "lu_numeric_factor_ex"]
 
 
 def library_path() -> str:
@@ -126,6 +127,8 @@ def load_library():
     lib.lu_numeric_scatter.restype = I32
     lib.lu_numeric_factor.argtypes = [I32, P, P, P, P, I32, P, P]
     lib.lu_numeric_factor.restype = I32
+    lib.lu_numeric_factor_ex.argtypes = [I32, P, P, P, P, I32, I32, P, P]
+    lib.lu_numeric_factor_ex.restype = I32
     lib.lu_sym_set_row_profile.restype = I32
     lib.lu_sym_deferred_flags.argtypes = [P, P, P]
     lib.lu_sym_deferred_flags.restype = I32
@@ -420,8 +423,12 @@ def numeric_scatter(row_ptr: torch.Tensor, col_idx: torch.Tensor, val: torch.Ten
     return val_lu
 
 
+NUMERIC_AUTO, NUMERIC_DENSE, NUMERIC_SPARSE = 0, 1, 2
+
+
 def numeric_factor(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, level_ptr: torch.Tensor,
-                   level_cols: torch.Tensor, val_lu: torch.Tensor, stream=None):
+                   level_cols: torch.Tensor, val_lu: torch.Tensor, stream=None,
+                   mode: str = "sparse"):
     """Algorithm 2 (L165-204) in place on val_lu (float32, CSR of L+U), level by level over a
     schedule of GLU3-rule levels (lu_numeric_factor): L strictly below, U on and above the
     diagonal.  Returns val_lu."""
@@ -434,15 +441,16 @@ def numeric_factor(row_ptr_lu: torch.Tensor, col_idx_lu: torch.Tensor, level_ptr
         raise ValueError("level_cols must list the n columns")
     nl = int(level_ptr.numel()) - 1
     opt = lambda t, dt, name: _dev(t, dt, name) if t.numel() else None  # noqa: E731
-    _check(load_library().lu_numeric_factor(
+    m = {"auto": NUMERIC_AUTO, "dense": NUMERIC_DENSE, "sparse": NUMERIC_SPARSE}[mode]
+    _check(load_library().lu_numeric_factor_ex(
         n, _dev(row_ptr_lu, torch.int64, "row_ptr_lu"), opt(col_idx_lu, torch.int32, "col_idx_lu"),
         _dev(level_ptr, torch.int64, "level_ptr"), opt(level_cols, torch.int32, "level_cols"), nl,
-        opt(val_lu, torch.float32, "val_lu"), _stream_ptr(stream)))
+        m, opt(val_lu, torch.float32, "val_lu"), _stream_ptr(stream)))
     return val_lu
 
 
 def factorize(row_ptr: torch.Tensor, col_idx: torch.Tensor, val: torch.Tensor,
-              options: Options | None = None, stream=None):
+              options: Options | None = None, stream=None, mode: str = "sparse"):
     """End to end on this GPU: symbolic (fill2, Alg. 1/3), GLU3-rule levels (Alg. 5), the
     level schedule and the numeric phase (Alg. 2).  Returns (row_ptr_lu, col_idx_lu, val_lu,
     level_ptr, level_cols)."""
@@ -455,7 +463,7 @@ def factorize(row_ptr: torch.Tensor, col_idx: torch.Tensor, val: torch.Tensor,
     level_ptr, level_cols = level_schedule(level, max(nl, 1) if level.numel() else 0,
                                            stream=stream)
     val_lu = numeric_scatter(row_ptr, col_idx, val, rp_lu, ci_lu, stream=stream)
-    numeric_factor(rp_lu, ci_lu, level_ptr, level_cols, val_lu, stream=stream)
+    numeric_factor(rp_lu, ci_lu, level_ptr, level_cols, val_lu, stream=stream, mode=mode)
     return rp_lu, ci_lu, val_lu, level_ptr, level_cols
 
 

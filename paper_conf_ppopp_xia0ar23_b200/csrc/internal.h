@@ -185,7 +185,7 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
                            const int64_t *h_level_ptr, const int64_t *level_ptr_d,
                            const int32_t *level_cols,
                            int32_t num_levels, int32_t num_sms, float *val, int *h_err,
-                           cudaStream_t s);
+                           cudaStream_t s, int dense_ctas = 0);
 
 // levelize_kernels.cu
 struct LevelizeScratch {

@@ -1545,7 +1545,18 @@ lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_
                             const int64_t *d_level_ptr, const int32_t *d_level_cols,
                             int32_t num_levels, float *d_val_lu, void *stream)
 {
+    return lu_numeric_factor_ex(n, d_row_ptr_lu, d_col_idx_lu, d_level_ptr, d_level_cols,
+                                num_levels, LU_NUMERIC_SPARSE, d_val_lu, stream);
+}
+
+lu_status lu_numeric_factor_ex(int32_t n, const int64_t *d_row_ptr_lu,
+                               const int32_t *d_col_idx_lu, const int64_t *d_level_ptr,
+                               const int32_t *d_level_cols, int32_t num_levels, int32_t mode,
+                               float *d_val_lu, void *stream)
+{
     g_err.clear();
+    if (mode != LU_NUMERIC_AUTO && mode != LU_NUMERIC_DENSE && mode != LU_NUMERIC_SPARSE)
+        return fail(LU_ERR_ARG, "mode %d", mode);
     if (n < 0 || num_levels < 0) return fail(LU_ERR_ARG, "negative size");
     if (n == 0) return LU_OK;
     if (num_levels < 1) return fail(LU_ERR_ARG, "num_levels must be >= 1 when n > 0");
@@ -1570,13 +1581,27 @@ lu_status lu_numeric_factor(int32_t n, const int64_t *d_row_ptr_lu, const int32_
                                     "pattern (a column repeated or out of range, or a strict "
                                     "entry (i,j) with level(min(i,j)) >= level(max(i,j)))");
     }
-    int dev = 0, sms = 0;
+    int dev = 0, sms = 0, bpsm = 0;
     CK(cudaGetDevice(&dev));
     CK(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+    CK(cudaDeviceGetAttribute(&bpsm, cudaDevAttrMaxBlocksPerMultiprocessor, dev));
+    // GLU3.0's dense column format needs an n-long map per concurrent CTA: at most
+    // M = L / (n sizeof) CTAs (L352).  The paper switches to the sparse format (Alg. 6) when
+    // n > L / (TB_max sizeof) (L372), L = device memory (here: free HBM), TB_max = resident CTAs.
+    int dense_ctas = 0;
+    if (mode != LU_NUMERIC_SPARSE) {
+        size_t free_b = 0, total_b = 0;
+        CK(cudaMemGetInfo(&free_b, &total_b));
+        const double L = 0.5 * (double)free_b;
+        const double tb_max = (double)sms * bpsm;
+        const bool dense = mode == LU_NUMERIC_DENSE || (double)n <= L / (tb_max * sizeof(float));
+        const double m = L / ((double)n * sizeof(int32_t));
+        if (dense) dense_ctas = (int)std::max(1.0, std::min(m, (double)sms * 8));
+    }
     int err = 0;
     CK(numeric_factor(n, d_row_ptr_lu, d_col_idx_lu, lp.data(), d_level_ptr, d_level_cols,
                       num_levels, sms,
-                      d_val_lu, &err, s));
+                      d_val_lu, &err, s, dense_ctas));
     if (err & 1) return fail(LU_ERR_INPUT, "zero pivot");
     if (err) return fail(LU_ERR_INPUT, "update outside the L+U pattern");
     return LU_OK;

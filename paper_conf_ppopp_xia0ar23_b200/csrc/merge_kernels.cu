@@ -356,10 +356,9 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
                 }
                 __syncthreads();
             }
-            if (tid == 0) {
-                h.cnt[cur] = 0;
-                ++n_rounds;
-            }
+            // (fsize > 0: the loop's barriers ordered every read of h.cnt[cur] before this)
+            if (tid == 0 && fsize) h.cnt[cur] = 0;
+            if (tid == 0) ++n_rounds;
             __syncthreads();
             cur = nxt;
         }

@@ -321,6 +321,62 @@ __global__ void k_pair_table(int64_t total, int32_t n, const int64_t *__restrict
     }
 }
 
+// GLU3.0's dense column format (reading R33): the target row i of an update
+// is expanded into a dense n-long map of its positions (D[k] = position of As(i,k)), so each
+// As(i,k) is addressed directly instead of searched (Alg. 6).  One (column j, L entry (i,j))
+// item per CTA at a time; the map is an n-int slot per CTA, which is what caps the concurrent
+// CTAs at M = L / (n * sizeof) (L352) — the memory limit the sparse mode removes.
+__global__ void __launch_bounds__(256) k_update_level_dense(
+    int32_t pos0, int32_t pos1, int64_t total, const int64_t *__restrict__ WL,
+    const int32_t *__restrict__ cols, const int64_t *__restrict__ rp,
+    const int32_t *__restrict__ ci, const int64_t *__restrict__ dpos,
+    const int64_t *__restrict__ cptr, const int32_t *__restrict__ lrow,
+    const int64_t *__restrict__ lpos, int32_t n, int32_t *dense, float *val, int *err)
+{
+    int32_t *D = dense + (size_t)blockIdx.x * n;
+    const int64_t wbase = WL[pos0];
+    for (int64_t t = blockIdx.x; t < total; t += gridDim.x) {
+        const int64_t g = wbase + t;
+        int lo = pos0, hi = pos1 - 1;  // last pos with WL[pos] <= g
+        while (lo < hi) {
+            const int mid = (lo + hi + 1) >> 1;
+            if (__ldg(WL + mid) <= g) lo = mid; else hi = mid - 1;
+        }
+        const int j = __ldg(cols + lo);
+        const int64_t e = __ldg(cptr + j) + (g - __ldg(WL + lo));
+        const int i = __ldg(lrow + e);
+        const int64_t pij = __ldg(lpos + e), iend = __ldg(rp + i + 1);
+        const int64_t dp = __ldg(dpos + j), jend = __ldg(rp + j + 1);
+        for (int64_t p = pij + 1 + threadIdx.x; p < iend; p += blockDim.x) D[__ldg(ci + p)] = (int32_t)p;
+        __syncthreads();
+        if (dp >= 0) {
+            const float l = val[pij], d = val[dp];
+            for (int64_t q = dp + 1 + threadIdx.x; q < jend; q += blockDim.x) {
+                const int32_t p = D[__ldg(ci + q)];
+                if (p < 0) atomicOr(err, kErrPattern);
+                else atomicAdd(val + p, -l * (val[q] / d));
+            }
+        }
+        __syncthreads();
+        for (int64_t p = pij + 1 + threadIdx.x; p < iend; p += blockDim.x) D[__ldg(ci + p)] = -1;
+        __syncthreads();
+    }
+}
+
+// strict-L entry counts of the columns in schedule order (for the dense mode's item scan)
+__global__ void k_lcount_sched(int32_t n, const int32_t *cols, const int64_t *dpos,
+                               const int64_t *cptr, int64_t *cnt)
+{
+    const int pos = blockIdx.x * blockDim.x + threadIdx.x;
+    if (pos > n) return;
+    if (pos == n) {
+        cnt[n] = 0;
+        return;
+    }
+    const int j = cols[pos];
+    cnt[pos] = dpos[j] < 0 ? 0 : cptr[j + 1] - cptr[j];
+}
+
 // lines 2-6 for every column at once (each column's strict-L entries and pivot are final once
 // its level has run), and the pivot check of every column: warp per row i
 __global__ void k_divide(int32_t n, const int64_t *rp, const int32_t *ci, const int64_t *dpos,
@@ -366,7 +422,7 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
                            const int64_t *h_level_ptr, const int64_t *level_ptr_d,
                            const int32_t *level_cols,
                            int32_t num_levels, int32_t num_sms, float *val, int *h_err,
-                           cudaStream_t s)
+                           cudaStream_t s, int dense_ctas)
 {
     *h_err = 0;
     if (n <= 0) return cudaSuccess;
@@ -417,6 +473,34 @@ cudaError_t numeric_factor(int32_t n, const int64_t *rp, const int32_t *ci,
     hW.resize(n + 1);
     NK(cudaMemcpyAsync(hW.data(), W, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, s));
     NK(cudaStreamSynchronize(s));
+    if (dense_ctas > 0) {
+        // dense column format (L350-356): items = the levels' L entries in schedule order,
+        // one launch per level, dense_ctas CTAs each with an n-int position map
+        int64_t *WL = nullptr, *lc = nullptr;
+        int32_t *dense = nullptr;
+        std::vector<int64_t> hWL((size_t)n + 1);
+        NK(dev_alloc((void **)&WL, sizeof(int64_t) * (n + 1), s));
+        NK(dev_alloc((void **)&lc, sizeof(int64_t) * (n + 1), s));
+        NK(dev_alloc((void **)&dense, sizeof(int32_t) * (size_t)n * dense_ctas, s));
+        NK(cudaMemsetAsync(dense, 0xff, sizeof(int32_t) * (size_t)n * dense_ctas, s));
+        k_lcount_sched<<<(n + 256) / 256, 256, 0, s>>>(n, level_cols, dpos, cptr, lc);
+        NK(cub::DeviceScan::ExclusiveSum(tmp, tmp2_bytes, lc, WL, n + 1, s));
+        NK(cudaMemcpyAsync(hWL.data(), WL, sizeof(int64_t) * (n + 1), cudaMemcpyDeviceToHost, s));
+        NK(cudaStreamSynchronize(s));
+        for (int32_t l = 0; l < num_levels; ++l) {
+            const int32_t p0 = (int32_t)h_level_ptr[l], p1 = (int32_t)h_level_ptr[l + 1];
+            const int64_t total = hWL[p1] - hWL[p0];
+            if (p1 <= p0 || total <= 0 || hW[p1] == hW[p0]) continue;
+            const int grid = (int)(total < dense_ctas ? total : dense_ctas);
+            k_update_level_dense<<<grid, 256, 0, s>>>(p0, p1, total, WL, level_cols, rp, ci, dpos,
+                                                      cptr, lrow, lpos, n, dense, val, err);
+        }
+        NK(cudaGetLastError());
+        NK(cudaStreamSynchronize(s));
+        dev_free(WL, s);
+        dev_free(lc, s);
+        dev_free(dense, s);
+    } else
     // levels in order (L206-208): one cooperative launch with a grid barrier per level, or
     // (LUSYM_NUMERIC_LAUNCH_PER_LEVEL=1, or no co-residency) one launch per level with a grid
     // sized to the level's pairs

@@ -48,8 +48,8 @@ def split_lu(rp, ci, v, n):
     return L, U
 
 
-def gpu_factor(rp, ci, val32):
-    rp_lu, ci_lu, val_lu, lptr, lcols = lu.factorize(t(rp), t(ci), t(val32))
+def gpu_factor(rp, ci, val32, mode="sparse"):
+    rp_lu, ci_lu, val_lu, lptr, lcols = lu.factorize(t(rp), t(ci), t(val32), mode=mode)
     torch.cuda.synchronize()
     return rp_lu.cpu().numpy(), ci_lu.cpu().numpy(), val_lu.cpu().numpy().astype(np.float64)
 
@@ -67,10 +67,10 @@ def check_backward(rp, ci, val32, rp_lu, ci_lu, g):
         f"backward error above 4ku|L||U| (max excess {viol.data.max():.3e})"
 
 
-def check_case(rp, ci, seed, tag="", with_oracle=True):
+def check_case(rp, ci, seed, tag="", with_oracle=True, mode="sparse"):
     n = len(rp) - 1
     val32 = gen.dominant_values(rp, ci, seed, dtype=np.float32)
-    rp_lu, ci_lu, g = gpu_factor(rp, ci, val32)
+    rp_lu, ci_lu, g = gpu_factor(rp, ci, val32, mode)
     check_backward(rp, ci, val32, rp_lu, ci_lu, g)
     if not with_oracle:
         return
@@ -216,3 +216,24 @@ def test_argument_checks():
     with pytest.raises(lu.LuSymError) as e:
         lu.level_schedule(lvb, nl_g)
     assert e.value.status == lu.LU_ERR_ARG
+
+
+@pytest.mark.parametrize("mode", ["dense", "auto"])
+def test_dense_column_mode(mode):
+    """GLU3.0's dense column format and the paper's dense/sparse switch
+    (L372, "auto": on one B200 every size here is dense) against the same forward / backward
+    bars as the sparse (Alg. 6) mode."""
+    rng = np.random.default_rng(88)
+    for case in range(12):
+        n = int(rng.integers(1, 160))
+        rp, ci = gen.random_pattern(n, float(rng.uniform(0.5, 4)), seed=9100 + case,
+                                    zero_free_diag=True, sym_frac=float(rng.uniform(0, 1)))
+        check_case(rp, ci, case, tag=f"{mode} random {case}", mode=mode)
+    for name, (rp, ci) in (("lap2d24", gen.lap2d(24)), ("lap3d8", gen.lap3d(8)),
+                           ("circuit", gen.circuit(32, 3)), ("arrow_first", gen.arrow_first(300)),
+                           ("band", gen.band(400, 5)), ("one", gen.diag_only(1))):
+        check_case(rp, ci, 5, tag=f"{mode} {name}", mode=mode)
+    check_case(*gen.lap3d(16), 11, tag=f"{mode} lap3d16", with_oracle=False, mode=mode)
+    with pytest.raises(lu.LuSymError):     # zero pivot
+        gpu_factor(np.array([0, 2, 4], dtype=np.int64), np.array([0, 1, 0, 1], dtype=np.int32),
+                   np.array([0.0, 1.0, 1.0, 1.0], dtype=np.float32), mode)
