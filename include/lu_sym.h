@@ -139,8 +139,10 @@ typedef struct {
     double ms_create;             /* validate + adjacency build + planning                  */
     double ms_count, ms_scan, ms_emit, ms_levelize; /* last call of each (device events)     */
     int64_t nnz_lu;               /* after lu_sym_scan                                       */
-    int64_t edges_read_count;     /* entries read from A's CSR (seed rows, heavy vertices),  */
-    int64_t edges_read_emit;      /*   last count / emit pass; ELL reads are not counted     */
+    int64_t edges_read_count;     /* entries read from A's CSR (seed rows and heavy rows,    */
+    int64_t edges_read_emit;      /*   last count / emit pass) — ELL reads of light rows are
+                                     not counted; the method's traversed edges TE (R24) come
+                                     from the oracle / closed forms (tests/golden)           */
     int64_t vertices_scanned_count, vertices_scanned_emit;
     int64_t spills;               /* frontier entries that spilled from smem to HBM          */
     int64_t scratch_bytes;        /* HBM scratch owned by the handle                         */
@@ -167,6 +169,8 @@ typedef struct {
     int64_t merge_waits;          /* ... members that were deferred rows still in progress   */
     double sample_mean_sv;        /* planner: mean vertices scanned per sampled row (reading
                                      G9); -1 if create did not sample                        */
+    int64_t heavy_rows;           /* rows of off-diagonal degree > ell_width, scanned by a
+                                     whole warp from A's CSR instead of one ELL load         */
 } lu_sym_stats;
 
 typedef struct lu_sym lu_sym;

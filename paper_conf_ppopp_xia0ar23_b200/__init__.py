@@ -79,7 +79,8 @@ class _Stats(ctypes.Structure):
                 ("kernel_launches", ctypes.c_int64), ("rows_deferred", ctypes.c_int64),
                 ("rows_merge_failed", ctypes.c_int64), ("merge_entries_read", ctypes.c_int64),
                 ("ms_tail", ctypes.c_double), ("merge_rounds", ctypes.c_int64),
-                ("merge_waits", ctypes.c_int64), ("sample_mean_sv", ctypes.c_double)]
+                ("merge_waits", ctypes.c_int64), ("sample_mean_sv", ctypes.c_double),
+                ("heavy_rows", ctypes.c_int64)]
 
 
 _lib = None

@@ -30,9 +30,6 @@
 namespace lusym {
 namespace f2 {
 
-#ifndef LUSYM_SWZ
-#define LUSYM_SWZ 1
-#endif
 #ifndef LUSYM_BATCH_TEST  // scan_level: load every neighbour's visited word before any atomic
 #define LUSYM_BATCH_TEST 0    // (A/B on B200: 3.7% slower on cfg2, 5% on cfg5 — kept as a knob)
 #endif
@@ -44,6 +41,9 @@ namespace f2 {
 #endif
 #ifndef LUSYM_PRED_TAS  // test_and_mark as predicated straight-line code (shared bitmaps)
 #define LUSYM_PRED_TAS 0
+#endif
+#ifndef LUSYM_ENC_ELL  // BFS of shared-map kernels reads neighbours pre-encoded as shared
+#define LUSYM_ENC_ELL 1    // bitmap addresses (enc_slot), decoding only newly visited ones
 #endif
 #ifndef LUSYM_TAM  // test_and_mark with one shared bit mask (0: visited() then mark())
 #define LUSYM_TAM 1
@@ -251,6 +251,41 @@ __device__ __forceinline__ bool test_and_mark(const VisMap<VIS> &m, uint32_t *sm
 #else
     return !visited(m, v) && mark(m, sm, v);
 #endif
+}
+
+// Encoded neighbour of the shared-map kernels (built by k_build_ell_enc): e = phys(v >> 5) << 7
+// | (v & 31).  e >> 5 is the byte offset of v's visited word (phys << 2 exactly: the bit index
+// shifts out), and a funnel shift by e uses only its low 5 bits, the bit of v — so the common
+// visited test is one shift, one shared load and one bit test; only a newly visited neighbour
+// is decoded back to v (the swizzle is an involution on the word index).
+__device__ __forceinline__ int dec_slot(int e)
+{
+    int pw = e >> 7;
+    if (LUSYM_SWZ) pw ^= (pw >> 5) & 31;
+    return (pw << 5) | (e & 31);
+}
+
+// test-and-set of the encoded neighbour e (kVisSmem): true iff this call set the bit; *v = the
+// decoded vertex when true
+template <int VIS>
+__device__ __forceinline__ bool test_and_mark_enc(const VisMap<VIS> &m, int e, int *v)
+{
+    const uint32_t off = (uint32_t)e >> 5;
+    uint32_t word;
+    asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(word) : "r"(off), "n"(kBmShared) : "memory");
+    const uint32_t b = 1u << (e & 31);
+    if (word & b) return false;
+    uint32_t old;
+    asm volatile("atom.shared.or.b32 %0, [%1+%2], %3;"
+                 : "=r"(old) : "r"(off), "n"(kBmShared), "r"(b) : "memory");
+    if (old & b) return false;
+    const int x = dec_slot(e);
+    *v = x;
+    if (old == 0)
+        asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(summary_saddr(m) + (uint32_t)(x >> 10) * 4u),
+                     "r"(1u << ((x >> 5) & 31))
+                     : "memory");
+    return true;
 }
 
 // ELL slots W in {4, 6, 8}; rows are stored 4 (W = 4) or 8 (W = 6, 8) entries wide.  A light
@@ -483,10 +518,31 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
         // one warp-aggregated append (a grid vertex has up to three neighbours further from
         // the BFS source); further ones (rare) are appended one by one
         int c = 0, f0 = 0, f1 = 0, f2 = 0;
+        const bool enc = LUSYM_ENC_ELL && VIS == kVisSmem && p.elle != nullptr;
         if (valid) {
-            load_nb<W>(p.ell, f, nb);
+            load_nb<W>(enc ? p.elle : p.ell, f, nb);
             heavy = nb[0] == kHeavy;
-            if (!heavy) {
+            if (enc && !heavy) {
+#pragma unroll
+                for (int s = 0; s < W; ++s) {
+                    int w;
+                    if (test_and_mark_enc(bm, nb[s], &w)) {
+                        if (w < t0) {
+                            if (c == 3) {
+                                put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
+                            } else {
+                                f2 = f1;
+                                f1 = f0;
+                                f0 = w;
+                                ++c;
+                            }
+                        } else if (w > i) {
+                            ++a.ucnt;
+                            a.lmax = max(a.lmax, w);
+                        }
+                    }
+                }
+            } else if (!heavy) {
                 // all W visited words first (independent loads in flight together), then the
                 // test-and-set only on the slots that looked unvisited (the atomic decides)
                 uint32_t um = 0;

@@ -5,6 +5,12 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+// XOR swizzle of the shared visited words inside groups of 32 (fill2_impl.cuh phys); the host
+// needs it too, for the encoded adjacency (encode_ell)
+#ifndef LUSYM_SWZ
+#define LUSYM_SWZ 1
+#endif
+
 namespace lusym {
 
 // Traversal adjacency entry marking a vertex whose off-diagonal degree exceeds the ELL width:
@@ -20,6 +26,8 @@ struct Fill2Params {
     const int64_t *rp;        // A row_ptr [n+1]
     const int32_t *ci;        // A col_idx
     const int32_t *ell;       // traversal adjacency, n x W int32 (16 B aligned)
+    const int32_t *elle;      // ... the same with light neighbours encoded (enc_slot) for the
+                              // shared-map kernels' BFS, or null
     int32_t row_begin, row_end;
     int32_t descending;       // 1: heaviest (largest id) first
     int32_t *fill_count;      // count pass
@@ -149,6 +157,10 @@ cudaError_t count_light(int32_t n, const int64_t *rp, const int32_t *ci, int w,
                         unsigned long long *d_cnt, cudaStream_t s);
 cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, int32_t *ell,
                       cudaStream_t s);
+// the encoded copy for the shared-map kernels: light slots v -> phys(v >> 5) << 7 | (v & 31)
+// (phys = the XOR swizzle of fill2_impl.cuh when swz), heavy records unchanged
+cudaError_t encode_ell(int32_t n, int w, bool swz, const int32_t *ell, int32_t *elle,
+                       cudaStream_t s);
 // row_ptr[0..n] = exclusive prefix sum of counts[0..n); chained: offsets start at the value
 // row_ptr[0] holds on entry (a row block continuing an earlier one), else at 0
 cudaError_t scan_counts(int32_t n, const int32_t *counts, int64_t *row_ptr, int64_t *blk,

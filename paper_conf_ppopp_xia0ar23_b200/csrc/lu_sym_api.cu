@@ -2,6 +2,8 @@
 #include "lu_sym.h"
 #include "internal.h"
 
+#include <nvtx3/nvtx3.hpp>  // header-only: a named range per ABI call (for nsys / ncu)
+
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -93,6 +95,7 @@ struct lu_sym {
     int device = 0;
     // traversal adjacency
     int32_t *ell = nullptr;
+    int32_t *elle = nullptr;  // encoded copy (shared-map BFS), n <= 2^21 only
     int w = 8;
     // plan
     bool gb = false;
@@ -222,7 +225,7 @@ lu_status salloc(lu_sym *h, T **p, size_t elems)
 void free_handle(lu_sym *h)
 {
     cudaStream_t s = h->stream;
-    void *bufs[] = {h->ell,        h->gbitmap,   h->dbitmap, h->gspill, h->dstats,
+    void *bufs[] = {h->ell,        h->elle,      h->gbitmap, h->dbitmap, h->gspill, h->dstats,
                     h->scan_blk,   h->dbad,      h->stg,     h->pool,   h->row_off,
                     h->unstaged,   h->ucut,      h->defer_list, h->fail_list, h->mspill,
                     h->mwait,      h->mgbitmap};
@@ -359,6 +362,7 @@ lu_status sample_mean_sv(lu_sym *h, const RowClass &c, int32_t lo, int32_t hi, i
     p.rp = h->rp;
     p.ci = h->ci;
     p.ell = h->ell;
+    p.elle = h->elle;
     p.descending = 1;
     p.fill_count = fc;
     p.rp_lu = nullptr;
@@ -654,6 +658,7 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     p.rp = h->rp;
     p.ci = h->ci;
     p.ell = h->ell;
+    p.elle = h->elle;
     p.descending = (h->opts.flags & LU_F_ASCENDING) ? 0 : 1;
     p.fill_count = fill_count;
     p.rp_lu = rp_lu;
@@ -991,6 +996,7 @@ const char *lu_last_error(void) { return g_err.c_str(); }
 lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d_row_ptr,
                         const int32_t *d_col_idx, const lu_sym_opts *opts, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_sym_create"};
     g_err.clear();
     if (!out) return fail(LU_ERR_ARG, "out is NULL");
     *out = nullptr;
@@ -1065,6 +1071,22 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
         if ((st = dalloc(h, &h->ell, (size_t)n * (w <= 4 ? 4 : 8))) != LU_OK) return bail(st);
         cudaError_t e = build_ell(n, d_row_ptr, d_col_idx, w, h->ell, s);
         if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
+        {  // rows scanned by a whole warp from A's CSR (off-diagonal degree > W)
+            unsigned long long light = 0;
+            e = count_light(n, d_row_ptr, d_col_idx, w, h->dstats + 15, s);
+            if (e == cudaSuccess)
+                e = cudaMemcpyAsync(&light, h->dstats + 15, 8, cudaMemcpyDeviceToHost, s);
+            if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+            if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
+            h->stats.heavy_rows = n - (int64_t)light;
+        }
+        // the encoded copy read by the shared-map kernels' BFS (only n whose bitmap can fit
+        // shared memory can have such classes)
+        if (n <= (1 << 21)) {
+            if ((st = dalloc(h, &h->elle, (size_t)n * (w <= 4 ? 4 : 8))) != LU_OK) return bail(st);
+            e = encode_ell(n, w, LUSYM_SWZ != 0, h->ell, h->elle, s);
+            if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
+        }
     }
     if ((st = plan(h)) != LU_OK) return bail(st);
     cudaEventRecord(t1, s);
@@ -1082,6 +1104,7 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
 lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d_fill_count,
                        void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_sym_count"};
     g_err.clear();
     if (!h) return fail(LU_ERR_ARG, "handle is NULL");
     if (row_begin < 0 || row_end > h->n || row_begin > row_end)
@@ -1139,6 +1162,7 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
 lu_status lu_sym_scan(lu_sym *h, const int32_t *d_fill_count, int64_t *d_row_ptr_lu,
                       int64_t *nnz_lu, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_sym_scan"};
     g_err.clear();
     if (!h) return fail(LU_ERR_ARG, "handle is NULL");
     if (!d_row_ptr_lu || (h->n > 0 && !d_fill_count))
@@ -1164,6 +1188,7 @@ lu_status lu_sym_scan(lu_sym *h, const int32_t *d_fill_count, int64_t *d_row_ptr
 lu_status lu_sym_emit(lu_sym *h, int32_t row_begin, int32_t row_end, const int64_t *d_row_ptr_lu,
                       int32_t *d_col_idx_lu, int64_t cap, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_sym_emit"};
     g_err.clear();
     if (!h) return fail(LU_ERR_ARG, "handle is NULL");
     if (row_begin < 0 || row_end > h->n || row_begin > row_end)
@@ -1240,6 +1265,7 @@ lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
                           int64_t *h_row_ptr_lu, int32_t *h_col_idx_lu, int64_t *nnz_lu,
                           void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_sym_run_host"};
     g_err.clear();
     if (!h) return fail(LU_ERR_ARG, "handle is NULL");
     if (nchunks < 0 || nchunks > kMaxChunks)
@@ -1438,6 +1464,7 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
                       const int32_t *d_col_idx_lu, int32_t dep_rule, int32_t *d_level,
                       int32_t *num_levels, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_levelize"};
     g_err.clear();
     if (n < 0) return fail(LU_ERR_ARG, "n < 0");
     if (dep_rule != LU_DEP_U && dep_rule != LU_DEP_GLU3)
@@ -1479,6 +1506,7 @@ lu_status lu_levelize(lu_sym *h, int32_t n, const int64_t *d_row_ptr_lu,
 lu_status lu_level_schedule(int32_t n, const int32_t *d_level, int32_t num_levels,
                             int64_t *d_level_ptr, int32_t *d_level_cols, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_level_schedule"};
     g_err.clear();
     if (n < 0 || num_levels < 0) return fail(LU_ERR_ARG, "negative size");
     if (!d_level_ptr || (n > 0 && (!d_level || !d_level_cols)))
@@ -1496,6 +1524,7 @@ lu_status lu_level_types(int32_t n, const int64_t *d_row_ptr_lu, const int32_t *
                          const int32_t *d_level, int32_t num_levels, int32_t min_cols,
                          int32_t max_sub_a, int32_t *d_type, int64_t *d_sub, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_level_types"};
     g_err.clear();
     if (n < 0 || num_levels < 0) return fail(LU_ERR_ARG, "negative size");
     if (n > 0 && num_levels < 1) return fail(LU_ERR_ARG, "num_levels must be >= 1 when n > 0");
@@ -1519,6 +1548,7 @@ lu_status lu_numeric_scatter(int32_t n, const int64_t *d_row_ptr_a, const int32_
                              const int32_t *d_col_idx_lu, int64_t nnz_lu, float *d_val_lu,
                              void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_numeric_scatter"};
     g_err.clear();
     if (n < 0 || nnz_lu < 0) return fail(LU_ERR_ARG, "negative size");
     if (n > 0 && (!d_row_ptr_a || !d_row_ptr_lu || (nnz_lu > 0 && (!d_col_idx_lu || !d_val_lu))))
@@ -1554,6 +1584,7 @@ lu_status lu_numeric_factor_ex(int32_t n, const int64_t *d_row_ptr_lu,
                                const int32_t *d_level_cols, int32_t num_levels, int32_t mode,
                                float *d_val_lu, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_numeric_factor_ex"};
     g_err.clear();
     if (mode != LU_NUMERIC_AUTO && mode != LU_NUMERIC_DENSE && mode != LU_NUMERIC_SPARSE)
         return fail(LU_ERR_ARG, "mode %d", mode);
@@ -1609,6 +1640,7 @@ lu_status lu_numeric_factor_ex(int32_t n, const int64_t *d_row_ptr_lu,
 
 lu_status lu_sym_deferred_flags(lu_sym *h, int32_t *d_flags, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_sym_deferred_flags"};
     g_err.clear();
     if (!h) return fail(LU_ERR_ARG, "handle is NULL");
     if (h->n > 0 && !d_flags) return fail(LU_ERR_ARG, "d_flags is NULL");
@@ -1625,6 +1657,7 @@ lu_status lu_sym_merge_deferred(lu_sym *h, const int32_t *d_flags, int32_t *d_fi
                                 int64_t *d_row_ptr_lu, const int32_t *d_col_idx_lu,
                                 int64_t *nnz_lu, void *stream)
 {
+    nvtx3::scoped_range nvtx_range{"lu_sym_merge_deferred"};
     g_err.clear();
     if (!h) return fail(LU_ERR_ARG, "handle is NULL");
     const int32_t n = h->n;

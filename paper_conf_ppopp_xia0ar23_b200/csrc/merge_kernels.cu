@@ -212,7 +212,9 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
         csync_impl(CL);
         if constexpr (CL) {
             if (tid == 0 && bm.rank != 0) h.row = cg::this_cluster().map_shared_rank(&h, 0)->row;
-            __syncthreads();
+            // no CTA may exit (on the final claim, -1) while another still reads its shared
+            // memory: a second barrier after the read of rank 0's claim
+            cg::this_cluster().sync();
         }
         const int i = h.row;
         if (i < 0) break;

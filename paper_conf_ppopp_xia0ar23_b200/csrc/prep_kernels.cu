@@ -111,6 +111,25 @@ __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int
     if constexpr (S == 8) dst[1] = make_int4(out[4], out[5], out[6], out[7]);
 }
 
+// shared-map encoding of the light ELL slots (fill2_impl.cuh enc_slot / dec_slot)
+__global__ void k_encode_ell(int64_t total, int stride, bool swz, const int32_t *ell,
+                             int32_t *elle)
+{
+    for (int64_t k = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; k < total;
+         k += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t row = k / stride;
+        const int32_t head = ell[row * stride];
+        const int32_t v = ell[k];
+        if (head == kHeavy || v < 0) {
+            elle[k] = v;
+        } else {
+            int w = v >> 5;
+            if (swz) w ^= (w >> 5) & 31;
+            elle[k] = (w << 7) | (v & 31);
+        }
+    }
+}
+
 // entries (i, j) of rows i < bound with j >= bound: pattern marks a split map sends to HBM
 __global__ void k_count_far(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
                             unsigned long long *cnt)
@@ -242,6 +261,18 @@ cudaError_t build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int w, in
         k_build_ell<6><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
     else
         k_build_ell<8><<<(n + 255) / 256, 256, 0, s>>>(n, rp, ci, ell);
+    return cudaGetLastError();
+}
+
+cudaError_t encode_ell(int32_t n, int w, bool swz, const int32_t *ell, int32_t *elle,
+                       cudaStream_t s)
+{
+    const int stride = w <= 4 ? 4 : 8;
+    const int64_t total = (int64_t)n * stride;
+    if (total == 0) return cudaSuccess;
+    const int64_t blocks = (total + 255) / 256;
+    k_encode_ell<<<(int)(blocks < 4096 ? blocks : 4096), 256, 0, s>>>(total, stride, swz, ell,
+                                                                       elle);
     return cudaGetLastError();
 }
 
