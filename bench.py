@@ -602,7 +602,6 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
     rp_h = torch.from_numpy(rp_np).pin_memory()      # the caller's input, in pinned memory
     ci_h = torch.from_numpy(ci_np).pin_memory()
     pinned = args.e2e_host == "pinned"
-    copy_stream = torch.cuda.Stream()
     rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
     e_ms, phases = [], {}
     for k in range(args.e2e_steps + 1):
@@ -645,27 +644,25 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
             out_rp.copy_(rp_lu, non_blocking=pinned)
             he.emit(rp_lu, ci_lu, rb, re_)                         # S6
             mark("emit")
-        # the pattern's D2H on a copy stream, overlapping the levelization on the main one
-        copy_stream.wait_stream(stream)
-        with torch.cuda.stream(copy_stream):
-            out_ci.copy_(ci_lu, non_blocking=pinned)
+        # levels first (their host read-back would queue behind the pattern's D2H on the copy
+        # engine), then the copies
         level, _ = he.levelize(rp_lu, ci_lu, args.rule)        # S8 + S9
+        mark("levelize")
+        out_ci.copy_(ci_lu, non_blocking=pinned)
         out_lv.copy_(level, non_blocking=pinned)
-        mark("levelize+d2h(levels)")
-        stream.wait_stream(copy_stream)
         b.record(stream)
         torch.cuda.synchronize()
         he.close()
         if k == 0:   # the first call of the process: allocator caches still cold
             cold = {"ms": a.elapsed_time(b), "phases_ms": {}}
             prev = a
-            for tag, e_ in marks + [("d2h(pattern) overlapping levelize", b)]:
+            for tag, e_ in marks + [("d2h(pattern, levels)", b)]:
                 cold["phases_ms"][tag] = prev.elapsed_time(e_)
                 prev = e_
         else:
             e_ms.append(a.elapsed_time(b))
             prev = a
-            for tag, e_ in marks + [("d2h(pattern) overlapping levelize", b)]:
+            for tag, e_ in marks + [("d2h(pattern, levels)", b)]:
                 phases.setdefault(tag, []).append(prev.elapsed_time(e_))
                 prev = e_
         if verify is not None:

@@ -3,6 +3,9 @@
 #include "internal.h"
 
 #include <cstdlib>
+#include <map>
+#include <mutex>
+#include <tuple>
 
 namespace lusym {
 
@@ -61,14 +64,51 @@ bool fill2_smem_base_ok(int dev)
     default: return cudaErrorInvalidValue;                                                   \
     }
 
-cudaError_t fill2_configure(int nt, int w, int vis, size_t smem)
+namespace {
+cudaError_t configure_impl(int nt, int w, int vis, size_t smem)
 {
     LUSYM_NT_SWITCH(fill2_configure_nt, w, vis, smem)
+}
+cudaError_t occupancy_impl(int nt, int w, int vis, size_t smem, int *occ)
+{
+    LUSYM_NT_SWITCH(fill2_occupancy_nt, w, vis, smem, occ)
+}
+// the planner queries many (CTA size, W, visited mode, shared bytes) combinations per handle:
+// set each kernel's attribute and compute each occupancy once per device and process
+std::mutex g_mu;
+std::map<std::tuple<int, int, int, int, size_t>, int> g_occ;
+std::map<std::tuple<int, int, int, int>, size_t> g_conf;
+int cur_dev()
+{
+    int d = 0;
+    cudaGetDevice(&d);
+    return d;
+}
+}  // namespace
+
+cudaError_t fill2_configure(int nt, int w, int vis, size_t smem)
+{
+    const auto key = std::make_tuple(cur_dev(), nt, w, vis);
+    std::lock_guard<std::mutex> lock(g_mu);
+    auto it = g_conf.find(key);
+    if (it != g_conf.end() && it->second >= smem) return cudaSuccess;
+    cudaError_t e = configure_impl(nt, w, vis, smem);
+    if (e == cudaSuccess) g_conf[key] = smem;
+    return e;
 }
 
 cudaError_t fill2_occupancy(int nt, int w, int vis, size_t smem, int *occ)
 {
-    LUSYM_NT_SWITCH(fill2_occupancy_nt, w, vis, smem, occ)
+    const auto key = std::make_tuple(cur_dev(), nt, w, vis, smem);
+    std::lock_guard<std::mutex> lock(g_mu);
+    auto it = g_occ.find(key);
+    if (it != g_occ.end()) {
+        *occ = it->second;
+        return cudaSuccess;
+    }
+    cudaError_t e = occupancy_impl(nt, w, vis, smem, occ);
+    if (e == cudaSuccess) g_occ[key] = *occ;
+    return e;
 }
 
 cudaError_t fill2_launch(const Fill2Params &p, int nt, int w, int mode, int vis, int grid,

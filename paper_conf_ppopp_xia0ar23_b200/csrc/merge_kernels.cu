@@ -26,6 +26,9 @@
 
 #include <climits>
 #include <cooperative_groups.h>
+#include <map>
+#include <mutex>
+#include <tuple>
 
 namespace cg = cooperative_groups;
 
@@ -521,6 +524,9 @@ int cluster_shift(int n, int g)
 
 }  // namespace
 
+cudaError_t merge_configure_impl(size_t smem);
+cudaError_t merge_max_clusters_impl(int g, size_t smem, int *clusters);
+
 size_t merge_smem_bytes(int n, int mode, int g, int q)
 {
     size_t b = kHdrBytes + (2 * (size_t)NT + kSent) * sizeof(long long) +
@@ -531,6 +537,17 @@ size_t merge_smem_bytes(int n, int mode, int g, int q)
 }
 
 cudaError_t merge_configure(size_t smem)
+{
+    static size_t done[64];  // per device: the largest size already set
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (dev >= 0 && dev < 64 && done[dev] >= smem) return cudaSuccess;
+    cudaError_t e0 = merge_configure_impl(smem);
+    if (e0 == cudaSuccess && dev >= 0 && dev < 64) done[dev] = smem;
+    return e0;
+}
+
+cudaError_t merge_configure_impl(size_t smem)
 {
     const void *fns[3] = {(const void *)k_merge_rows<0>, (const void *)k_merge_rows<1>,
                           (const void *)k_merge_rows<2>};
@@ -544,6 +561,24 @@ cudaError_t merge_configure(size_t smem)
 }
 
 cudaError_t merge_max_clusters(int g, size_t smem, int *clusters)
+{
+    static std::map<std::tuple<int, int, size_t>, int> cache;
+    static std::mutex mu;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    std::lock_guard<std::mutex> lock(mu);
+    const auto key = std::make_tuple(dev, g, smem);
+    auto it = cache.find(key);
+    if (it != cache.end()) {
+        *clusters = it->second;
+        return cudaSuccess;
+    }
+    cudaError_t e0 = merge_max_clusters_impl(g, smem, clusters);
+    if (e0 == cudaSuccess) cache[key] = *clusters;
+    return e0;
+}
+
+cudaError_t merge_max_clusters_impl(int g, size_t smem, int *clusters)
 {
     cudaLaunchConfig_t cfg = {};
     cfg.gridDim = dim3(g * 64, 1, 1);

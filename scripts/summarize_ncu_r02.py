@@ -31,7 +31,9 @@ SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "ns": 1, "us": 1e3
 path = os.path.join(OUT, "ncu_summary.json")
 summary = json.load(open(path)) if os.path.exists(path) else {}
 for arg in sys.argv[1:]:
-    cfg, spec = arg.split("=", 1)
+    key, spec = arg.split("=", 1)
+    cfg, _, kkey = key.partition("/")
+    kkey = kkey or "fill2_stage"
     rep, _, log = spec.partition(":")
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True,
                          text=True).stdout
@@ -58,11 +60,14 @@ for arg in sys.argv[1:]:
             if mm and "==PROF" not in line:
                 rec["rows"] = [int(mm.group(1)), int(mm.group(2))]
                 rec["sv"] = int(mm.group(4))
-    summary.setdefault(cfg, {})["fill2_stage"] = rec
-    summary[cfg]["_source"] = (f"ncu --set full --import-source on of scripts/prof_count.py "
-                               f"({os.path.basename(rep)}); rows {rec.get('rows', 'all')}")
-    with open(os.path.join(OUT, f"ncu_{cfg}.txt"), "w") as f:
-        f.write(f"# {summary[cfg]['_source']}\n# kernel: {kname}\n")
+    summary.setdefault(cfg, {})[kkey] = rec
+    src = (f"ncu --set full --import-source on of scripts/prof_count.py "
+           f"({os.path.basename(rep)}); rows {rec.get('rows', 'all')}")
+    if kkey == "fill2_stage":
+        summary[cfg]["_source"] = src
+    fname = f"ncu_{cfg}.txt" if kkey == "fill2_stage" else f"ncu_{cfg}_{kkey}.txt"
+    with open(os.path.join(OUT, fname), "w") as f:
+        f.write(f"# {src}\n# kernel: {kname}\n")
         t = rec["time_ns"] / 1e9
         f.write(f"duration_ms            {rec['time_ns'] / 1e6:.3f}\n")
         f.write(f"dram_bytes             {rec['dram_bytes']:.4e}  ({rec['dram_bytes'] / t / 1e9:.1f} GB/s)\n")
