@@ -45,6 +45,12 @@ namespace f2 {
 #ifndef LUSYM_ENC_ELL  // BFS of shared-map kernels reads neighbours pre-encoded as shared
 #define LUSYM_ENC_ELL 1    // bitmap addresses (enc_slot), decoding only newly visited ones
 #endif
+#ifndef LUSYM_PREFETCH_NEXT  // prefetch a new frontier vertex's adjacency row into L1
+#define LUSYM_PREFETCH_NEXT 0  // A/B: +7..15% slower (profiles/r02/ab_prefetch.log)
+#endif
+#ifndef LUSYM_WARP_EXIT  // warps past the end of a BFS level / threshold window leave early
+#define LUSYM_WARP_EXIT 0  // A/B: +1.6..6.9% slower (profiles/r02/ab_wexit.log)
+#endif
 #ifndef LUSYM_TAM  // test_and_mark with one shared bit mask (0: visited() then mark())
 #define LUSYM_TAM 1
 #endif
@@ -504,6 +510,11 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
     const uint32_t ncnt_s = (uint32_t)__cvta_generic_to_shared(ncnt);
     unsigned nloc = 0;  // vertices expanded by self-continuation (statistics, lane 0)
     for (int base = 0; base < cnt; base += NT) {
+#if LUSYM_WARP_EXIT
+        // a warp past the end of the level leaves (warp-uniform) instead of running the body
+        // with no valid lane: levels narrower than the CTA are most of a BFS's levels
+        if (base + (tid & ~31) >= cnt) break;
+#endif
         const int k = base + tid;
         bool valid = k < cnt;
         int f = valid ? (k < p.q ? L[k] : __ldcg(gL + k)) : 0;
@@ -528,6 +539,11 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                     int w;
                     if (test_and_mark_enc(bm, nb[s], &w)) {
                         if (w < t0) {
+#if LUSYM_PREFETCH_NEXT
+                            // the next level reads w's adjacency: start it towards L1 now
+                            asm volatile("prefetch.global.L1 [%0];" ::"l"(
+                                p.elle + (size_t)w * ell_stride<W>()));
+#endif
                             if (c == 3) {
                                 put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
                             } else {
@@ -967,6 +983,9 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
             if (tid == 0) h.sv += wc;
             int nm = INT_MAX;
             for (int base = 0; base < wc; base += NT) {
+#if LUSYM_WARP_EXIT
+                if (base + (tid & ~31) >= wc) break;  // warp-uniform, as in scan_level
+#endif
                 const int k = base + tid;
                 const bool valid = k < wc;
                 const int t = valid ? qA[k] : 0;
