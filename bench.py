@@ -457,6 +457,10 @@ def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
     # N > 1: rows deferred on any rank are finished after the pattern exchange (reading G8)
     sym_opts = dict(flags=args.flags | (lu.F_DEFER_GLOBAL if world > 1 else 0),
                     threads_per_row=args.threads_per_row, queue_capacity=args.queue_capacity)
+    if os.environ.get("LUSYM_BENCH_ONE_GPU") and world > 1:
+        # test hook only: the ranks share one GPU, so each takes its share of the memory
+        free, _ = torch.cuda.mem_get_info()
+        sym_opts["scratch_budget_bytes"] = int(0.4 * free / world)
     h = lu.Symbolic(rp, ci, **sym_opts)
     ms_create = h.stats()["ms_create"]
     cost = lu.row_cost_upper_bound(rp_np)

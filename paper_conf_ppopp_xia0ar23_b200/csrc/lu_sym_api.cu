@@ -65,6 +65,7 @@ lu_status fail(lu_status s, const char *fmt, ...)
     } while (0)
 
 enum { kEvCount = 0, kEvScan = 1, kEvEmit = 2, kEvLev = 3, kEvTail = 4, kEvN = 5 };
+constexpr int kSparseDeferWindows = 1024;  // sparse class (G9): see the comment in plan()
 enum { kSlotPoolCursor = 9, kSlotUnstaged = 10, kSlotList = 11, kSlotClassCounter = 16,
        kSlotSetStride = 32, kSlotDefer = 112 /* [0] deferred rows, [1] tail claims,
        [2] failed rows, [3..5] tail statistics */, kStatSlots = 128, kMaxChunks = 64, kSets = 3 };
@@ -80,6 +81,7 @@ struct RowClass {
     size_t smem;
     int64_t cap = 0;  // per-CTA spill / staging capacity (entries)
     int grid = 0;
+    int defer_win = 0;  // > 0: this class's own deferral threshold (windows), else the handle's
     // this class's disjoint scratch regions (classes run concurrently)
     int64_t spill_off = 0, stg_off = 0, map_off = 0;
     cudaStream_t stream = nullptr;  // classes after the first run on their own stream
@@ -514,9 +516,10 @@ lu_status plan(lu_sym *h)
         Cfg g;
         if ((st = best_cfg(h, 0, kVisGlobal, smem_optin, &g, 64, 256)) != LU_OK) return st;
         size_t kc = 0;
-        // candidates: the classes whose shared map holds them below 8 rows per SM
-        while (g.key >= 0 && kc < h->classes.size() && h->classes[kc].occ < 8 &&
-               h->classes[kc].occ < g.occ)
+        // candidates: the classes (from the top) with fewer rows per SM than the sparse class,
+        // considered only when the top class's shared map holds it below 8 rows per SM
+        while (g.key >= 0 && kc < h->classes.size() && h->classes[kc].occ < g.occ &&
+               h->classes.front().occ < 8)
             ++kc;
         const bool force = getenv("LUSYM_FORCE_SPARSE") != nullptr;  // test knob
         if (force && g.key >= 0) kc = h->classes.size();
@@ -530,6 +533,11 @@ lu_status plan(lu_sym *h)
                 h->classes.erase(h->classes.begin(), h->classes.begin() + (long)kc);
                 h->classes.insert(h->classes.begin(),
                                   RowClass{lo, n, kVisGlobal, 0, 0, g.nt, g.q, g.occ, g.smem});
+                // 64 threads and 256-entry windows make each threshold window slow: abandon a
+                // row (G8) after fewer windows than a shared-map class would
+                h->classes.front().defer_win = kSparseDeferWindows;
+                if (const char *e = getenv("LUSYM_SPARSE_DEFER_WINDOWS"))  // A/B knob
+                    h->classes.front().defer_win = atoi(e);
             }
         }
     }
@@ -687,6 +695,8 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     bool forked = false;
     for (size_t k = 0; k < h->classes.size(); ++k) {
         const RowClass &c = h->classes[k];
+        if (p.defer_win > 0 && c.defer_win > 0) p.defer_win = std::min(h->defer_win, c.defer_win);
+        else if (p.defer_win > 0) p.defer_win = h->defer_win;
         // a row list (rows that did not fit the staging pool) runs in the top class only
         if (row_list && k > 0) break;
         const int32_t lo = row_list ? 0 : std::max(rb, c.lo), hi = row_list ? 0 : std::min(re, c.hi);

@@ -37,7 +37,10 @@ namespace {
 
 constexpr int NT = kMergeNT;
 constexpr int NW = NT / 32;
-constexpr int kU = 4;      // pool loads in flight per thread
+#ifndef LUSYM_MERGE_KU
+#define LUSYM_MERGE_KU 4
+#endif
+constexpr int kU = LUSYM_MERGE_KU;  // pool loads in flight per thread
 constexpr int kSent = 64;  // sentinel starts past the last segment
 
 struct MHdr {

@@ -99,11 +99,21 @@ def assemble_pattern(col_idx_lu: torch.Tensor, row_ptr_lu: torch.Tensor, bounds,
     idx = torch.as_tensor(np.asarray(bounds, dtype=np.int64), device=row_ptr_lu.device)
     offs = row_ptr_lu.index_select(0, idx).cpu().numpy()
     sizes = np.diff(offs)
+    mx = max(int(sizes.max()), 1)
     if _device_collectives(col_idx_lu, group) and dist.get_backend(group) == "nccl":
         views = [col_idx_lu[int(offs[r]):int(offs[r + 1])] for r in range(world)]
-        dist.all_gather(views, views[rank], group=group)
+        try:
+            dist.all_gather(views, views[rank], group=group)
+        except (RuntimeError, ValueError):
+            # a torch without uneven all_gather: one padded all_gather_into_tensor on the device
+            send = torch.zeros(mx, dtype=col_idx_lu.dtype, device=col_idx_lu.device)
+            send[:sizes[rank]] = views[rank]
+            recv = torch.empty(world * mx, dtype=col_idx_lu.dtype, device=col_idx_lu.device)
+            dist.all_gather_into_tensor(recv, send, group=group)
+            for r in range(world):
+                if r != rank and sizes[r]:
+                    views[r].copy_(recv[r * mx:r * mx + sizes[r]])
         return col_idx_lu
-    mx = max(int(sizes.max()), 1)
     send = torch.zeros(mx, dtype=col_idx_lu.dtype)
     send[:sizes[rank]] = col_idx_lu[int(offs[rank]):int(offs[rank + 1])].cpu()
     recv = [torch.empty(mx, dtype=col_idx_lu.dtype) for _ in range(world)]
