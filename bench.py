@@ -587,6 +587,16 @@ def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
         rec["partition"] = {"bounds": [int(b) for b in bounds],
                             "by": "a-priori bound row_ptr[i+1]" if args.apriori_partition
                             else "per-row cycles measured in a profiled pass"}
+    if headline and world == 1:
+        # the library's own count of the method's work (F_COUNT_TE, outside the timed region)
+        hc = lu.Symbolic(rp, ci, flags=args.flags | lu.F_COUNT_TE | lu.F_NO_DEFER)
+        hc.count()
+        sc = hc.stats()
+        hc.close()
+        rec["work_units_library"] = {
+            "traversed_edges": sc["edges_read_count"], "scanned_vertices":
+            sc["vertices_scanned_count"],
+            "match_golden": sc["edges_read_count"] == te and sc["vertices_scanned_count"] == sv}
     if headline and not args.no_e2e:
         rec["e2e"] = e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank,
                          bounds, verify)
@@ -747,6 +757,7 @@ def run_ours(args, rank, world, local_rank):
         "symbolic_s": head["symbolic_s"], "levelize_s": head["levelize_s"], "teps": head["teps"],
         "traversed_edges_per_pass": head["traversed_edges_per_pass"],
         "scanned_vertices_per_pass": head["scanned_vertices_per_pass"],
+        "work_units_library": head.get("work_units_library"),
         "roofline": head["roofline"], "cpu_baseline": cpu, "e2e": head.get("e2e"),
         "gpu_launches": head["gpu_launches"], "clocks": head["clocks"], "plan": head["plan"],
         "per_config": per,

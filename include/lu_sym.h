@@ -101,6 +101,10 @@ enum {
                                     sparse class (HBM visited slots, 16 rows per SM) that a
                                     create-time sample of rows selects when they visit < n/16
                                     vertices on average (reading G9)              */
+    LU_F_COUNT_TE = 1 << 17,     /* a statistics handle: lu_sym_count counts the traversed
+                                    edges of every scanned vertex, so stats.edges_read_count
+                                    is the method's exact TE (reading R24); its count pass
+                                    does not stage rows (lu_sym_emit then traverses again)   */
     LU_F_DEFER_GLOBAL = 1 << 16  /* row sharding (reading G8 across GPUs): lu_sym_count may
                                     defer rows even when the rows below them are counted on
                                     other GPUs; it then runs no tail: the deferred rows keep
@@ -139,11 +143,12 @@ typedef struct {
     double ms_create;             /* validate + adjacency build + planning                  */
     double ms_count, ms_scan, ms_emit, ms_levelize; /* last call of each (device events)     */
     int64_t nnz_lu;               /* after lu_sym_scan                                       */
-    int64_t edges_read_count;     /* entries read from A's CSR (seed rows and heavy rows,    */
-    int64_t edges_read_emit;      /*   last count / emit pass) — ELL reads of light rows are
-                                     not counted; the method's traversed edges TE (R24) come
-                                     from the oracle / closed forms (tests/golden)           */
-    int64_t vertices_scanned_count, vertices_scanned_emit;
+    int64_t edges_read_count;     /* traversed edges (R24) of the last count / emit pass:    */
+    int64_t edges_read_emit;      /*   exact with LU_F_COUNT_TE; without it only the entries
+                                     read from A's CSR (seed rows, heavy rows)               */
+    int64_t vertices_scanned_count, vertices_scanned_emit; /* scanned vertices (every
+                                     threshold once + every BFS vertex), exact; rows deferred
+                                     to the tail (G8) contribute what they scanned before    */
     int64_t spills;               /* frontier entries that spilled from smem to HBM          */
     int64_t scratch_bytes;        /* HBM scratch owned by the handle                         */
     int32_t rows_in_flight;       /* CTAs (= rows processed concurrently)                    */

@@ -42,7 +42,7 @@ F_GLOBAL_BITMAP, F_NO_BATCH, F_ASCENDING, F_NO_PRUNE, F_KAHN_WIDE_ONLY = 1, 2, 4
 F_NO_CONTRACT, F_TWO_PASS, F_ONE_CLASS, F_FORCE_CLASSES = 32, 64, 128, 256
 F_SELF_CONT, F_NO_SELF_CONT, F_PAPER_CHUNKS = 512, 1024, 2048
 F_MANAGED, F_MANAGED_PREFETCH, F_NO_DEFER, F_NO_SPARSE = 4096, 8192, 16384, 32768
-F_DEFER_GLOBAL = 65536
+F_DEFER_GLOBAL, F_COUNT_TE = 65536, 131072
 
 
 class LuSymError(RuntimeError):

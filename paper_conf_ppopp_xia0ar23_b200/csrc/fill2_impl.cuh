@@ -318,6 +318,26 @@ __device__ __forceinline__ void load_nb(const int32_t *ell, int f, int (&nb)[ell
     }
 }
 
+// Traversed edges of a scanned light vertex (reading R24: its full row, diagonal included):
+// the slots that are not its own padding, + 1 for the diagonal (build_ell makes every row
+// without a diagonal a heavy record, whose CSR length is counted instead).  pad = the padding
+// value of the row: the vertex itself, encoded as the slots are.
+template <int W>
+__device__ __forceinline__ int row_edges(const int (&nb)[ell_stride<W>()], int pad)
+{
+    int d = 1;
+#pragma unroll
+    for (int s = 0; s < W; ++s) d += nb[s] != pad;
+    return d;
+}
+
+__device__ __forceinline__ int enc_vertex(int v)
+{
+    int pw = v >> 5;
+    if (LUSYM_SWZ) pw ^= (pw >> 5) & 31;
+    return (pw << 7) | (v & 31);
+}
+
 // store a frontier entry (shared memory, HBM past q)
 __device__ __forceinline__ void put(int pos, int w, int32_t *NF, int32_t *gNF, int q)
 {
@@ -499,7 +519,7 @@ struct RowAcc {
 // only the other discoveries go through the next-level queue.  Worth it only where a row has
 // an SM to itself and waits on each level's latency (the planner sets kloc per row class):
 // with many rows per SM the extra rounds, in which lanes drop out, cost issue slots.
-template <int NT, int W, int VIS, bool SC>
+template <int NT, int W, int VIS, bool SC, int MODE>
 __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm,
                                            uint32_t *sm, const int32_t *L, const int32_t *gL,
                                            int cnt, int *ncnt, int32_t *NF, int32_t *gNF,
@@ -509,6 +529,7 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
     const unsigned lt = (1u << lane) - 1u;
     const uint32_t ncnt_s = (uint32_t)__cvta_generic_to_shared(ncnt);
     unsigned nloc = 0;  // vertices expanded by self-continuation (statistics, lane 0)
+    unsigned long long te_loc = 0;  // traversed edges of light vertices (p.count_te)
     for (int base = 0; base < cnt; base += NT) {
 #if LUSYM_WARP_EXIT
         // a warp past the end of the level leaves (warp-uniform) instead of running the body
@@ -533,6 +554,8 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
         if (valid) {
             load_nb<W>(enc ? p.elle : p.ell, f, nb);
             heavy = nb[0] == kHeavy;
+            if constexpr (MODE == kCount)  // the statistics pass only (LU_F_COUNT_TE)
+                if (p.count_te && !heavy) te_loc += row_edges<W>(nb, enc ? enc_vertex(f) : f);
             if (enc && !heavy) {
 #pragma unroll
                 for (int s = 0; s < W; ++s) {
@@ -664,6 +687,11 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
       }
     }
     if (SC && lane == 0 && nloc) atomicAdd(&h.sv, (unsigned long long)nloc);
+    if (MODE == kCount && p.count_te) {
+#pragma unroll
+        for (int o = 16; o; o >>= 1) te_loc += __shfl_xor_sync(kFull, te_loc, o);
+        if (lane == 0 && te_loc) atomicAdd(&h.te, te_loc);
+    }
 }
 
 // Plain level-synchronous variant of scan_level with VPT frontier vertices per thread per
@@ -769,7 +797,7 @@ __device__ __forceinline__ void scan_level_multi(const Fill2Params &p, Hdr &h,
 // HBM halves); the level counters rotate through h.cnt[0..2] so one barrier per level suffices.
 // Queue and spill addresses are recomputed from the launch parameters each level rather than
 // carried in registers (at 32 registers per thread they would otherwise spill).
-template <int NT, int W, int VIS>
+template <int NT, int W, int VIS, int MODE>
 __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_t *sm, int32_t *qA,
                     const int i, const int t0, RowAcc &a)
 {
@@ -786,7 +814,7 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_
         const int nxt = cur == 2 ? 0 : cur + 1;
         int32_t *gA = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
         if (p.kloc)
-            scan_level<NT, W, VIS, true>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
+            scan_level<NT, W, VIS, true, MODE>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
                                          fsize, &h.cnt[nxt], qA + (par ^ 1) * p.q,
                                          gA + (par ^ 1) * p.spill_cap, i, t0, a);
         else if (LUSYM_VPT > 1)
@@ -795,7 +823,7 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_
                                                     qA + (par ^ 1) * p.q,
                                                     gA + (par ^ 1) * p.spill_cap, i, t0, a);
         else
-            scan_level<NT, W, VIS, false>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
+            scan_level<NT, W, VIS, false, MODE>(p, h, bm, sm, qA + par * p.q, gA + par * p.spill_cap,
                                           fsize, &h.cnt[nxt], qA + (par ^ 1) * p.q,
                                           gA + (par ^ 1) * p.spill_cap, i, t0, a);
         __syncthreads();
@@ -980,8 +1008,8 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                     }
                 }
             }
-            if (tid == 0) h.sv += wc;
             int nm = INT_MAX;
+            unsigned long long w_te = 0;  // traversed edges of this thread's done thresholds
             for (int base = 0; base < wc; base += NT) {
 #if LUSYM_WARP_EXIT
                 if (base + (tid & ~31) >= wc) break;  // warp-uniform, as in scan_level
@@ -1008,6 +1036,8 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                         atomicMin(&h.tns, t);
                     } else {
                         done = true;
+                        if constexpr (MODE == kCount)
+                            if (p.count_te) w_te += row_edges<W>(nb, t);
 #pragma unroll
                         for (int s = 0; s < W; ++s) {
                             const int w = nb[s];
@@ -1036,7 +1066,8 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                         if (w < tt && !visited(bm, w)) ok = false;
                     }
                     ok = __all_sync(kFull, ok);
-                    if (lane == 0) atomicAdd(&h.te, (unsigned long long)len);
+                    // a heavy threshold is scanned once: when it is simple here, else by its BFS
+                    if (lane == 0 && ok) atomicAdd(&h.te, (unsigned long long)len);
                     if (lane == src) done = ok;
                     if (!ok) {
                         if (lane == 0) atomicMin(&h.tns, tt);
@@ -1055,6 +1086,15 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
                     }
                 }
                 if (valid) qB[k] = done ? 1 : 0;
+                // scanned vertices: a threshold counts once, when it is done here
+                // (simple) or when its BFS starts (non-simple ones are re-collected until then)
+                const unsigned db = __ballot_sync(kFull, valid && done);
+                if (lane == 0 && db) atomicAdd(&h.sv, (unsigned long long)__popc(db));
+            }
+            if (MODE == kCount && p.count_te) {
+#pragma unroll
+                for (int o = 16; o; o >>= 1) w_te += __shfl_xor_sync(kFull, w_te, o);
+                if (lane == 0 && w_te) atomicAdd(&h.te, w_te);
             }
             if (nm != INT_MAX) atomicMin(&h.newmin, nm);
             __syncthreads();
@@ -1080,7 +1120,7 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
             if (nptr <= ptr) __syncthreads();
             PH_MARK(ph_win);
             if (m <= last && m == tns) {  // smallest pending threshold: below-exploration
-                bfs<NT, W, VIS>(p, h, bm, sm, qA, i, m, a);
+                bfs<NT, W, VIS, MODE>(p, h, bm, sm, qA, i, m, a);
                 ++n_bfs;
             }
             cap = m <= last ? min(cap, kSmallWin) : min(2 * cap, p.wcap);

@@ -60,6 +60,9 @@ struct Fill2Params {
     int64_t *row_prof;
     // self-continuation rounds per BFS level (scan_level); 0 = plain level-synchronous BFS
     int32_t kloc;
+    // count the traversed edges of light vertices too (exact TE, reading R24; ~W+2 integer
+    // instructions per scanned vertex, so only when LU_F_COUNT_TE asks for it)
+    int32_t count_te = 0;
     // row_list length read on the device (a list built by an earlier kernel), when non-null
     const unsigned long long *list_len_dev = nullptr;
     // kStage: entries <= i of each staged row (L part + diagonal), for the row-merge tail

@@ -683,6 +683,7 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
     p.row_prof = h->row_prof;
     p.ucut = h->ucut;
     p.list_len_dev = list_len_dev;
+    p.count_te = (h->opts.flags & LU_F_COUNT_TE) ? 1 : 0;
     if (mode == kStage && h->defer_active && !row_list) {
         p.defer_win = h->defer_win;
         p.defer_from = h->defer_from;
@@ -1130,7 +1131,9 @@ lu_status lu_sym_count(lu_sym *h, int32_t row_begin, int32_t row_end, int32_t *d
     bool defer = false, global_defer = false;
     h->tail_ran = false;
     h->deferred_pending = false;
-    if (h->staging) {
+    // LU_F_COUNT_TE: a statistics handle, counts only (the edge counting is compiled into the
+    // count kernels alone, so the staged pass carries no per-vertex test for it)
+    if (h->staging && !(h->opts.flags & LU_F_COUNT_TE)) {
         if ((st = ensure_merge(h)) != LU_OK) return st;
         st = ensure_pool(h);
         if (st != LU_OK) return st;

@@ -56,12 +56,10 @@ __global__ void k_count_light(int32_t n, const int64_t *rp, const int32_t *ci, i
     if (i < n) {
         const int64_t a = rp[i], b = rp[i + 1];
         const int64_t len = b - a;
-        if (len <= w) {
-            light = true;
-        } else if (len == w + 1) {
+        // light = in the ELL: the diagonal present and at most w off-diagonal entries
+        if (len <= w + 1)
             for (int64_t k = a; k < b; ++k)
                 if (ci[k] == i) light = true;
-        }
     }
     const unsigned m = __ballot_sync(kFull, light);
     if ((threadIdx.x & 31) == 0 && m) atomicAdd(cnt, (unsigned long long)__popc(m));
@@ -85,9 +83,13 @@ __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int
     bool heavy = len > W + 1;
     if (!heavy) {
         int m = 0;
+        bool diag = false;
         for (int64_t k = a; k < b; ++k) {
             const int c = ci[k];
-            if (c == i) continue;
+            if (c == i) {
+                diag = true;
+                continue;
+            }
             if (m == W) {
                 heavy = true;
                 break;
@@ -97,6 +99,9 @@ __global__ void k_build_ell(int32_t n, const int64_t *rp, const int32_t *ci, int
                 if (s == m) out[s] = c;
             ++m;
         }
+        // a light row always has its diagonal, so its traversed edges are its non-padding
+        // slots + 1 (fill2 row_edges); a row without one is read from the CSR instead
+        if (!diag) heavy = true;
     }
     if (heavy) {
         out[0] = kHeavy;

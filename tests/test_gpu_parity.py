@@ -654,3 +654,29 @@ def test_deferred_rows_across_shards(defer_windows):
         fc, rp_lu, ci_lu = lu.sharded_pass(h, 0, n, [0, n])
         assert np.array_equal(ci_lu.cpu().numpy(), ref["col_idx"])
         h.close()
+
+
+@pytest.mark.parametrize("knob", [dict(), dict(flags=lu.F_NO_BATCH), dict(flags=lu.F_SELF_CONT),
+                                  dict(flags=lu.F_GLOBAL_BITMAP), dict(flags=lu.F_FORCE_CLASSES),
+                                  dict(queue_capacity=32), dict(threads_per_row=1024)], ids=str)
+def test_stats_are_the_methods_work_units(knob):
+    """The library's own counters are the method's work (reading R24): scanned
+    vertices (every threshold once + every BFS vertex) and, with F_COUNT_TE, traversed edges
+    (seed row + every scanned vertex's row, diagonal included) equal the oracle's per-row TE /
+    SV summed — checked with and without diagonals, heavy rows and the knobs that change the
+    traversal's schedule."""
+    d = dev()
+    knob = dict(knob)
+    flags = knob.pop("flags", 0) | lu.F_COUNT_TE | lu.F_NO_DEFER
+    for rp, ci in (gen.lap3d(9), gen.lap2d(20), gen.circuit(40, 2), _hub_matrix(),
+                   gen.random_pattern(700, 2.5, seed=9),
+                   gen.random_pattern(500, 2.2, seed=3, zero_free_diag=False)):
+        ref = oracle.fill2(rp, ci, emit=False)
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d), flags=flags,
+                        **knob)
+        fc = h.count()
+        st = h.stats()
+        assert np.array_equal(fc.cpu().numpy(), ref["counts"])
+        assert st["vertices_scanned_count"] == int(ref["sv"].sum()), (knob, st)
+        assert st["edges_read_count"] == int(ref["te"].sum()), (knob, st)
+        h.close()
