@@ -45,6 +45,9 @@ namespace f2 {
 #ifndef LUSYM_ENC_ELL  // BFS of shared-map kernels reads neighbours pre-encoded as shared
 #define LUSYM_ENC_ELL 1    // bitmap addresses (enc_slot), decoding only newly visited ones
 #endif
+#ifndef LUSYM_GB_DIRECT_ATOMIC  // HBM visited slots: test-and-set by the atomic alone
+#define LUSYM_GB_DIRECT_ATOMIC 0
+#endif
 #ifndef LUSYM_PREFETCH_NEXT  // prefetch a new frontier vertex's adjacency row into L1
 #define LUSYM_PREFETCH_NEXT 0  // A/B: +7..15% slower (profiles/r02/ab_prefetch.log)
 #endif
@@ -245,6 +248,18 @@ __device__ __forceinline__ bool test_and_mark(const VisMap<VIS> &m, uint32_t *sm
     const uint32_t b = 1u << (v & 31);
     const int w = v >> 5;
     const bool sh = in_smem(m, w);
+#if LUSYM_GB_DIRECT_ATOMIC
+    if (VIS == kVisGlobal) {
+        // HBM slot: one L2 round trip (the atomic returns the old word) instead of a load
+        // followed, for an unvisited bit, by the atomic
+        const uint32_t old = atomicOr(m.g + w, b);
+        if (old == 0)
+            asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(summary_saddr(m) + (uint32_t)(v >> 10) * 4u),
+                         "r"(1u << (w & 31))
+                         : "memory");
+        return !(old & b);
+    }
+#endif
     const uint32_t word = sh ? lds_bm(phys<VIS>(m, w)) : __ldcg(m.g + w);
     if (word & b) return false;
     const uint32_t old = sh ? atom_or_bm(phys<VIS>(m, w), b) : atomicOr(m.g + w, b);
