@@ -105,6 +105,12 @@ enum {
                                     edges of every scanned vertex, so stats.edges_read_count
                                     is the method's exact TE (reading R24); its count pass
                                     does not stage rows (lu_sym_emit then traverses again)   */
+    LU_F_ASYNC_BFS = 1 << 18,    /* below-threshold traversal without level barriers (warp
+                                    rings + a CTA pool; the order below a threshold is free,
+                                    reading R5) in every row class of the 1024-thread
+                                    one-CTA-per-SM kernel, not only in classes with at most
+                                    2 rows per SM                                             */
+    LU_F_NO_ASYNC_BFS = 1 << 19, /* level-synchronous BFS in every row class                 */
     LU_F_DEFER_GLOBAL = 1 << 16  /* row sharding (reading G8 across GPUs): lu_sym_count may
                                     defer rows even when the rows below them are counted on
                                     other GPUs; it then runs no tail: the deferred rows keep

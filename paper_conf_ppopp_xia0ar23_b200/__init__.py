@@ -43,6 +43,7 @@ F_NO_CONTRACT, F_TWO_PASS, F_ONE_CLASS, F_FORCE_CLASSES = 32, 64, 128, 256
 F_SELF_CONT, F_NO_SELF_CONT, F_PAPER_CHUNKS = 512, 1024, 2048
 F_MANAGED, F_MANAGED_PREFETCH, F_NO_DEFER, F_NO_SPARSE = 4096, 8192, 16384, 32768
 F_DEFER_GLOBAL, F_COUNT_TE = 65536, 131072
+F_ASYNC_BFS, F_NO_ASYNC_BFS = 1 << 18, 1 << 19
 
 
 class LuSymError(RuntimeError):

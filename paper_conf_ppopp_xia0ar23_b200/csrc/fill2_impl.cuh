@@ -71,6 +71,9 @@ struct Hdr {
     long long stage_off;
     unsigned long long te, sv, spills;  // statistics of this CTA (thread 0 / shared atomics)
     int scan[40];
+    // asynchronous BFS (bfs_async): pool lock, pool entries, vertices discovered and not yet
+    // expanded (in a ring, in the pool or being expanded), idle warps
+    int alock, ptop, outst, idle;
 };
 static_assert(sizeof(Hdr) <= kHdrBytes, "header too large");
 
@@ -807,15 +810,268 @@ __device__ __forceinline__ void scan_level_multi(const Fill2Params &p, Hdr &h,
     }
 }
 
+// ---- Asynchronous below-threshold traversal (reading R5: which vertices below t0 are reached
+// is fixed, the order is free, so no level barrier is needed).  Each warp expands up to 32
+// vertices at a time from its own ring in shared memory (head/tail in registers: no atomics on
+// the queue) and appends what they discover to the same ring.  A warp whose ring is empty takes
+// work from the CTA's pool (a stack in the rest of the queues' shared memory, continued in the
+// HBM frontier spill region, under a shared-memory lock); a warp with a long ring donates half of it while other warps are idle, and a warp
+// whose ring would overflow moves its ring to the pool.  h.outst counts the vertices
+// discovered and not yet expanded (rings + pool + being expanded); the traversal is over when
+// it is 0.  A warp's children are added to h.outst before any of them can reach another warp
+// (at the latest when the warp donates), so it never reads 0 while work is left.
+
+// lane 0 takes the pool lock; every lane returns after it is held
+__device__ __forceinline__ void pool_lock(Hdr &h)
+{
+    if ((threadIdx.x & 31) == 0) {
+        while (atomicCAS(&h.alock, 0, 1) != 0) __nanosleep(32);
+        __threadfence_block();
+    }
+    __syncwarp();
+}
+
+// every lane's pool and ring accesses are ordered before lane 0 releases the lock
+__device__ __forceinline__ void pool_unlock(Hdr &h)
+{
+    __threadfence_block();
+    __syncwarp();
+    if ((threadIdx.x & 31) == 0) atomicExch(&h.alock, 0);
+    __syncwarp();
+}
+
+// Move the cnt oldest entries of the warp's ring to the pool (warp-uniform).  pend = children
+// appended since the warp last updated h.outst: they are counted before the pool publishes them.
+__device__ __forceinline__ void ring_donate(Hdr &h, int32_t *ring, int R, int &head, int cnt,
+                                            int32_t *spool, int pcap, int32_t *pool, int &pend,
+                                            unsigned long long &nspill)
+{
+    __syncwarp();
+    pool_lock(h);
+    const int lane = threadIdx.x & 31;
+    int top = 0;
+    if (lane == 0) {
+        if (pend) atomicAdd(&h.outst, pend);
+        top = *(volatile int *)&h.ptop;
+    }
+    top = __shfl_sync(kFull, top, 0);
+    for (int k = lane; k < cnt; k += 32) {
+        const int x = top + k, v = ring[(head + k) & (R - 1)];
+        if (x < pcap)
+            spool[x] = v;
+        else
+            __stcg(pool + (x - pcap), v);
+    }
+    __threadfence_block();
+    if (lane == 0) *(volatile int *)&h.ptop = top + cnt;
+    pool_unlock(h);
+    pend = 0;
+    head += cnt;
+    if (top + cnt > pcap) nspill += (unsigned long long)(top + cnt - max(top, pcap));
+}
+
+// warp-aggregated append of v (lanes with pred; b = their ballot) to the warp's ring
+__device__ __forceinline__ void ring_append(Hdr &h, bool pred, unsigned b, int v, int32_t *ring,
+                                            int R, int &head, int &tail, int32_t *spool, int pcap,
+                                            int32_t *pool, int &pend, unsigned long long &nspill)
+{
+    const int tot = __popc(b);
+    if (tail - head + tot > R)
+        ring_donate(h, ring, R, head, tail - head, spool, pcap, pool, pend, nspill);
+    if (pred) ring[(tail + __popc(b & ((1u << (threadIdx.x & 31)) - 1u))) & (R - 1)] = v;
+    tail += tot;
+    pend += tot;
+}
+
+template <int NT, int W, int VIS, int MODE>
+__device__ void bfs_async(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_t *sm,
+                          int32_t *qA, const int i, const int t0, RowAcc &a)
+{
+    constexpr int NW = NT / 32;
+    const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+    const int R = p.aring;  // ring entries per warp (a power of two >= 64)
+    int32_t *ring = qA + wid * R;
+    // the pool: the rest of the two frontier queues' shared memory, then the HBM spill region
+    int32_t *spool = qA + NW * R;
+    const int pcap = 2 * p.q - NW * R;
+    int32_t *pool = p.gspill + (size_t)blockIdx.x * 2 * p.spill_cap;
+    if (threadIdx.x == 0) {
+        h.alock = 0;
+        h.ptop = 0;
+        h.outst = 1;
+        h.idle = NW - 1;
+        ring[0] = t0;
+    }
+    __syncthreads();
+    int head = 0, tail = wid == 0 ? 1 : 0;  // warp-uniform ring positions
+    int pend = 0;                           // children not yet added to h.outst (uniform)
+    unsigned long long nproc = 0, nspill = 0, te_loc = 0;
+    bool idle = wid != 0;
+    const bool enc = LUSYM_ENC_ELL && VIS == kVisSmem && p.elle != nullptr;
+    for (;;) {
+        if (tail == head) {
+            // no work of its own: take from the pool, or stop when nothing is left anywhere
+            if (!idle) {
+                idle = true;
+                if (lane == 0) atomicAdd(&h.idle, 1);
+            }
+            int got = 0;
+            for (;;) {
+                int top = 0, out = 0;
+                if (lane == 0) {
+                    top = *(volatile int *)&h.ptop;
+                    out = *(volatile int *)&h.outst;
+                }
+                top = __shfl_sync(kFull, top, 0);
+                out = __shfl_sync(kFull, out, 0);
+                if (top > 0) {
+                    pool_lock(h);
+                    int t = 0;
+                    if (lane == 0) {
+                        t = *(volatile int *)&h.ptop;
+                        got = min(t, 32);
+                        *(volatile int *)&h.ptop = t - got;
+                    }
+                    t = __shfl_sync(kFull, t, 0);
+                    got = __shfl_sync(kFull, got, 0);
+                    if (lane < got) {
+                        const int x = t - got + lane;
+                        ring[(tail + lane) & (R - 1)] =
+                            x < pcap ? spool[x] : __ldcg(pool + (x - pcap));
+                    }
+                    pool_unlock(h);
+                    if (got) break;
+                } else if (out == 0) {
+                    break;
+                }
+                __nanosleep(p.asleep);
+            }
+            if (!got) break;
+            tail += got;
+            idle = false;
+            if (lane == 0) atomicSub(&h.idle, 1);
+        } else if (tail - head > p.akeep + 8) {
+            // other warps idle and the pool nearly empty: keep akeep entries, hand over the rest
+            int ask = 0;
+            if (lane == 0)
+                ask = *(volatile int *)&h.idle > 0 && *(volatile int *)&h.ptop < 32;
+            if (__shfl_sync(kFull, ask, 0))
+                ring_donate(h, ring, R, head, tail - head - p.akeep, spool, pcap, pool, pend,
+                            nspill);
+        }
+        __syncwarp();
+        const int m = min(tail - head, 32);
+        const bool valid = lane < m;
+        const int f = valid ? ring[(head + lane) & (R - 1)] : 0;
+        head += m;
+        nproc += (unsigned long long)m;
+        int nb[ell_stride<W>()];
+#pragma unroll
+        for (int s = 0; s < ell_stride<W>(); ++s) nb[s] = 0;
+        bool heavy = false;
+        unsigned newm = 0;  // slots whose neighbour joins the frontier (nb[s] then holds it)
+        if (valid) {
+            load_nb<W>(enc ? p.elle : p.ell, f, nb);
+            heavy = nb[0] == kHeavy;
+            if constexpr (MODE == kCount)
+                if (p.count_te && !heavy) te_loc += row_edges<W>(nb, enc ? enc_vertex(f) : f);
+            if (!heavy) {
+#pragma unroll
+                for (int s = 0; s < W; ++s) {
+                    int w = nb[s];
+                    bool fresh;
+                    if (enc)
+                        fresh = test_and_mark_enc(bm, nb[s], &w);
+                    else
+                        fresh = test_and_mark(bm, sm, w);
+                    if (fresh) {
+                        if (w < t0) {
+                            newm |= 1u << s;
+                            nb[s] = w;
+                        } else if (w > i) {
+                            ++a.ucnt;
+                            a.lmax = max(a.lmax, w);
+                        }
+                    }
+                }
+            }
+        }
+        // the new frontier vertices, one per lane per round
+        for (;;) {
+            const bool has = newm != 0;
+            const unsigned b = __ballot_sync(kFull, has);
+            if (!b) break;
+            int v = 0;
+            if (has) {
+                const int s0 = __ffs(newm) - 1;
+                newm &= newm - 1;
+#pragma unroll
+                for (int s = 0; s < W; ++s)
+                    if (s == s0) v = nb[s];
+            }
+            ring_append(h, has, b, v, ring, R, head, tail, spool, pcap, pool, pend, nspill);
+        }
+        // heavy vertices (degree > W): one warp each, over A's CSR row
+        unsigned hm = __ballot_sync(kFull, valid && heavy);
+        while (hm) {
+            const int src = __ffs(hm) - 1;
+            hm &= hm - 1;
+            const int len = __shfl_sync(kFull, nb[1], src);
+            const int64_t off =
+                heavy_off(__shfl_sync(kFull, nb[2], src), __shfl_sync(kFull, nb[3], src));
+            if (lane == 0) atomicAdd(&h.te, (unsigned long long)len);
+            for (int eb = 0; eb < len; eb += 32) {
+                const int e = eb + lane;
+                bool fr = false;
+                int w = -1;
+                if (e < len) {
+                    w = __ldg(p.ci + off + e);
+                    if (test_and_mark(bm, sm, w)) {
+                        if (w < t0) {
+                            fr = true;
+                        } else if (w > i) {
+                            ++a.ucnt;
+                            a.lmax = max(a.lmax, w);
+                        }
+                    }
+                }
+                const unsigned b = __ballot_sync(kFull, fr);
+                if (b) ring_append(h, fr, b, w, ring, R, head, tail, spool, pcap, pool, pend, nspill);
+            }
+        }
+        // the m expanded vertices leave the count, their children join it (one update;
+        // children donated to the pool on the way were counted by ring_donate)
+        if (lane == 0 && pend != m) atomicAdd(&h.outst, pend - m);
+        pend = 0;
+    }
+    if (lane == 0) {
+        atomicAdd(&h.sv, nproc);
+        if (nspill) atomicAdd(&h.spills, nspill);
+    }
+    if (MODE == kCount && p.count_te) {
+#pragma unroll
+        for (int o = 16; o; o >>= 1) te_loc += __shfl_xor_sync(kFull, te_loc, o);
+        if (lane == 0 && te_loc) atomicAdd(&h.te, te_loc);
+    }
+    __syncthreads();
+    a.lmin = 0;  // marks somewhere below t0: clear from word 0 (summary walk)
+}
+
 // Level-synchronous BFS from threshold t0 over unvisited vertices < t0 (Alg. 1).
 // Level lev reads queue lev&1 and writes queue (lev+1)&1 (shared, spilling to the CTA's two
 // HBM halves); the level counters rotate through h.cnt[0..2] so one barrier per level suffices.
 // Queue and spill addresses are recomputed from the launch parameters each level rather than
 // carried in registers (at 32 registers per thread they would otherwise spill).
-template <int NT, int W, int VIS, int MODE>
+template <int NT, int W, int VIS, int MODE, bool ASYNC>
 __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_t *sm, int32_t *qA,
                     const int i, const int t0, RowAcc &a)
 {
+    if constexpr (ASYNC) {
+        if (p.aring) {
+            bfs_async<NT, W, VIS, MODE>(p, h, bm, sm, qA, i, t0, a);
+            return;
+        }
+    }
     const int tid = threadIdx.x;
     if (tid == 0) {
         qA[0] = t0;
@@ -1135,7 +1391,7 @@ __global__ void __launch_bounds__(NtCfg<KEY>::NT, NtCfg<KEY>::MINB)
             if (nptr <= ptr) __syncthreads();
             PH_MARK(ph_win);
             if (m <= last && m == tns) {  // smallest pending threshold: below-exploration
-                bfs<NT, W, VIS, MODE>(p, h, bm, sm, qA, i, m, a);
+                bfs<NT, W, VIS, MODE, (KEY == 1025)>(p, h, bm, sm, qA, i, m, a);
                 ++n_bfs;
             }
             cap = m <= last ? min(cap, kSmallWin) : min(2 * cap, p.wcap);

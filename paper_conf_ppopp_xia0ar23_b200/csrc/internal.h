@@ -73,6 +73,11 @@ struct Fill2Params {
     int32_t defer_win = 0, defer_from = 0, defer_max = 0;
     int32_t *defer_list = nullptr;
     unsigned long long *defer_cnt = nullptr;
+    // below-threshold traversal without level barriers (bfs_async): ring entries per warp in
+    // the frontier queues' shared memory (a power of two >= 64); 0 = level-synchronous BFS
+    int32_t aring = 0;
+    int32_t akeep = 32;    // bfs_async: entries a warp keeps when it donates to idle warps
+    int32_t asleep = 1500; // bfs_async: ns an idle warp sleeps between polls of the pool
 };
 enum Fill2Mode { kCount = 0, kEmit = 1, kStage = 2 };
 // row_off value of a row deferred to the row-merge tail and not finished yet

@@ -283,6 +283,21 @@ void free_handle(lu_sym *h)
 #define LUSYM_KLOC_OCC 2
 #endif
 
+// classes with at most this many rows per SM run the asynchronous BFS (LUSYM_ASYNC_OCC: A/B)
+const int g_async_occ = [] {
+    const char *e = getenv("LUSYM_ASYNC_OCC");
+    return e ? atoi(e) : 0;
+}();
+
+const int g_async_keep = [] {  // LUSYM_ASYNC_KEEP: A/B knob (entries kept when donating)
+    const char *e = getenv("LUSYM_ASYNC_KEEP");
+    return e ? std::max(1, std::min(atoi(e), 64)) : 32;
+}();
+const int g_async_sleep = [] {  // LUSYM_ASYNC_SLEEP: A/B knob (ns between pool polls)
+    const char *e = getenv("LUSYM_ASYNC_SLEEP");
+    return e ? atoi(e) : 1500;
+}();
+
 struct Cfg {
     int nt, q, occ;
     size_t smem;
@@ -732,6 +747,20 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
                   !(h->opts.flags & LU_F_NO_SELF_CONT))
                      ? LUSYM_KLOC
                      : 0;
+        // rows with the SM (nearly) to themselves: BFS without level barriers (bfs_async),
+        // its per-warp rings carved out of the class's two frontier queues
+        // (compiled into the 1024-thread one-CTA-per-SM kernel only: at 32 registers per
+        // thread it would spill in the other kernels' hot loops)
+        p.aring = 0;
+        if (c.nt == 1025 && !(h->opts.flags & LU_F_NO_ASYNC_BFS) &&
+            (c.occ <= g_async_occ || (h->opts.flags & LU_F_ASYNC_BFS))) {
+            const int nwarps = (c.nt > 1024 ? 1024 : c.nt) / 32;
+            int r = 1024;
+            while (r > c.q / nwarps) r >>= 1;  // rings: half the queues; pool: the rest
+            if (r >= 64) p.aring = r;
+            p.akeep = g_async_keep;
+            p.asleep = g_async_sleep;
+        }
         if ((h->opts.flags & LU_F_PAPER_CHUNKS) && !row_list) {
             // Alg. 3 / Alg. 4 as printed: chunk_size = L / (c n) rows per launch (c = 6 words of
             // 4 B per vertex, L = scratch budget, reading R16), launches in increasing row order

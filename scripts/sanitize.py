@@ -31,7 +31,9 @@ def hubs(n=600, k=4, deg=200):
 cases = [("lap2d16", gen.lap2d(16)), ("lap3d7", gen.lap3d(7)), ("circuit24", gen.circuit(24, 1)),
          ("hubs", hubs())]
 knobs = [dict(), dict(defer_windows=1), dict(flags=lu.F_FORCE_CLASSES, queue_capacity=32),
-         dict(flags=lu.F_GLOBAL_BITMAP), dict(flags=lu.F_TWO_PASS)]
+         dict(flags=lu.F_GLOBAL_BITMAP), dict(flags=lu.F_TWO_PASS),
+         dict(threads_per_row=1025, flags=lu.F_ASYNC_BFS, queue_capacity=2048),
+         dict(threads_per_row=1025, flags=lu.F_ASYNC_BFS | lu.F_GLOBAL_BITMAP)]
 ok = True
 for name, (rp, ci) in cases:
     ref = oracle.fill2(rp, ci)

@@ -139,6 +139,14 @@ KNOBS = [
     dict(threads_per_row=128), dict(threads_per_row=512), dict(threads_per_row=1024),
     dict(threads_per_row=1025),                      # 1024 threads, one-CTA-per-SM registers
     dict(threads_per_row=1025, queue_capacity=32, flags=lu.F_FORCE_CLASSES),
+    # bfs_async (warp rings + CTA pool, no level barriers) and the level-synchronous BFS on
+    # the one-CTA-per-SM kernel; 2048-entry queues give 64-entry rings: constant donations
+    dict(threads_per_row=1025, flags=lu.F_NO_ASYNC_BFS),
+    dict(threads_per_row=1025, flags=lu.F_ASYNC_BFS, queue_capacity=2048),
+    dict(threads_per_row=1025, flags=lu.F_ASYNC_BFS | lu.F_GLOBAL_BITMAP),
+    dict(threads_per_row=1025, flags=lu.F_ASYNC_BFS | lu.F_FORCE_CLASSES, queue_capacity=2048),
+    dict(threads_per_row=1025, flags=lu.F_ASYNC_BFS | lu.F_TWO_PASS, ell_width=4),
+    dict(threads_per_row=1025, flags=lu.F_ASYNC_BFS | lu.F_NO_BATCH),
     dict(ell_width=4), dict(ell_width=6), dict(ell_width=8),
     dict(flags=lu.F_GLOBAL_BITMAP, queue_capacity=32, rows_in_flight=5),
     dict(flags=lu.F_NO_PRUNE), dict(flags=lu.F_KAHN_WIDE_ONLY), dict(flags=lu.F_NO_CONTRACT),
@@ -658,7 +666,8 @@ def test_deferred_rows_across_shards(defer_windows):
 
 @pytest.mark.parametrize("knob", [dict(), dict(flags=lu.F_NO_BATCH), dict(flags=lu.F_SELF_CONT),
                                   dict(flags=lu.F_GLOBAL_BITMAP), dict(flags=lu.F_FORCE_CLASSES),
-                                  dict(queue_capacity=32), dict(threads_per_row=1024)], ids=str)
+                                  dict(queue_capacity=32), dict(threads_per_row=1024),
+                                  dict(threads_per_row=1025, queue_capacity=2048)], ids=str)
 def test_stats_are_the_methods_work_units(knob):
     """The library's own counters are the method's work (reading R24): scanned
     vertices (every threshold once + every BFS vertex) and, with F_COUNT_TE, traversed edges
