@@ -54,6 +54,9 @@ namespace f2 {
 #ifndef LUSYM_WARP_EXIT  // warps past the end of a BFS level / threshold window leave early
 #define LUSYM_WARP_EXIT 0  // A/B: +1.6..6.9% slower (profiles/r02/ab_wexit.log)
 #endif
+#ifndef LUSYM_ROUNDS  // scan_level (encoded neighbours): batch visited test, then atomics in
+#define LUSYM_ROUNDS 0    // warp-uniform rounds of one candidate per lane (A/B: 12-17% slower)
+#endif
 #ifndef LUSYM_TAM  // test_and_mark with one shared bit mask (0: visited() then mark())
 #define LUSYM_TAM 1
 #endif
@@ -299,6 +302,25 @@ __device__ __forceinline__ bool test_and_mark_enc(const VisMap<VIS> &m, int e, i
     asm volatile("ld.shared.u32 %0, [%1+%2];" : "=r"(word) : "r"(off), "n"(kBmShared) : "memory");
     const uint32_t b = 1u << (e & 31);
     if (word & b) return false;
+    uint32_t old;
+    asm volatile("atom.shared.or.b32 %0, [%1+%2], %3;"
+                 : "=r"(old) : "r"(off), "n"(kBmShared), "r"(b) : "memory");
+    if (old & b) return false;
+    const int x = dec_slot(e);
+    *v = x;
+    if (old == 0)
+        asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(summary_saddr(m) + (uint32_t)(x >> 10) * 4u),
+                     "r"(1u << ((x >> 5) & 31))
+                     : "memory");
+    return true;
+}
+
+// the set half of test_and_mark_enc (the bit looked clear): true iff this call set it
+template <int VIS>
+__device__ __forceinline__ bool set_enc(const VisMap<VIS> &m, int e, int *v)
+{
+    const uint32_t off = (uint32_t)e >> 5;
+    const uint32_t b = 1u << (e & 31);
     uint32_t old;
     asm volatile("atom.shared.or.b32 %0, [%1+%2], %3;"
                  : "=r"(old) : "r"(off), "n"(kBmShared), "r"(b) : "memory");
@@ -569,12 +591,24 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
         // the BFS source); further ones (rare) are appended one by one
         int c = 0, f0 = 0, f1 = 0, f2 = 0;
         const bool enc = LUSYM_ENC_ELL && VIS == kVisSmem && p.elle != nullptr;
+        uint32_t um = 0;  // LUSYM_ROUNDS: slots whose neighbour looked unvisited
         if (valid) {
             load_nb<W>(enc ? p.elle : p.ell, f, nb);
             heavy = nb[0] == kHeavy;
             if constexpr (MODE == kCount)  // the statistics pass only (LU_F_COUNT_TE)
                 if (p.count_te && !heavy) te_loc += row_edges<W>(nb, enc ? enc_vertex(f) : f);
-            if (enc && !heavy) {
+            if (enc && !heavy && LUSYM_ROUNDS) {
+                // every slot's visited bit first (straight-line, no branch per slot); the
+                // candidates are test-and-set after this block in warp-uniform rounds
+#pragma unroll
+                for (int s = 0; s < W; ++s) {
+                    uint32_t word;
+                    asm volatile("ld.shared.u32 %0, [%1+%2];"
+                                 : "=r"(word) : "r"((uint32_t)nb[s] >> 5), "n"(kBmShared)
+                                 : "memory");
+                    um |= (((word >> (nb[s] & 31)) & 1u) ^ 1u) << s;
+                }
+            } else if (enc && !heavy) {
 #pragma unroll
                 for (int s = 0; s < W; ++s) {
                     int w;
@@ -617,6 +651,36 @@ __device__ __forceinline__ void scan_level(const Fill2Params &p, Hdr &h, const V
                     const int w = nb[s];
                     if ((um >> s & 1u) &&
                         (LUSYM_BATCH_TEST ? mark(bm, sm, w) : test_and_mark(bm, sm, w))) {
+                        if (w < t0) {
+                            if (c == 3) {
+                                put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);
+                            } else {
+                                f2 = f1;
+                                f1 = f0;
+                                f0 = w;
+                                ++c;
+                            }
+                        } else if (w > i) {
+                            ++a.ucnt;
+                            a.lmax = max(a.lmax, w);
+                        }
+                    }
+                }
+            }
+        }
+        if (LUSYM_ROUNDS && enc) {
+            // the candidates, one per lane per round: the atomic path is issued once per round
+            // for the warp instead of once per slot
+            while (__any_sync(kFull, um != 0)) {
+                if (um) {
+                    const int s0 = __ffs(um) - 1;
+                    um &= um - 1;
+                    int e = nb[0];
+#pragma unroll
+                    for (int s = 1; s < W; ++s)
+                        if (s == s0) e = nb[s];
+                    int w;
+                    if (set_enc(bm, e, &w)) {
                         if (w < t0) {
                             if (c == 3) {
                                 put(atomicAdd(ncnt, 1), w, NF, gNF, p.q);

@@ -17,7 +17,7 @@ PHASES = [("---- seed", "kernel: seed"), ("---- thresholds in increasing order",
 
 def main():
     out = subprocess.run(["ncu", "-i", sys.argv[1], "--page", "source", "--csv",
-                          "--print-source", "cuda"], capture_output=True, text=True).stdout
+                          "--print-source", "cuda,sass"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(out)))
     hdr, fname, acc = None, "", {}
     tot_i = tot_s = 0.0
@@ -31,8 +31,8 @@ def main():
         elif r[0] == "Line No":
             hdr = r
         elif hdr and r[0].isdigit():
-            d = dict(zip(hdr, r))
-            src = d.get("Source", "")
+            d = dict(zip(hdr[2:], r[2:]))
+            src = r[1]
             if fname == "fill2_impl.cuh":
                 m = DEF.match(src.strip())
                 if m and not src.startswith(" "):
