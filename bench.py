@@ -38,6 +38,7 @@ from inputs import gen  # noqa: E402
 METRIC = "fill entries/s"
 UNIT = "entries/s"
 L2_FLUSH_BYTES = 256 << 20
+E2E_BOUND_MAX_BYTES = 8 << 30  # e2e: use the capacity bound when its outputs stay under this
 
 
 def parse():
@@ -51,6 +52,8 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-two-call", action="store_true",
+                    help="e2e through the two-call protocol even when the capacity bound is usable")
     ap.add_argument("--e2e-host", default="pinned", choices=["pinned", "pageable"],
                     help="host output buffers of the e2e run (allocated inside the timed region)")
     ap.add_argument("--per-config", default="1,2,3,4,5",
@@ -645,7 +648,20 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
         mark("h2d")
         he = lu.Symbolic(rpd, cid, **sym_opts)                 # S1 + S2
         mark("create")
-        if world > 1:
+        cap = he.nnz_bound() if world == 1 and not args.e2e_two_call else -1
+        one_call = 0 <= cap and cap * 4 <= E2E_BOUND_MAX_BYTES
+        if one_call:
+            # capacity from A alone (Theorem 1 row envelopes): allocate the outputs first,
+            # then one call streams the pattern to the host behind the traversal
+            mark("capacity bound")
+            out_rp = torch.empty(n + 1, dtype=torch.int64, pin_memory=pinned)
+            out_ci = torch.empty(cap, dtype=torch.int32, pin_memory=pinned)
+            out_lv = torch.empty(n, dtype=torch.int32, pin_memory=pinned)
+            mark("alloc (host outputs)")
+            fc, rp_lu, ci_lu = he.run_host(cap, out_rp, out_ci)   # S3-S6 + D2H of the pattern
+            nz = int(ci_lu.numel())
+            mark("count+scan+emit+d2h(pattern), overlapped")
+        elif world > 1:
             fc, rp_lu, ci_lu = lu.sharded_pass(he, rb, re_, bounds)
             nz = int(ci_lu.numel())
             mark("count+scan+emit+exchange")
@@ -671,7 +687,8 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
         # engine), then the copies
         level, _ = he.levelize(rp_lu, ci_lu, args.rule)        # S8 + S9
         mark("levelize")
-        out_ci.copy_(ci_lu, non_blocking=pinned)
+        if not one_call:
+            out_ci.copy_(ci_lu, non_blocking=pinned)
         out_lv.copy_(level, non_blocking=pinned)
         b.record(stream)
         torch.cuda.synchronize()
@@ -689,7 +706,7 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
                 phases.setdefault(tag, []).append(prev.elapsed_time(e_))
                 prev = e_
         if verify is not None:
-            verify.host(out_rp.numpy(), out_ci.numpy(), out_lv.numpy())
+            verify.host(out_rp.numpy(), out_ci.numpy()[:nz], out_lv.numpy())
         del out_rp, out_ci, out_lv, ci_lu, rp_lu, fc
     t = torch.tensor([float(np.mean(e_ms))], dtype=torch.float64, device=dev)
     if world > 1:
@@ -704,7 +721,11 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
                              "call of the process is first_call)"
                              if pinned else "pageable, allocated inside the timed region"),
             "first_call": cold,
-            "mode": "two-call protocol: count + scan -> nnz -> allocate -> emit -> copies",
+            "mode": ("one call: outputs allocated from the a-priori capacity bound "
+                     "(lu_sym_nnz_bound, Theorem 1 row envelopes), then lu_sym_run_host streams "
+                     "the pattern to pinned host memory behind the traversal" if one_call else
+                     "two-call protocol: count + scan -> nnz -> allocate -> emit -> copies"),
+            "capacity_bound": cap if one_call else None,
             "parity": "host copies verified against the reference every step" if verify else None}
 
 

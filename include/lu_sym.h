@@ -239,6 +239,17 @@ lu_status lu_sym_run(lu_sym *h, int32_t *d_fill_count, int64_t *d_row_ptr_lu,
                      int32_t *d_col_idx_lu, int64_t cap, int64_t *nnz_lu, void *stream);
 
 /*
+ * A-priori capacity of the pattern from A alone (no traversal): *bound (host) >= nnz(L+U).
+ * By Theorem 1 ((i,j) fills iff a path i -> j has every intermediate vertex
+ * < min(i,j)), row i of L+U lies in [min(i, min A(i,:)), max(i, max over u <= i of
+ * max A(u,:))], and *bound is the sum of those row spans.  It is exact when every such span
+ * fills (banded matrices, e.g. natural-ordered grids) and loose when a late dense row or
+ * column widens the envelope (hub rows ordered last).  Lets a caller allocate the device and
+ * host outputs before lu_sym_run_host instead of after a count pass.  Synchronises.
+ */
+lu_status lu_sym_nnz_bound(lu_sym *h, int64_t *bound, void *stream);
+
+/*
  * Whole symbolic pass with the result streamed to the host while later rows are still being
  * traversed: Alg. 3's out-of-core chunks (L239-270) taken in INCREASING row order, nchunks row
  * ranges of equal a-priori traversal cost (0 => min(16, max(1, n/4096)); at most 64).  Per chunk: symbolic_1 with

@@ -92,7 +92,7 @@ EXPORTED = ["lu_sym_abi_version", "lu_sym_default_opts", "lu_sym_create", "lu_sy
             "lu_sym_destroy", "lu_status_str", "lu_last_error", "lu_sym_set_row_profile",
             "lu_level_schedule", "lu_sym_run_host", "lu_level_types", "lu_numeric_scatter",
             "lu_numeric_factor", "lu_sym_deferred_flags", "lu_sym_merge_deferred",
-            "lu_numeric_factor_ex"]
+            "lu_numeric_factor_ex", "lu_sym_nnz_bound"]
 
 
 def library_path() -> str:
@@ -117,6 +117,8 @@ def load_library():
     lib.lu_sym_emit.argtypes = [P, I32, I32, P, P, I64, P]
     lib.lu_sym_run.argtypes = [P, P, P, P, I64, P, P]
     lib.lu_sym_run_host.argtypes = [P, I32, P, P, P, I64, P, P, P, P]
+    lib.lu_sym_nnz_bound.argtypes = [P, P, P]
+    lib.lu_sym_nnz_bound.restype = I32
     lib.lu_levelize.argtypes = [P, I32, P, P, I32, P, P, P]
     lib.lu_sym_get_stats.argtypes = [P, P]
     lib.lu_sym_destroy.argtypes = [P]
@@ -293,6 +295,13 @@ class Symbolic:
             ctypes.byref(nnz), _stream_ptr(stream)))
         self.nnz_lu = int(nnz.value)
         return fc, rp_lu, ci_lu[: self.nnz_lu]
+
+    def nnz_bound(self, stream=None) -> int:
+        """A-priori capacity >= nnz(L+U) from A alone (lu_sym_nnz_bound: the Theorem 1 row
+        envelopes), for allocating run_host's outputs before the traversal."""
+        b = ctypes.c_int64(0)
+        _check(load_library().lu_sym_nnz_bound(self._h, ctypes.byref(b), _stream_ptr(stream)))
+        return int(b.value)
 
     # -- row sharding with deferred rows (F_DEFER_GLOBAL, reading G8 across GPUs)
     def deferred_flags(self, flags=None, stream=None):

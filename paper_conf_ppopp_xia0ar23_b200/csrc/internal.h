@@ -177,6 +177,10 @@ size_t scan_scratch_elems(int32_t n);
 cudaError_t count_far_entries(int32_t n, const int64_t *rp, const int32_t *ci, int32_t bound,
                               unsigned long long *d_cnt, cudaStream_t s);
 
+// bound_kernels.cu — a-priori capacity of L+U from A (Theorem 1 row envelopes); synchronises
+cudaError_t nnz_upper_bound(int32_t n, const int64_t *rp, const int32_t *ci, int64_t *h_bound,
+                            cudaStream_t s);
+
 // place_kernels.cu — symbolic_2 for staged rows: copy pool rows to their CSR slots
 cudaError_t place_rows(int32_t row_begin, int32_t row_end, const int64_t *rp_lu,
                        const int64_t *row_off, const int32_t *pool, int32_t *ci_lu,

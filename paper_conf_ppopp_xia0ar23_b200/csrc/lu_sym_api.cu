@@ -1302,6 +1302,20 @@ lu_status lu_sym_run(lu_sym *h, int32_t *d_fill_count, int64_t *d_row_ptr_lu,
     return lu_sym_emit(h, 0, h->n, d_row_ptr_lu, d_col_idx_lu, cap, stream);
 }
 
+lu_status lu_sym_nnz_bound(lu_sym *h, int64_t *bound, void *stream)
+{
+    nvtx3::scoped_range nvtx_range{"lu_sym_nnz_bound"};
+    g_err.clear();
+    if (!h || !bound) return fail(LU_ERR_ARG, "null pointer");
+    lu_status st = check_device(h);
+    if (st != LU_OK) return st;
+    cudaStream_t s = (cudaStream_t)stream;
+    h->stream = s;
+    CK(nnz_upper_bound(h->n, h->rp, h->ci, bound, s));
+    h->launches += h->n > 0 ? 4 : 0;
+    return LU_OK;
+}
+
 lu_status lu_sym_run_host(lu_sym *h, int32_t nchunks, int32_t *d_fill_count,
                           int64_t *d_row_ptr_lu, int32_t *d_col_idx_lu, int64_t cap,
                           int64_t *h_row_ptr_lu, int32_t *h_col_idx_lu, int64_t *nnz_lu,
