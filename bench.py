@@ -603,7 +603,7 @@ def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
     # the device-resident run's handle and outputs are released before the e2e run, as a
     # caller's earlier factorization would be: the e2e handle then reuses the memory the pool
     # keeps reserved instead of growing it (mapping new pages) while this one still holds its own
-    if headline:
+    if headline and world == 1 and not args.no_cpu_baseline:   # the CPU baseline's levels
         rec["_state"] = {"rp_lu": state["rp_lu"].cpu().numpy(),
                          "ci_lu": state["ci_lu"].cpu().numpy()}
     else:

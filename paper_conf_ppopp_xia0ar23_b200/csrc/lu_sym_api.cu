@@ -4,6 +4,7 @@
 
 #include <nvtx3/nvtx3.hpp>  // header-only: a named range per ABI call (for nsys / ncu)
 
+#include <chrono>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -298,6 +299,19 @@ const int g_async_sleep = [] {  // LUSYM_ASYNC_SLEEP: A/B knob (ns between pool 
     return e ? atoi(e) : 1500;
 }();
 
+// LUSYM_DEBUG_CREATE: host milliseconds of each create / plan step on stderr (diagnostic)
+const bool g_dbg_create = getenv("LUSYM_DEBUG_CREATE") != nullptr;
+std::chrono::steady_clock::time_point g_tc;
+void dbg_lap(cudaStream_t s, const char *what)
+{
+    if (!g_dbg_create) return;
+    cudaStreamSynchronize(s);
+    const auto now = std::chrono::steady_clock::now();
+    fprintf(stderr, "lusym create: %-14s %8.3f ms\n", what,
+            std::chrono::duration<double, std::milli>(now - g_tc).count());
+    g_tc = now;
+}
+
 struct Cfg {
     int nt, q, occ;
     size_t smem;
@@ -465,6 +479,7 @@ lu_status plan(lu_sym *h)
             lbw = want;
         }
     }
+    dbg_lap(h->stream, "plan: top cfg");
     // lower row classes (Alg. 4): halve the shared part while that adds rows in flight
     h->classes.clear();
     int hi = n;
@@ -507,6 +522,7 @@ lu_status plan(lu_sym *h)
         h->classes.push_back(RowClass{0, hi, vis, sw_words, vis == kVisGlobal ? 0 : sw_words,
                                       cur.nt, cur.q, cur.occ, cur.smem});
     }
+    dbg_lap(h->stream, "plan: classes");
     size_t free_b = 0, total_b = 0;
     CK(cudaMemGetInfo(&free_b, &total_b));
     const uint64_t budget = h->opts.scratch_budget_bytes ? h->opts.scratch_budget_bytes
@@ -556,6 +572,7 @@ lu_status plan(lu_sym *h)
             }
         }
     }
+    dbg_lap(h->stream, "plan: sparse");
     // HBM budget: everything the handle allocates stays within scratch_budget_bytes.
     // Per row in flight: frontier spill (2 x cap) + L staging (cap) + done map (+ the HBM
     // visited slot); cap = rows of the class (a row's frontier and L part lie below i).  Every
@@ -600,6 +617,7 @@ lu_status plan(lu_sym *h)
     }
     h->grid = max_grid;
     h->map_words = (int64_t)need_map;
+    dbg_lap(h->stream, "plan: budget");
     if ((st = salloc(h, &h->gspill, need_spill)) != LU_OK) return st;
     if (need_hbm_map && (st = salloc(h, &h->gbitmap, need_map)) != LU_OK) return st;
     if ((st = salloc(h, &h->dbitmap, need_map)) != LU_OK) return st;
@@ -613,6 +631,7 @@ lu_status plan(lu_sym *h)
         if ((st = salloc(h, &h->row_off, (size_t)n)) != LU_OK) return st;
         if ((st = salloc(h, &h->ucut, (size_t)n)) != LU_OK) return st;
     }
+    dbg_lap(h->stream, "plan: alloc");
     // deferred rows (reading G8)
     {
         const int dw = h->opts.defer_windows, dm = h->opts.defer_max;
@@ -1065,6 +1084,8 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
     if (cudaEventCreate(&t0) != cudaSuccess || cudaEventCreate(&t1) != cudaSuccess)
         return bail(fail(LU_ERR_CUDA, "cudaEventCreate failed"));
     cudaEventRecord(t0, s);
+    g_tc = std::chrono::steady_clock::now();
+    auto lap = [&](const char *what) { dbg_lap(s, what); };
     if ((st = dalloc(h, &h->dstats, kStatSlots)) != LU_OK) return bail(st);
     if ((st = dalloc(h, &h->dbad, 2)) != LU_OK) return bail(st);
     if ((st = dalloc(h, &h->scan_blk, scan_scratch_elems(n))) != LU_OK) return bail(st);
@@ -1086,6 +1107,7 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
                              (long long)(bad >> 8), what[code < 6 ? code : 0]));
         }
     }
+    lap("validate");
     if (n == 0) {
         cudaEventDestroy(t0);
         cudaEventDestroy(t1);
@@ -1108,6 +1130,7 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
             if (cand == 8 || light >= (unsigned long long)(0.995 * n)) w = cand;
         }
         h->w = w;
+        lap("ell width");
         if ((st = dalloc(h, &h->ell, (size_t)n * (w <= 4 ? 4 : 8))) != LU_OK) return bail(st);
         cudaError_t e = build_ell(n, d_row_ptr, d_col_idx, w, h->ell, s);
         if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
@@ -1128,7 +1151,9 @@ lu_status lu_sym_create(lu_sym **out, int32_t n, int64_t nnz_a, const int64_t *d
             if (e != cudaSuccess) return bail(fail(LU_ERR_CUDA, "%s", cudaGetErrorString(e)));
         }
     }
+    lap("ell build");
     if ((st = plan(h)) != LU_OK) return bail(st);
+    lap("plan");
     cudaEventRecord(t1, s);
     if (cudaEventSynchronize(t1) != cudaSuccess)
         return bail(fail(LU_ERR_CUDA, "create: %s", cudaGetErrorString(cudaGetLastError())));
