@@ -299,6 +299,17 @@ const int g_async_sleep = [] {  // LUSYM_ASYNC_SLEEP: A/B knob (ns between pool 
     return e ? atoi(e) : 1500;
 }();
 
+// LUSYM_HEAVY_TOP / LUSYM_HEAVY_GRID (A/B knobs): the last rows in a shared-map class next
+// to the sparse class, and that class's rows in flight
+const int g_heavy_top = [] {
+    const char *e = getenv("LUSYM_HEAVY_TOP");
+    return e ? atoi(e) : 0;
+}();
+const int g_heavy_grid = [] {
+    const char *e = getenv("LUSYM_HEAVY_GRID");
+    return e ? atoi(e) : 0;
+}();
+
 // LUSYM_DEBUG_CREATE: host milliseconds of each create / plan step on stderr (diagnostic)
 const bool g_dbg_create = getenv("LUSYM_DEBUG_CREATE") != nullptr;
 std::chrono::steady_clock::time_point g_tc;
@@ -561,6 +572,7 @@ lu_status plan(lu_sym *h)
             if (force) sv = 0;
             h->sparse_sv = sv;
             if (sv >= 0 && sv < (double)n / 16) {
+                const RowClass top0 = h->classes.front();
                 h->classes.erase(h->classes.begin(), h->classes.begin() + (long)kc);
                 h->classes.insert(h->classes.begin(),
                                   RowClass{lo, n, kVisGlobal, 0, 0, g.nt, g.q, g.occ, g.smem});
@@ -569,6 +581,17 @@ lu_status plan(lu_sym *h)
                 h->classes.front().defer_win = kSparseDeferWindows;
                 if (const char *e = getenv("LUSYM_SPARSE_DEFER_WINDOWS"))  // A/B knob
                     h->classes.front().defer_win = atoi(e);
+                // heavy top rows (the last separators of a nested-dissection order scan a large
+                // part of the graph): back to the shared-map top class (A/B knob)
+                const int heavy = g_heavy_top;
+                if (heavy > 0 && heavy < n - lo && top0.vis == kVisSmem) {
+                    RowClass t = top0;
+                    t.lo = n - heavy;
+                    t.hi = n;
+                    t.defer_win = h->classes.front().defer_win;
+                    h->classes.front().hi = n - heavy;
+                    h->classes.insert(h->classes.begin(), t);
+                }
             }
         }
     }
@@ -603,6 +626,9 @@ lu_status plan(lu_sym *h)
         int64_t grid = (int64_t)sms * c.occ;
         if (h->opts.rows_in_flight > 0 && h->opts.rows_in_flight < grid)
             grid = h->opts.rows_in_flight;
+        if (k == 0 && g_heavy_top > 0 && g_heavy_grid > 0 && h->classes.size() > 1 &&
+            h->classes[1].vis == kVisGlobal && g_heavy_grid < grid)
+            grid = g_heavy_grid;
         const int64_t extra = std::min<int64_t>(grid - 1, (int64_t)(have / per_row[k]));
         c.grid = (int)(1 + std::max<int64_t>(extra, 0));
         have -= (uint64_t)(c.grid - 1) * per_row[k];
