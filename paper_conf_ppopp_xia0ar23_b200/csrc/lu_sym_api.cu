@@ -310,6 +310,13 @@ const int g_heavy_grid = [] {
     return e ? atoi(e) : 0;
 }();
 
+// class boundaries at the largest shared map that adds rows in flight (LUSYM_TIGHT_CLASSES=0:
+// halve the map per class instead, round 1's ladder)
+const bool g_tight_classes = [] {
+    const char *e = getenv("LUSYM_TIGHT_CLASSES");
+    return e ? atoi(e) != 0 : true;
+}();
+
 // LUSYM_DEBUG_CREATE: host milliseconds of each create / plan step on stderr (diagnostic)
 const bool g_dbg_create = getenv("LUSYM_DEBUG_CREATE") != nullptr;
 std::chrono::steady_clock::time_point g_tc;
@@ -491,7 +498,8 @@ lu_status plan(lu_sym *h)
         }
     }
     dbg_lap(h->stream, "plan: top cfg");
-    // lower row classes (Alg. 4): halve the shared part while that adds rows in flight
+    // lower row classes (Alg. 4): shrink the shared part to the largest one that adds rows in
+    // flight (a binary search over whole swizzle groups; or halve it), while that adds rows
     h->classes.clear();
     int hi = n;
     const bool one_class = (h->opts.flags & LU_F_ONE_CLASS) != 0;
@@ -499,6 +507,24 @@ lu_status plan(lu_sym *h)
         int nl = (lbw / 2 + 31) / 32 * 32;
         if (nl < 64 || nl >= lbw) break;
         Cfg c;
+        if (g_tight_classes && vis != kVisGlobal && !(h->opts.flags & LU_F_FORCE_CLASSES)) {
+            // the largest shared part (whole swizzle groups) that adds rows in flight, instead
+            // of half of the current one (occupancy only grows as the part shrinks): cfg4
+            // 8,505 -> 7,337 ms (profiles/r02/ab_tight_classes.log)
+            int ulo = 2, uhi = lbw / 32 - 1, best_u = 0;
+            while (ulo <= uhi) {
+                const int um = (ulo + uhi) / 2;
+                Cfg t;
+                if ((st = best_cfg(h, um * 32, kVisSplit, smem_optin, &t)) != LU_OK) return st;
+                if (t.key >= 0 && t.occ > cur.occ) {
+                    best_u = um;
+                    ulo = um + 1;
+                } else {
+                    uhi = um - 1;
+                }
+            }
+            if (best_u) nl = best_u * 32;
+        }
         if ((st = best_cfg(h, nl, kVisSplit, smem_optin, &c)) != LU_OK) return st;
         if (c.key < 0) {
             if (vis != kVisGlobal) break;
