@@ -107,6 +107,18 @@ struct MergeParams {
     unsigned long long *fail_cnt;
     unsigned long long *stats;         // [0] U entries read, [1] rounds, [2] waits
     int32_t q;                         // shared frontier capacity per buffer
+    // grid-wide mode (k_merge_grid): the whole GPU finishes the deferred rows one at a time in
+    // increasing order when there are at most grid_max of them (0: never)
+    int32_t grid_max = 0;
+    uint32_t *gbits = nullptr;         // [ceil(n/32)] visited bitmap of the row in progress
+    int32_t *gq = nullptr;             // [2 n] frontier buffers
+    long long *glen = nullptr;         // [n] U segment length of each frontier member
+    long long *goff = nullptr;         // [n] its pool offset
+    long long *gstart = nullptr;       // [n + 64] flat start of each non-empty segment (compacted)
+    long long *gcoff = nullptr;        // [n] its pool offset (compacted)
+    long long *gpart = nullptr;        // [4 * grid + 8] per-CTA partial sums, the row's pool offset
+    int32_t *gctrl = nullptr;          // [16] counters
+    int32_t grid_filter = 0;           // shared-memory filter words per CTA (0: none)
 };
 // mode 0: one CTA per row, bitmap in shared memory; 1: one CTA, bitmap in an HBM slot;
 // 2: a cluster of g CTAs per row, bitmap sliced over their shared memories (DSMEM)
@@ -118,6 +130,11 @@ cudaError_t merge_sort_list(int32_t *list, const unsigned long long *cnt, int32_
                             cudaStream_t s);
 cudaError_t merge_launch(const MergeParams &p, int mode, int g, int grid, size_t smem,
                          cudaStream_t s);
+// the grid-wide mode: one cooperative launch of *grid CTAs (set by merge_grid_size); it does
+// nothing when the list holds more than p.grid_max rows, else it finishes them all and marks
+// the list claimed so that the cluster kernel launched after it exits at once
+cudaError_t merge_grid_size(int n, int *grid, int *filter_words);
+cudaError_t merge_grid_launch(const MergeParams &p, int grid, cudaStream_t s);
 // row sharding with deferred rows (LU_F_DEFER_GLOBAL)
 cudaError_t zero_deferred_counts(const int32_t *list, const unsigned long long *cnt, int32_t max,
                                  int32_t *fill_count, cudaStream_t s);

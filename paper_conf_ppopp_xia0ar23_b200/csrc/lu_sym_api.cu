@@ -90,6 +90,11 @@ struct RowClass {
 };
 
 struct lu_sym {
+    // grid-wide tail (k_merge_grid) for lists of at most mg_max deferred rows
+    int mg_max = 0, mg_grid = 0, mg_filter = 0;
+    uint32_t *mg_bits = nullptr;
+    int32_t *mg_q = nullptr, *mg_ctrl = nullptr;
+    long long *mg_ll = nullptr;
     int32_t n = 0;
     int64_t nnz_a = 0;
     const int64_t *rp = nullptr;
@@ -231,7 +236,7 @@ void free_handle(lu_sym *h)
     void *bufs[] = {h->ell,        h->elle,      h->gbitmap, h->dbitmap, h->gspill, h->dstats,
                     h->scan_blk,   h->dbad,      h->stg,     h->pool,   h->row_off,
                     h->unstaged,   h->ucut,      h->defer_list, h->fail_list, h->mspill,
-                    h->mwait,      h->mgbitmap};
+                    h->mwait,      h->mgbitmap, h->mg_bits, h->mg_q, h->mg_ll, h->mg_ctrl};
     if (!h->managed.empty()) cudaStreamSynchronize(s);
     std::vector<void *> all(std::begin(bufs), std::end(bufs));
     for (int k = 1; k < kSets; ++k)
@@ -1004,6 +1009,34 @@ lu_status ensure_merge(lu_sym *h)
         if ((st = salloc(h, &h->mgbitmap, (size_t)grid * (size_t)words)) != LU_OK) return st;
         CK(cudaMemsetAsync(h->mgbitmap, 0, (size_t)grid * (size_t)words * 4, h->stream));
     }
+    // the grid-wide mode for short lists (k_merge_grid): whole-GPU scratch
+    // LUSYM_MERGE_GRID_MAX (A/B knob, off by default): deferred-row lists of at most that many
+    // rows are finished by the whole grid, one row at a time (k_merge_grid), instead of by
+    // 4-CTA clusters in parallel.  Measured on cfg3's 32 hubs: 19.1 ms against 17.4 (396
+    // rounds; the per-round phases and grid barriers cost what the extra SMs save).
+    h->mg_max = 0;
+    if (const char *e = getenv("LUSYM_MERGE_GRID_MAX")) h->mg_max = atoi(e);
+    if (h->mg_max > 0 && merge_grid_size(n, &h->mg_grid, &h->mg_filter) == cudaSuccess &&
+        h->mg_grid > 0) {
+        const size_t need = (size_t)words * 4 + (size_t)2 * n * 4 + (size_t)4 * n * 8 + 64 * 8 +
+                            ((size_t)4 * h->mg_grid + 8) * 8 + 64;
+        const uint64_t left2 = h->budget > (uint64_t)h->scratch_bytes
+                                   ? h->budget - (uint64_t)h->scratch_bytes : 0;
+        if (need <= left2) {
+            if ((st = salloc(h, &h->mg_bits, (size_t)words)) != LU_OK) return st;
+            if ((st = salloc(h, &h->mg_q, (size_t)2 * n)) != LU_OK) return st;
+            if ((st = salloc(h, &h->mg_ll, (size_t)4 * n + 64 + 4 * (size_t)h->mg_grid + 8)) !=
+                LU_OK)
+                return st;
+            if ((st = salloc(h, &h->mg_ctrl, 16)) != LU_OK) return st;
+            CK(cudaMemsetAsync(h->mg_bits, 0, (size_t)words * 4, h->stream));
+        } else {
+            h->mg_max = 0;
+        }
+    } else {
+        cudaGetLastError();
+        h->mg_max = 0;
+    }
     return LU_OK;
 }
 
@@ -1054,6 +1087,23 @@ lu_status run_tail_list(lu_sym *h, int32_t *fill_count, const int32_t *list,
     mp.fail_cnt = slots + 2;
     mp.stats = slots + 3;
     mp.q = h->merge_q;
+    if (h->mg_max > 0) {
+        // a short list: the whole grid, one row at a time (k_merge_grid); a longer one is left
+        // to the clusters (the kernel checks the device-side count)
+        const size_t n = (size_t)h->n;
+        mp.grid_max = h->mg_max;
+        mp.gbits = h->mg_bits;
+        mp.gq = h->mg_q;
+        mp.glen = h->mg_ll;
+        mp.goff = h->mg_ll + n;
+        mp.gcoff = h->mg_ll + 2 * n;
+        mp.gstart = h->mg_ll + 3 * n;
+        mp.gpart = h->mg_ll + 4 * n + 64;
+        mp.gctrl = h->mg_ctrl;
+        mp.grid_filter = h->mg_filter;
+        CK(merge_grid_launch(mp, h->mg_grid, s));
+        h->launches += 1;
+    }
     CK(merge_launch(mp, h->merge_mode, h->merge_g, h->merge_grid, h->merge_smem, s));
     h->launches += 2;
     lu_status st = run_pass(h, kStage, 0, h->n, fill_count, nullptr, nullptr, s, fail_list, 0,

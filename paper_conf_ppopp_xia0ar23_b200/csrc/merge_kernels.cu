@@ -25,6 +25,7 @@
 #include "internal.h"
 
 #include <climits>
+#include <cstdio>
 #include <cooperative_groups.h>
 #include <map>
 #include <mutex>
@@ -39,6 +40,9 @@ constexpr int NT = kMergeNT;
 constexpr int NW = NT / 32;
 #ifndef LUSYM_MERGE_KU
 #define LUSYM_MERGE_KU 4
+#endif
+#ifndef LUSYM_MERGE_PROF
+#define LUSYM_MERGE_PROF 0
 #endif
 constexpr int kU = LUSYM_MERGE_KU;  // pool loads in flight per thread
 constexpr int kSent = 64;  // sentinel starts past the last segment
@@ -449,6 +453,393 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
     }
 }
 
+// ---- grid-wide mode (k_merge_grid): when only a few rows were deferred (cfg3: its 32 hubs),
+// the clusters above finish them one after another anyway (each hub's closure contains the
+// hubs below it), each on 4 SMs.  Here the whole grid takes the rows one at a time, in
+// increasing order, so every deferred row below i is finished before i starts and nothing
+// waits: the frontier's U segments are read by every SM (the step is a stream of pool reads)
+// and test-and-set goes to one visited bitmap in HBM (L2-resident, n bits).  Grid barriers
+// separate the phases: seed, then per round (lengths -> compaction -> expansion), then the
+// output (popcounts -> pool offset -> sorted write).
+
+__device__ __forceinline__ bool tas_g(uint32_t *bits, int v)
+{
+    const uint32_t b = 1u << (v & 31);
+    uint32_t *w = bits + (v >> 5);
+    if (__ldcg(w) & b) return false;
+    return !(atomicOr(w, b) & b);
+}
+
+// ... behind a per-CTA filter in shared memory (fw words, 0: none): bits are only ever set
+// during a row, so a bit this CTA has seen set (in the filter) is set; a miss reads the global
+// word and keeps every bit it holds.  Nearly every pool entry of a hub's closure is a member
+// already found (cfg3: 1.3e9 entries read for 2.7e7 members), so most tests end in shared memory.
+__device__ __forceinline__ bool tas_f(uint32_t *bits, uint32_t *filt, bool use, int v)
+{
+    const uint32_t b = 1u << (v & 31);
+    const int w = v >> 5;
+    if (use && (filt[w] & b)) return false;
+    const uint32_t g = __ldcg(bits + w);
+    bool fresh = false;
+    uint32_t now = g;
+    if (!(g & b)) {
+        const uint32_t old = atomicOr(bits + w, b);
+        fresh = !(old & b);
+        now = old | b;
+    }
+    if (use) atomicOr(filt + w, now);
+    return fresh;
+}
+
+// warp-aggregated append to a global frontier list
+__device__ __forceinline__ void gpush(bool pred, int32_t v, int32_t *cnt, int32_t *list)
+{
+    const unsigned b = __ballot_sync(0xffffffffu, pred);
+    if (!b) return;
+    const int lane = threadIdx.x & 31, leader = __ffs(b) - 1;
+    int base = 0;
+    if (lane == leader) base = atomicAdd(cnt, __popc(b));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    if (pred) list[base + __popc(b & ((1u << lane) - 1u))] = v;
+}
+
+__device__ __forceinline__ int ld_cg_int(const int32_t *p) { return __ldcg(p); }
+
+// new frontier members of this CTA, collected in shared memory and appended to the global
+// list with one atomic per CTA per phase (a single global counter hit by every warp of the
+// grid serialises at its L2 slice); past kGBuf entries a warp appends directly
+constexpr int kGBuf = 4096;
+struct GBuf {
+    int32_t v[kGBuf];
+    int cnt, base;
+};
+// segments staged for the expansion (starts with kSent look-ahead entries, pool offsets)
+constexpr int kGSeg = 1024;
+struct GSeg {
+    long long st[kGSeg + kSent];
+    long long off[kGSeg + kSent];
+    int m;
+};
+
+__device__ __forceinline__ void gbuf_push(bool pred, int32_t v, GBuf &sb, int32_t *cnt,
+                                          int32_t *list)
+{
+    const unsigned b = __ballot_sync(0xffffffffu, pred);
+    if (!b) return;
+    const int lane = threadIdx.x & 31, leader = __ffs(b) - 1;
+    int base = 0;
+    if (lane == leader) base = atomicAdd(&sb.cnt, __popc(b));
+    base = __shfl_sync(0xffffffffu, base, leader);
+    const int slot = base + __popc(b & ((1u << lane) - 1u));
+    if (pred && slot < kGBuf) sb.v[slot] = v;
+    gpush(pred && slot >= kGBuf, v, cnt, list);  // the part past the buffer, directly
+}
+
+// append the CTA's collected members to the global list (block-uniform; ends with a barrier)
+__device__ __forceinline__ void gbuf_flush(GBuf &sb, int32_t *cnt, int32_t *list)
+{
+    __syncthreads();
+    const int m = min(sb.cnt, kGBuf);
+    if (threadIdx.x == 0) sb.base = m ? atomicAdd(cnt, m) : 0;
+    __syncthreads();
+    for (int k = threadIdx.x; k < m; k += NT) list[sb.base + k] = sb.v[k];
+    __syncthreads();
+    if (threadIdx.x == 0) sb.cnt = 0;
+    __syncthreads();
+}
+
+__global__ void __launch_bounds__(NT, 1) k_merge_grid(const MergeParams p)
+{
+    cg::grid_group grid = cg::this_grid();
+    __shared__ MHdr h;
+    __shared__ GBuf sb;
+    __shared__ GSeg sg;
+    extern __shared__ uint32_t filt[];  // p.grid_filter words (0: no filter)
+    const int tid = threadIdx.x, wid = tid >> 5, lane = tid & 31;
+    const bool use_f = p.grid_filter > 0;
+    if (tid == 0) sb.cnt = 0;
+    for (int w = tid; w < p.grid_filter; w += NT) filt[w] = 0;
+    __syncthreads();
+    const int G = gridDim.x, b = blockIdx.x;
+    const int nlist = (int)min(*p.list_cnt, (unsigned long long)p.list_max);
+    if (nlist == 0 || nlist > p.grid_max) return;  // uniform: the cluster kernel takes them
+    const int n = p.n, nw = (n + 31) >> 5;
+    uint32_t *bits = p.gbits;  // zero on entry; every row clears what it set
+    int32_t *ctrl = p.gctrl;   // [0], [1]: frontier counters; [2]: fail; [3]: diagonal
+    long long *part = p.gpart;
+    unsigned long long n_read = 0, n_rounds = 0;
+#if LUSYM_MERGE_PROF  // diagnostic build: ns per phase (CTA 0's view), printed at the end
+    unsigned long long tp[6] = {0, 0, 0, 0, 0, 0}, tq = 0;
+#define MPROF(k)                                                                 \
+    do {                                                                         \
+        unsigned long long now_;                                                 \
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(now_));                 \
+        if (tq) tp[k] += now_ - tq;                                              \
+        tq = now_;                                                               \
+    } while (0)
+#else
+#define MPROF(k) do { } while (0)
+#endif
+    for (int r = 0; r < nlist; ++r) {
+        const int i = p.list[r];
+        MPROF(5);
+        if (b == 0 && tid == 0) ctrl[0] = ctrl[1] = ctrl[2] = ctrl[3] = 0;
+        grid.sync();  // (also orders the previous row's bitmap clears before this row's marks)
+        if (b == 0 && tid == 0) atomicOr(bits + (i >> 5), 1u << (i & 31));
+        // ---- seed: S = A(i,:); members t < i form the first frontier
+        {
+            const int64_t rb = p.rp[i], re = p.rp[i + 1];
+            for (int64_t e0 = rb + (int64_t)b * NT; e0 < re; e0 += (int64_t)G * NT) {
+                const int64_t e = e0 + tid;
+                bool fr = false;
+                int v = -1;
+                if (e < re) {
+                    v = __ldg(p.ci + e);
+                    if (v == i) ctrl[3] = 1;
+                    else fr = tas_f(bits, filt, use_f, v) && v < i;
+                }
+                gbuf_push(fr, v, sb, ctrl + 0, p.gq);
+            }
+            gbuf_flush(sb, ctrl + 0, p.gq);
+        }
+        grid.sync();
+        MPROF(0);
+        int cur = 0;
+        for (;;) {
+            // (the fail flag is only read right after the barrier that follows its writes:
+            // every CTA must take the same branches around grid.sync)
+            const int fsize = ld_cg_int(ctrl + cur);
+            if (fsize == 0) break;
+            const int nxt = cur ^ 1;
+            const int32_t *F = p.gq + (size_t)cur * n;
+            int32_t *NF = p.gq + (size_t)nxt * n;
+            // (a) each member's U segment (pool offset, length); per-CTA sums over a
+            //     contiguous chunk of members: total length and non-empty segments
+            const int chunk = (fsize + G - 1) / G;
+            const int k0 = min(fsize, b * chunk), k1 = min(fsize, k0 + chunk);
+            long long sl = 0, sn = 0;
+            for (int k = k0 + tid; k < k1; k += NT) {
+                const int t = __ldcg(F + k);
+                const int64_t o = ld_acquire(p.row_off + t);
+                long long len = 0, off = 0;
+                if (o < 0) {
+                    ctrl[2] = 1;  // row t is not in the pool (unstaged, or failed)
+                } else {
+                    const int uc = __ldcg(p.ucut + t);
+                    off = o + uc;
+                    len = (long long)__ldcg(p.fill_count + t) - uc;
+                }
+                p.glen[k] = len;
+                p.goff[k] = off;
+                sl += len;
+                sn += len > 0;
+            }
+            block_sum2(sl, sn, h);
+            if (tid == 0) {
+                part[b] = sl;
+                part[G + b] = sn;
+            }
+            if (b == 0 && tid == 0) ctrl[nxt] = 0;  // last read as a fsize two barriers ago
+            grid.sync();
+            MPROF(1);
+            if (ld_cg_int(ctrl + 2)) break;
+            // (b) compaction of the non-empty segments, in member order
+            long long bl = 0, bn = 0, E = 0, M = 0;
+            for (int c = tid; c < G; c += NT) {
+                const long long x = __ldcg(part + c), y = __ldcg(part + G + c);
+                E += x;
+                M += y;
+                if (c < b) {
+                    bl += x;
+                    bn += y;
+                }
+            }
+            block_sum2(bl, bn, h);
+            block_sum2(E, M, h);
+            for (int kb = k0; kb < k1; kb += NT) {
+                const int k = kb + tid;
+                long long len = 0;
+                if (k < k1) len = __ldcg(p.glen + k);
+                long long tot;
+                // (len << 20 | nonempty): chunk <= ceil(n / G) members, so counts fit 20 bits
+                const long long st = scan_excl((len << 20) | (len > 0 ? 1 : 0), h, &tot);
+                if (len > 0) {
+                    const long long m = bn + (st & 0xfffff);
+                    p.gstart[m] = bl + (st >> 20);
+                    p.gcoff[m] = __ldcg(p.goff + k);
+                }
+                bl += tot >> 20;
+                bn += tot & 0xfffff;
+            }
+            if (b == 0 && tid < kSent) p.gstart[M + tid] = LLONG_MAX;
+            if (b == 0 && tid == 0) n_read += (unsigned long long)E;
+            grid.sync();
+            MPROF(2);
+            // (c) expansion: CTA b takes the flat positions [b per, (b+1) per); the starts and
+            //     offsets of the segments they cover are staged in shared memory kGSeg at a
+            //     time, then each warp expands a contiguous chunk as k_merge_rows does (one
+            //     search, then 32 start bits per window, all in shared memory)
+            {
+                const long long per = ((E + G - 1) / G + 31) & ~31ll;
+                const long long fb = min(E, (long long)b * per), fe = min(E, fb + per);
+                if (fb < fe) {
+                    if (tid == 0) {
+                        int lo = 0, hi = (int)M - 1;  // last segment starting at or before fb
+                        while (lo < hi) {
+                            const int mid = (lo + hi + 1) >> 1;
+                            if (__ldcg(p.gstart + mid) <= fb) lo = mid; else hi = mid - 1;
+                        }
+                        sg.m = lo;
+                    }
+                    __syncthreads();
+                    int m = sg.m;
+                    long long pos = fb;
+                    while (pos < fe) {
+                        for (int k = tid; k < kGSeg + kSent; k += NT) {
+                            const long long mk = (long long)m + k;
+                            sg.st[k] = mk < M + kSent ? __ldcg(p.gstart + mk) : LLONG_MAX;
+                            sg.off[k] = mk < M ? __ldcg(p.gcoff + mk) : 0;
+                        }
+                        __syncthreads();
+                        const long long bend = min(fe, sg.st[kGSeg]);
+                        const long long C = ((bend - pos + NW - 1) / NW + 31) & ~31ll;
+                        long long pw = pos + (long long)wid * C;
+                        const long long pend = min(bend, pw + C);
+                        if (pw < pend) {
+                            int src = 0;
+#pragma unroll
+                            for (int step = kGSeg / 2; step >= 1; step >>= 1)
+                                if (src + step < kGSeg && sg.st[src + step] <= pw) src += step;
+                            while (pw < pend) {
+                                int jv[kU];
+#pragma unroll
+                                for (int u = 0; u < kU; ++u) {
+                                    jv[u] = -1;
+                                    if (pw < pend) {
+                                        const long long snx = sg.st[src + 1 + lane];
+                                        const unsigned bit =
+                                            snx < pw + 32 ? 1u << (int)(snx - pw) : 0u;
+                                        const unsigned mask = __reduce_or_sync(0xffffffffu, bit);
+                                        const int my = src + __popc(mask & ((2u << lane) - 1u));
+                                        if (pw + lane < pend)
+                                            jv[u] = p.pool[sg.off[my] + (pw + lane - sg.st[my])];
+                                        const int last = __shfl_sync(0xffffffffu, my, 31);
+                                        src = last + (sg.st[last + 1] == pw + 32 ? 1 : 0);
+                                        pw += 32;
+                                    }
+                                }
+#pragma unroll
+                                for (int u = 0; u < kU; ++u) {
+                                    const int j = jv[u];
+                                    const bool fr = j >= 0 && tas_f(bits, filt, use_f, j) && j < i;
+                                    gbuf_push(fr, j, sb, ctrl + nxt, NF);
+                                }
+                            }
+                        }
+                        __syncthreads();
+                        pos = bend;
+                        m += kGSeg;
+                    }
+                }
+            }
+            gbuf_flush(sb, ctrl + nxt, NF);
+            ++n_rounds;
+            grid.sync();
+            MPROF(3);
+            cur = nxt;
+        }
+        const bool fail = ld_cg_int(ctrl + 2) != 0;
+        const bool diag = ld_cg_int(ctrl + 3) != 0;
+        // ---- output: the set bits, ascending, into the pool (each CTA a contiguous run of
+        // words at the offset of the runs before it); publish the row
+        const int wchunk = (nw + G - 1) / G;
+        const int w0 = min(nw, b * wchunk), w1 = min(nw, w0 + wchunk);
+        if (!fail) {
+            if (!diag && tid == 0 && (i >> 5) >= w0 && (i >> 5) < w1)
+                atomicAnd(bits + (i >> 5), ~(1u << (i & 31)));
+            __syncthreads();
+            long long c = 0, lo = 0;
+            for (int w = w0 + tid; w < w1; w += NT) {
+                const uint32_t x = __ldcg(bits + w);
+                const int pc = __popc(x);
+                c += pc;
+                if (w < (i >> 5)) lo += pc;
+                else if (w == (i >> 5))
+                    lo += __popc(x & ((i & 31) == 31 ? 0xffffffffu : ((2u << (i & 31)) - 1u)));
+            }
+            block_sum2(c, lo, h);
+            if (tid == 0) {
+                part[2 * G + b] = c;
+                part[3 * G + b] = lo;
+            }
+            grid.sync();
+            long long before = 0, tc = 0, tl = 0, dummy = 0;
+            for (int q = tid; q < G; q += NT) {
+                const long long x = __ldcg(part + 2 * G + q);
+                tc += x;
+                tl += __ldcg(part + 3 * G + q);
+                if (q < b) before += x;
+            }
+            block_sum2(before, dummy, h);
+            block_sum2(tc, tl, h);
+            if (b == 0 && tid == 0) {
+                const unsigned long long o = atomicAdd(p.pool_cursor, (unsigned long long)tc);
+                const bool fits = o + (unsigned long long)tc <= (unsigned long long)p.pool_cap;
+                part[4 * G] = fits ? (long long)o : -1ll;
+                if (fits) {
+                    p.fill_count[i] = (int32_t)tc;
+                    p.ucut[i] = (int32_t)tl;
+                } else {
+                    ctrl[2] = 1;
+                }
+            }
+            grid.sync();
+            const long long off = __ldcg(part + 4 * G);
+            if (off >= 0) {
+                int32_t *dst = p.pool + off + before;
+                long long run = 0;
+                for (int wb = w0; wb < w1; wb += NT) {
+                    const int w = wb + tid;
+                    uint32_t x = w < w1 ? __ldcg(bits + w) : 0u;
+                    long long tot;
+                    long long pos = run + scan_excl(__popc(x), h, &tot);
+                    for (; x; x &= x - 1, ++pos) dst[pos] = (w << 5) + __ffs(x) - 1;
+                    run += tot;
+                }
+                __threadfence();
+            }
+        }
+        grid.sync();  // every CTA's pool writes (and reads of the bitmap) are done
+        if (b == 0 && tid == 0) {
+            const long long off = fail ? -1ll : __ldcg(part + 4 * G);
+            if (off >= 0) {
+                st_release(p.row_off + i, off);
+            } else {
+                p.fail_list[atomicAdd(p.fail_cnt, 1ull)] = i;
+                st_release(p.row_off + i, -1);
+            }
+        }
+        // fill(:) = 0 for the next row (L115): each CTA its own words, and its whole filter
+        for (int w = w0 + tid; w < w1; w += NT) bits[w] = 0;
+        for (int w = tid; w < p.grid_filter; w += NT) filt[w] = 0;
+        MPROF(4);
+        // (the next row's first barrier orders this before its seed)
+    }
+#if LUSYM_MERGE_PROF
+    if (b == 0 && tid == 0)
+        printf("k_merge_grid: rows %d rounds %llu read %llu | ns seed %llu lens %llu compact %llu "
+               "expand %llu output %llu other %llu\n", nlist, n_rounds, n_read, tp[0], tp[1],
+               tp[2], tp[3], tp[4], tp[5]);
+#endif
+    if (b == 0 && tid == 0) {
+        *p.counter = (unsigned long long)nlist;  // the cluster kernel after this claims nothing
+        if (p.stats) {
+            atomicAdd(p.stats + 0, n_read);
+            atomicAdd(p.stats + 1, n_rounds);
+        }
+    }
+}
+
 // ascending bitonic sort of list[0..min(*cnt, max)) in shared memory (max <= kMergeSortMax)
 __global__ void __launch_bounds__(1024) k_sort_list(int32_t *list, const unsigned long long *cnt,
                                                     int32_t max)
@@ -526,6 +917,47 @@ int cluster_shift(int n, int g)
 }
 
 }  // namespace
+
+size_t merge_grid_smem(int n, int *filter_words)
+{
+    int dev = 0, optin = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&optin, cudaDevAttrMaxSharedMemoryPerBlockOptin, dev);
+    cudaFuncAttributes fa;
+    if (cudaFuncGetAttributes(&fa, k_merge_grid) != cudaSuccess) {
+        cudaGetLastError();
+        *filter_words = 0;
+        return 0;
+    }
+    const size_t fw = (size_t)(n + 31) / 32;
+    const bool fits = fa.sharedSizeBytes + fw * 4 <= (size_t)optin &&
+                      !getenv("LUSYM_MERGE_GRID_NOFILTER");  // A/B knob
+    *filter_words = fits ? (int)fw : 0;
+    return fits ? fw * 4 : 0;
+}
+
+cudaError_t merge_grid_size(int n, int *grid, int *filter_words)
+{
+    int dev = 0, sms = 0, occ = 0;
+    cudaGetDevice(&dev);
+    const size_t smem = merge_grid_smem(n, filter_words);
+    cudaError_t e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (e == cudaSuccess)
+        e = cudaFuncSetAttribute((const void *)k_merge_grid,
+                                 cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e == cudaSuccess)
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, k_merge_grid, NT, smem);
+    if (e != cudaSuccess) return e;
+    *grid = sms * (occ > 0 ? occ : 0);
+    return cudaSuccess;
+}
+
+cudaError_t merge_grid_launch(const MergeParams &p, int grid, cudaStream_t s)
+{
+    void *args[] = {(void *)&p};
+    return cudaLaunchCooperativeKernel((const void *)k_merge_grid, grid, NT, args,
+                                       (size_t)p.grid_filter * 4, s);
+}
 
 cudaError_t merge_configure_impl(size_t smem);
 cudaError_t merge_max_clusters_impl(int g, size_t smem, int *clusters);
