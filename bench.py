@@ -520,6 +520,8 @@ def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
             st = h.stats()
             for key in keys:
                 k_ms[key].append(st["ms_" + key])
+            if world > 1:
+                k_ms.setdefault("assemble", []).append(getattr(h, "ms_assemble", 0.0))
             if verify is not None:                           # outside the events
                 verify(state["fc"], state["rp_lu"], state["ci_lu"], state["level"], state["nl"])
         barrier()

@@ -536,14 +536,24 @@ def sharded_pass(h: Symbolic, rb: int, re: int, bounds, group=None, stream=None)
     fc = torch.zeros(n, dtype=torch.int32, device=h.device)
     h.count(rb, re, fc, stream=stream)
     flags = h.deferred_flags(stream=stream)
+    # device time of the exchange steps (S7), recorded on the current stream: h.ms_assemble
+    ev = [torch.cuda.Event(enable_timing=True) for _ in range(4)] if world > 1 else None
     if world > 1:
+        ev[0].record()
         assemble_counts(fc, group)
         assemble_counts(flags, group)
+        ev[1].record()
     rp_lu, nnz = h.scan(fc, stream=stream)
     ci_lu = torch.empty(nnz, dtype=torch.int32, device=h.device)
     h.emit(rp_lu, ci_lu, rb, re, stream=stream)
     if world > 1:
+        ev[2].record()
         assemble_pattern(ci_lu, rp_lu, bounds, group)
+        ev[3].record()
+        ev[3].synchronize()
+        h.ms_assemble = ev[0].elapsed_time(ev[1]) + ev[2].elapsed_time(ev[3])
+    else:
+        h.ms_assemble = 0.0
     if int(flags.sum()) > 0:
         nnz = h.merge_deferred(flags, fc, rp_lu, ci_lu, stream=stream)
         ci_lu = torch.empty(nnz, dtype=torch.int32, device=h.device)
