@@ -44,6 +44,12 @@ constexpr int NW = NT / 32;
 #ifndef LUSYM_MERGE_PROF
 #define LUSYM_MERGE_PROF 0
 #endif
+#ifndef LUSYM_MERGE_HASH  // cluster mode: new members spread over the ranks by a hash of their id
+#define LUSYM_MERGE_HASH 1
+#endif
+#ifndef LUSYM_MERGE_BATCH  // expansion: the kU windows' visited words loaded before any atomic
+#define LUSYM_MERGE_BATCH 0
+#endif
 constexpr int kU = LUSYM_MERGE_KU;  // pool loads in flight per thread
 constexpr int kSent = 64;  // sentinel starts past the last segment
 
@@ -140,6 +146,43 @@ __device__ __forceinline__ void q_push(bool pred, int32_t w, int *cnt, int32_t *
     }
 }
 
+// Cluster mode: a new member goes to the frontier of the rank a hash of its id picks (DSMEM
+// atomics on that rank's counter, stores into its queue), not to the discovering rank's: the
+// ranks then expand equal shares of the next round instead of waiting at the cluster barrier
+// for the rank that happened to discover the most (cfg3's largest hub: 54% of the tail's stall
+// samples were cluster barrier waits).
+template <int MODE>
+__device__ __forceinline__ void q_push_hashed(bool pred, int32_t w, int *cnt_local,
+                                              int32_t *sq_local, int32_t *gq_rank0, int64_t gstride,
+                                              int rank, int g, int q)
+{
+    const unsigned any = __ballot_sync(0xffffffffu, pred);
+    if (!any) return;
+    const int lane = threadIdx.x & 31;
+    const int dst = pred ? (int)((((uint32_t)w * 2654435761u) >> 16) % (uint32_t)g) : -1;
+    auto cl = cg::this_cluster();
+    for (int r = 0; r < g; ++r) {
+        const unsigned b = __ballot_sync(0xffffffffu, dst == r);
+        if (!b) continue;
+        const int leader = __ffs(b) - 1;
+        int base = 0;
+        if (lane == leader) {
+            int *c = r == rank ? cnt_local : cl.map_shared_rank(cnt_local, r);
+            base = atomicAdd(c, __popc(b));
+        }
+        base = __shfl_sync(0xffffffffu, base, leader);
+        if (dst == r) {
+            const int pos = base + __popc(b & ((1u << lane) - 1u));
+            if (pos < q) {
+                int32_t *d = r == rank ? sq_local : cl.map_shared_rank(sq_local, r);
+                d[pos] = w;
+            } else {
+                gq_rank0[(int64_t)r * gstride + pos] = w;
+            }
+        }
+    }
+}
+
 // The row's visited bitmap: whole in this CTA (shared memory or HBM slot), or sliced over the
 // cluster, word w in rank w >> sh at local index w & (wpc - 1).
 template <bool CL>
@@ -228,6 +271,10 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
         }
         const int i = h.row;
         if (i < 0) break;
+#if LUSYM_MERGE_PROF
+        unsigned long long t_claim = 0, t_firstwait = 0, t_lastwait = 0, rows_r = 0, nwaits_r = 0;
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_claim));
+#endif
         // ---- seed: S = A(i,:); members t < i form the first frontier (entries split by rank)
         if (tid == 0 && bm.rank == 0) atomicOr(bm.word(i >> 5), 1u << (i & 31));
         csync_impl(CL);
@@ -278,10 +325,17 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
                 // every member left is a deferred row still in progress: wait for them (each
                 // was claimed before row i by a running cluster), then expand them
                 const int nwt = h.nwait;
+#if LUSYM_MERGE_PROF
+                if (!t_firstwait) asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_firstwait));
+                nwaits_r += nwt;
+#endif
                 for (int k = tid; k < nwt; k += NT) {
                     const int t = wait[k];
                     while (ld_acquire(p.row_off + t) == kRowDeferred) __nanosleep(200);
                 }
+#if LUSYM_MERGE_PROF
+                asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_lastwait));
+#endif
                 if (tid == 0) n_waits += nwt;
                 __syncthreads();
                 for (int k = tid; k < nwt; k += NT) {
@@ -358,11 +412,30 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
                                 pw += 32;
                             }
                         }
+#if LUSYM_MERGE_BATCH
+                        // every window's visited word first (kU loads in flight, DSMEM in
+                        // cluster mode), then the atomics on the bits that looked clear
+                        uint32_t wv[kU];
+#pragma unroll
+                        for (int u = 0; u < kU; ++u)
+                            wv[u] = jv[u] >= 0 ? *bm.word(jv[u] >> 5) : ~0u;
+#endif
 #pragma unroll
                         for (int u = 0; u < kU; ++u) {
                             const int j = jv[u];
+#if LUSYM_MERGE_BATCH
+                            const uint32_t bb = 1u << (j & 31);
+                            const bool fr = j >= 0 && !(wv[u] & bb) &&
+                                            !(atomicOr(bm.word(j >> 5), bb) & bb) && j < i;
+#else
                             const bool fr = j >= 0 && bm.tas(j) && j < i;
-                            q_push(fr, j, &h.cnt[nxt], nq, gnq, p.q);
+#endif
+                            if constexpr (CL && LUSYM_MERGE_HASH)
+                                q_push_hashed<MODE>(fr, j, &h.cnt[nxt], nq,
+                                                    gnq - (int64_t)bm.rank * 2 * p.spill_cap,
+                                                    2 * p.spill_cap, bm.rank, bm.g, p.q);
+                            else
+                                q_push(fr, j, &h.cnt[nxt], nq, gnq, p.q);
                         }
                     }
                 }
@@ -371,6 +444,9 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
             // (fsize > 0: the loop's barriers ordered every read of h.cnt[cur] before this)
             if (tid == 0 && fsize) h.cnt[cur] = 0;
             if (tid == 0) ++n_rounds;
+#if LUSYM_MERGE_PROF
+            ++rows_r;
+#endif
             __syncthreads();
             cur = nxt;
         }
@@ -441,6 +517,17 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
             p.fail_list[atomicAdd(p.fail_cnt, 1ull)] = i;
             st_release(p.row_off + i, -1);
         }
+#if LUSYM_MERGE_PROF
+        if (tid == 0 && bm.rank == 0) {
+            unsigned long long t_end;
+            asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_end));
+            printf("k_merge_rows: row %d cta %d claim %llu first_wait %+lld last_wait %+lld end %+lld "
+                   "(ns after claim) rounds %llu waits %llu\n", i, (int)blockIdx.x, t_claim % 1000000000ull,
+                   t_firstwait ? (long long)(t_firstwait - t_claim) : -1ll,
+                   t_lastwait ? (long long)(t_lastwait - t_claim) : -1ll,
+                   (long long)(t_end - t_claim), rows_r, nwaits_r);
+        }
+#endif
         // ---- fill(:) = 0 for the next row (L115)
         __syncthreads();
         for (int w = bm.lo + tid; w < bm.hi; w += NT) lw[w] = 0;

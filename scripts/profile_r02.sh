@@ -21,7 +21,7 @@ python scripts/summarize_ncu_r02.py cfg1=$P/p2_cfg1.ncu-rep:gpurun_out/p2_cfg1.l
 mkdir -p gpurun_out/r02prof
 cp profiles/r02/ncu_summary.json profiles/r02/ncu_cfg*.txt gpurun_out/r02prof/ 2>/dev/null
 for c in cfg1 cfg2 cfg3 cfg4 cfg5 merge_cfg3; do
-  python scripts/ncu_hot.py $P/p2_$c.ncu-rep 30 > gpurun_out/r02prof/hot_$c.txt 2>&1
+  python scripts/ncu_hot.py $P/p2_$c.ncu-rep 3000 > gpurun_out/r02prof/hot_$c.txt 2>&1
   python scripts/ncu_regions.py $P/p2_$c.ncu-rep > gpurun_out/r02prof/regions_$c.txt 2>&1
   python scripts/ncu_funcs.py $P/p2_$c.ncu-rep > gpurun_out/r02prof/funcs_$c.txt 2>&1
   ncu -i $P/p2_$c.ncu-rep --page details --csv > gpurun_out/r02prof/details_$c.csv 2>/dev/null
