@@ -818,8 +818,13 @@ lu_status run_pass(lu_sym *h, int mode, int32_t rb, int32_t re, int32_t *fill_co
         p.lbw = c.lbw;
         p.q = c.q;
         p.wcap = (h->opts.flags & LU_F_NO_BATCH) ? 1 : c.q;
-        // one row per SM: a BFS level is latency-bound, let lanes run ahead a little
-        p.kloc = ((c.occ <= LUSYM_KLOC_OCC || (h->opts.flags & LU_F_SELF_CONT)) &&
+        // one row per SM, or a pass with at most two rows per CTA in flight (cfg1: 4,096 rows on
+        // 2,368 CTAs): a BFS level is latency-bound, let lanes run ahead a little (cfg1 count
+        // 0.328 -> 0.305 ms; with many rows per CTA the extra rounds cost issue slots: cfg2 and
+        // cfg5 twice as slow, profiles/r02/knobs_sc.log)
+        // (the class's whole row range, not this call's: a chunk of lu_sym_run_host is short)
+        const bool few_rows = (int64_t)(c.hi - c.lo) <= 2 * (int64_t)c.grid;
+        p.kloc = ((c.occ <= LUSYM_KLOC_OCC || few_rows || (h->opts.flags & LU_F_SELF_CONT)) &&
                   !(h->opts.flags & LU_F_NO_SELF_CONT))
                      ? LUSYM_KLOC
                      : 0;

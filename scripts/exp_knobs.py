@@ -22,7 +22,7 @@ for spec in sys.argv[4:]:
     h = lu.Symbolic(trp, tci, **kw)
     fc = torch.zeros(n, dtype=torch.int32, device=dev)
     ts = []
-    for _ in range(2):
+    for _ in range(int(os.environ.get('REPS', '2'))):
         e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         e0.record()
         h.count(lo, hi, fc)
@@ -33,7 +33,7 @@ for spec in sys.argv[4:]:
     if ref is None:
         ref = got
     st = h.stats()
-    print(f"{name} [{lo},{hi}) {spec}: count ms {min(ts):.1f} same={np.array_equal(got, ref)} "
+    print(f"{name} [{lo},{hi}) {spec}: count ms {min(ts):.3f} same={np.array_equal(got, ref)} "
           f"rif={st['rows_in_flight']} tpr={st['threads_per_row']} smem={st['smem_bytes_per_row']} "
           f"classes={st['row_classes']} q={st['queue_capacity']} spills={st['spills']}", flush=True)
     h.close()
