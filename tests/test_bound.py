@@ -80,3 +80,40 @@ def test_library_bound_matches():
         h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
         assert h.nnz_bound() == bound(rp, ci)
         h.close()
+
+
+@pytest.mark.gpu
+def test_run_host_with_bound_capacity():
+    """The e2e protocol of bench.py: outputs allocated from the bound, one lu_sym_run_host call
+    streaming the pattern to pinned host memory; bit-exact against the oracle."""
+    import torch
+    lu = pytest.importorskip("paper_conf_ppopp_xia0ar23_b200")
+    d = torch.device("cuda", torch.cuda.current_device())
+    for rp, ci in [gen.lap2d(40), gen.lap3d(9), gen.circuit(32, 2),
+                   gen.random_pattern(900, 2.5, seed=5)]:
+        ref = oracle.fill2(rp, ci)
+        n = len(rp) - 1
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+        cap = h.nnz_bound()
+        assert cap >= int(ref["row_ptr"][-1])
+        hrp = torch.empty(n + 1, dtype=torch.int64, pin_memory=True)
+        hci = torch.empty(cap, dtype=torch.int32, pin_memory=True)
+        fc, rp_lu, ci_lu = h.run_host(cap, hrp, hci)
+        nz = int(ci_lu.numel())
+        assert np.array_equal(hrp.numpy(), ref["row_ptr"])
+        assert np.array_equal(hci.numpy()[:nz], ref["col_idx"])
+        assert np.array_equal(fc.cpu().numpy(), ref["counts"])
+        h.close()
+
+
+@pytest.mark.gpu
+def test_bound_degenerate():
+    import torch
+    lu = pytest.importorskip("paper_conf_ppopp_xia0ar23_b200")
+    d = torch.device("cuda", torch.cuda.current_device())
+    # n = 0, and rows with no entries at all (no diagonal)
+    for rp, ci in [(np.zeros(1, np.int64), np.zeros(0, np.int32)),
+                   (np.array([0, 0, 1, 1], np.int64), np.array([0], np.int32))]:
+        h = lu.Symbolic(torch.from_numpy(rp).to(d), torch.from_numpy(ci).to(d))
+        assert h.nnz_bound() == bound(rp, ci)
+        h.close()
