@@ -549,15 +549,8 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
 // separate the phases: seed, then per round (lengths -> compaction -> expansion), then the
 // output (popcounts -> pool offset -> sorted write).
 
-__device__ __forceinline__ bool tas_g(uint32_t *bits, int v)
-{
-    const uint32_t b = 1u << (v & 31);
-    uint32_t *w = bits + (v >> 5);
-    if (__ldcg(w) & b) return false;
-    return !(atomicOr(w, b) & b);
-}
-
-// ... behind a per-CTA filter in shared memory (fw words, 0: none): bits are only ever set
+// Test-and-set in the grid's visited bitmap (HBM, L2-resident) behind a per-CTA filter in
+// shared memory (fw words, 0: none): bits are only ever set
 // during a row, so a bit this CTA has seen set (in the filter) is set; a miss reads the global
 // word and keeps every bit it holds.  Nearly every pool entry of a hub's closure is a member
 // already found (cfg3: 1.3e9 entries read for 2.7e7 members), so most tests end in shared memory.
