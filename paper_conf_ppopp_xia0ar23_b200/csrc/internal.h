@@ -110,6 +110,7 @@ struct MergeParams {
     // grid-wide mode (k_merge_grid): the whole GPU finishes the deferred rows one at a time in
     // increasing order when there are at most grid_max of them (0: never)
     int32_t grid_max = 0;
+    int32_t grid_head = 0;             // > 0: the grid takes the first grid_head rows of any list
     uint32_t *gbits = nullptr;         // [ceil(n/32)] visited bitmap of the row in progress
     int32_t *gq = nullptr;             // [2 n] frontier buffers
     long long *glen = nullptr;         // [n] U segment length of each frontier member

@@ -91,7 +91,7 @@ struct RowClass {
 
 struct lu_sym {
     // grid-wide tail (k_merge_grid) for lists of at most mg_max deferred rows
-    int mg_max = 0, mg_grid = 0, mg_filter = 0;
+    int mg_max = 0, mg_head = 0, mg_grid = 0, mg_filter = 0;
     uint32_t *mg_bits = nullptr;
     int32_t *mg_q = nullptr, *mg_ctrl = nullptr;
     long long *mg_ll = nullptr;
@@ -1019,9 +1019,16 @@ lu_status ensure_merge(lu_sym *h)
     // rows are finished by the whole grid, one row at a time (k_merge_grid), instead of by
     // 4-CTA clusters in parallel.  Measured on cfg3's 32 hubs: 19.1 ms against 17.4 (396
     // rounds; the per-round phases and grid barriers cost what the extra SMs save).
+    // mg_head > 0: the grid takes only the first rows of a list and the clusters the rest.
     h->mg_max = 0;
     if (const char *e = getenv("LUSYM_MERGE_GRID_MAX")) h->mg_max = atoi(e);
-    if (h->mg_max > 0 && merge_grid_size(n, &h->mg_grid, &h->mg_filter) == cudaSuccess &&
+    // LUSYM_MERGE_GRID_HEAD: the grid takes the first rows of every list (default 2): the
+    // head of the hubs' chain, whose closure is the cluster tail's critical path (cfg3 tail
+    // 16.5 -> 15.2-15.3 ms with 2 or 3, profiles/r02/merge_grid_head.log)
+    h->mg_head = 2;
+    if (const char *e = getenv("LUSYM_MERGE_GRID_HEAD")) h->mg_head = atoi(e);
+    if ((h->mg_max > 0 || h->mg_head > 0) &&
+        merge_grid_size(n, &h->mg_grid, &h->mg_filter) == cudaSuccess &&
         h->mg_grid > 0) {
         const size_t need = (size_t)words * 4 + (size_t)2 * n * 4 + (size_t)4 * n * 8 + 64 * 8 +
                             ((size_t)4 * h->mg_grid + 8) * 8 + 64;
@@ -1036,11 +1043,11 @@ lu_status ensure_merge(lu_sym *h)
             if ((st = salloc(h, &h->mg_ctrl, 16)) != LU_OK) return st;
             CK(cudaMemsetAsync(h->mg_bits, 0, (size_t)words * 4, h->stream));
         } else {
-            h->mg_max = 0;
+            h->mg_max = h->mg_head = 0;
         }
     } else {
         cudaGetLastError();
-        h->mg_max = 0;
+        h->mg_max = h->mg_head = 0;
     }
     return LU_OK;
 }
@@ -1092,11 +1099,12 @@ lu_status run_tail_list(lu_sym *h, int32_t *fill_count, const int32_t *list,
     mp.fail_cnt = slots + 2;
     mp.stats = slots + 3;
     mp.q = h->merge_q;
-    if (h->mg_max > 0) {
+    if (h->mg_max > 0 || h->mg_head > 0) {
         // a short list: the whole grid, one row at a time (k_merge_grid); a longer one is left
         // to the clusters (the kernel checks the device-side count)
         const size_t n = (size_t)h->n;
         mp.grid_max = h->mg_max;
+        mp.grid_head = h->mg_head;
         mp.gbits = h->mg_bits;
         mp.gq = h->mg_q;
         mp.glen = h->mg_ll;

@@ -641,8 +641,12 @@ __global__ void __launch_bounds__(NT, 1) k_merge_grid(const MergeParams p)
     for (int w = tid; w < p.grid_filter; w += NT) filt[w] = 0;
     __syncthreads();
     const int G = gridDim.x, b = blockIdx.x;
-    const int nlist = (int)min(*p.list_cnt, (unsigned long long)p.list_max);
-    if (nlist == 0 || nlist > p.grid_max) return;  // uniform: the cluster kernel takes them
+    const int nall = (int)min(*p.list_cnt, (unsigned long long)p.list_max);
+    // all rows of a short list, or (grid_head) the first rows of any list: the head of the
+    // hubs' dependency chain, whose closure is the tail's critical path on a cluster
+    int nlist = nall <= p.grid_max ? nall : 0;
+    if (p.grid_head > 0) nlist = min(nall, max(nlist, p.grid_head));
+    if (nlist == 0) return;  // uniform: the cluster kernel takes them
     const int n = p.n, nw = (n + 31) >> 5;
     uint32_t *bits = p.gbits;  // zero on entry; every row clears what it set
     int32_t *ctrl = p.gctrl;   // [0], [1]: frontier counters; [2]: fail; [3]: diagonal
