@@ -39,13 +39,16 @@ namespace {
 constexpr int NT = kMergeNT;
 constexpr int NW = NT / 32;
 #ifndef LUSYM_MERGE_KU
-#define LUSYM_MERGE_KU 4
+#define LUSYM_MERGE_KU 1  // windows in flight per warp (A/B on cfg3: 1 = 14.8 ms tail, 2 = 15.2, 4 = 15.2, 8 = 15.4)
 #endif
 #ifndef LUSYM_MERGE_PROF
 #define LUSYM_MERGE_PROF 0
 #endif
 #ifndef LUSYM_MERGE_HASH  // cluster mode: new members spread over the ranks by a hash of their id
 #define LUSYM_MERGE_HASH 1
+#endif
+#ifndef LUSYM_MERGE_LDCG  // expansion: pool entries read through L2 only (ld.global.cg)
+#define LUSYM_MERGE_LDCG 0
 #endif
 #ifndef LUSYM_MERGE_BATCH  // expansion: the kU windows' visited words loaded before any atomic
 #define LUSYM_MERGE_BATCH 0
@@ -272,6 +275,7 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
         const int i = h.row;
         if (i < 0) break;
 #if LUSYM_MERGE_PROF
+        long long prof_setup = 0, prof_expand = 0, prof_tiles = 0, prof_entries = 0;
         unsigned long long t_claim = 0, t_firstwait = 0, t_lastwait = 0, rows_r = 0, nwaits_r = 0;
         asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t_claim));
 #endif
@@ -354,6 +358,9 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
             const int32_t *fq = sq + cur * p.q, *gfq = gq0 + (size_t)cur * p.spill_cap;
             int32_t *nq = sq + nxt * p.q, *gnq = gq0 + (size_t)nxt * p.spill_cap;
             for (int base = 0; base < fsize; base += NT) {
+#if LUSYM_MERGE_PROF
+                long long c_t0 = clock64();
+#endif
                 const int k = base + tid;
                 long long off = 0, len = 0;
                 if (k < fsize) {
@@ -382,6 +389,10 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
                 if (tid < kSent) c_start[nsrc + tid] = LLONG_MAX;
                 __syncthreads();
                 if (tid == 0) n_read += (unsigned long long)E;
+#if LUSYM_MERGE_PROF
+                long long c_t1 = clock64();
+                if (tid == 0) prof_setup += c_t1 - c_t0;
+#endif
                 // each warp expands a contiguous chunk of the E flat positions, 32 at a time: one
                 // binary search for the chunk's first owner, then the owner of lane l of a window
                 // [p, p+32) is that window's owner plus the segments starting in (p, p+l]
@@ -406,7 +417,9 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
                                 const unsigned mask = __reduce_or_sync(0xffffffffu, bit);
                                 const int my = src + __popc(mask & ((2u << lane) - 1u));
                                 if (pw + lane < pend)
-                                    jv[u] = p.pool[c_off[my] + (pw + lane - c_start[my])];
+                                    jv[u] = LUSYM_MERGE_LDCG
+                                                ? __ldcg(p.pool + c_off[my] + (pw + lane - c_start[my]))
+                                                : p.pool[c_off[my] + (pw + lane - c_start[my])];
                                 const int last = __shfl_sync(0xffffffffu, my, 31);
                                 src = last + (c_start[last + 1] == pw + 32 ? 1 : 0);
                                 pw += 32;
@@ -440,6 +453,13 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
                     }
                 }
                 __syncthreads();
+#if LUSYM_MERGE_PROF
+                if (tid == 0) {
+                    prof_expand += clock64() - c_t1;
+                    ++prof_tiles;
+                    prof_entries += E;
+                }
+#endif
             }
             // (fsize > 0: the loop's barriers ordered every read of h.cnt[cur] before this)
             if (tid == 0 && fsize) h.cnt[cur] = 0;
@@ -526,6 +546,8 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
                    t_firstwait ? (long long)(t_firstwait - t_claim) : -1ll,
                    t_lastwait ? (long long)(t_lastwait - t_claim) : -1ll,
                    (long long)(t_end - t_claim), rows_r, nwaits_r);
+            printf("k_merge_rows: row %d rank0 tiles %lld entries %lld setup cycles %lld expand "
+                   "cycles %lld\n", i, prof_tiles, prof_entries, prof_setup, prof_expand);
         }
 #endif
         // ---- fill(:) = 0 for the next row (L115)
