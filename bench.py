@@ -51,7 +51,7 @@ def parse():
     ap.add_argument("--rule", default="u", choices=["u", "glu3"])
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--e2e-steps", type=int, default=3)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--e2e-two-call", action="store_true",
                     help="e2e through the two-call protocol even when the capacity bound is usable")
     ap.add_argument("--e2e-host", default="pinned", choices=["pinned", "pageable"],
@@ -614,6 +614,7 @@ def measure(args, cfg, steps, warmup, world, rank, local_rank, headline):
     h.close()
     del h
     if headline and not args.no_e2e:
+        torch.cuda.empty_cache()  # torch's cached blocks back to the device before the e2e run
         rec["e2e"] = e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank,
                          bounds, verify)
     return rec
@@ -631,7 +632,7 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
     ci_h = torch.from_numpy(ci_np).pin_memory()
     pinned = args.e2e_host == "pinned"
     rb, re_ = int(bounds[rank]), int(bounds[rank + 1])
-    e_ms, phases = [], {}
+    e_ms, phases, step_phases = [], {}, []
     for k in range(args.e2e_steps + 1):
         if world > 1:
             dist.barrier()
@@ -704,9 +705,12 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
         else:
             e_ms.append(a.elapsed_time(b))
             prev = a
+            st_ph = {}
             for tag, e_ in marks + [("d2h(pattern, levels)", b)]:
                 phases.setdefault(tag, []).append(prev.elapsed_time(e_))
+                st_ph[tag] = round(prev.elapsed_time(e_), 3)
                 prev = e_
+            step_phases.append(st_ph)
         if verify is not None:
             verify.host(out_rp.numpy(), out_ci.numpy()[:nz], out_lv.numpy())
         del out_rp, out_ci, out_lv, ci_lu, rp_lu, fc
@@ -717,6 +721,8 @@ def e2e(args, lu, dev, stream, rp_np, ci_np, nnz, sym_opts, world, rank, bounds,
             "h2d_bytes_per_step": int(rp_np.nbytes + ci_np.nbytes),
             "d2h_bytes_per_step": int((n + 1) * 8 + nnz * 4 + n * 4) if rank == 0 else 0,
             "ms_per_step": float(t.item()),
+            "steps_ms": [float(x) for x in e_ms],
+            "steps_phases_ms": step_phases,
             "phases_ms": {k: float(np.mean(v)) for k, v in phases.items()},
             "host_buffers": ("pinned, allocated inside the timed region once nnz is known "
                              "(torch's caching host allocator serves repeated calls; the first "

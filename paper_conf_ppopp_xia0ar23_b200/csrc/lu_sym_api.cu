@@ -5,6 +5,7 @@
 #include <nvtx3/nvtx3.hpp>  // header-only: a named range per ABI call (for nsys / ncu)
 
 #include <chrono>
+#include <mutex>
 #include <cstdarg>
 #include <cstdio>
 #include <cstdlib>
@@ -322,6 +323,41 @@ const bool g_tight_classes = [] {
     return e ? atoi(e) != 0 : true;
 }();
 
+// Free device memory for the planner's budget.  cudaMemGetInfo takes from 0.1 ms to 95 ms
+// (measured in bench.py's e2e loop, a create after another handle's destroy),
+// so a reading younger than 30 s is reused per device.  The budget is 0.85 of it, the staging
+// pool falls back to re-traversal if its allocation fails, and other allocations that still
+// fail return LU_ERR_NOMEM.
+cudaError_t mem_info(size_t *free_b, size_t *total_b)
+{
+    struct Reading {
+        size_t free_b = 0, total_b = 0;
+        std::chrono::steady_clock::time_point t;
+        bool valid = false;
+    };
+    static Reading cache[64];
+    static std::mutex mu;
+    int dev = 0;
+    cudaError_t e = cudaGetDevice(&dev);
+    if (e != cudaSuccess) return e;
+    const auto now = std::chrono::steady_clock::now();
+    {
+        std::lock_guard<std::mutex> lock(mu);
+        if (dev >= 0 && dev < 64 && cache[dev].valid &&
+            now - cache[dev].t < std::chrono::seconds(30)) {
+            *free_b = cache[dev].free_b;
+            *total_b = cache[dev].total_b;
+            return cudaSuccess;
+        }
+    }
+    e = cudaMemGetInfo(free_b, total_b);
+    if (e == cudaSuccess && dev >= 0 && dev < 64) {
+        std::lock_guard<std::mutex> lock(mu);
+        cache[dev] = Reading{*free_b, *total_b, now, true};
+    }
+    return e;
+}
+
 // LUSYM_DEBUG_CREATE: host milliseconds of each create / plan step on stderr (diagnostic)
 const bool g_dbg_create = getenv("LUSYM_DEBUG_CREATE") != nullptr;
 std::chrono::steady_clock::time_point g_tc;
@@ -566,7 +602,8 @@ lu_status plan(lu_sym *h)
     }
     dbg_lap(h->stream, "plan: classes");
     size_t free_b = 0, total_b = 0;
-    CK(cudaMemGetInfo(&free_b, &total_b));
+    CK(mem_info(&free_b, &total_b));
+    dbg_lap(h->stream, "plan: meminfo");
     const uint64_t budget = h->opts.scratch_budget_bytes ? h->opts.scratch_budget_bytes
                                                          : (uint64_t)(0.85 * (double)free_b);
     h->budget = budget;
@@ -924,7 +961,7 @@ lu_status ensure_pool(lu_sym *h)
 {
     if (h->pool || h->pool_cap < 0) return LU_OK;
     size_t free_b = 0, total_b = 0;
-    CK(cudaMemGetInfo(&free_b, &total_b));
+    CK(mem_info(&free_b, &total_b));
     uint64_t want = h->opts.pool_bytes;
     if (want == 0) {
         const uint64_t budget = h->budget > (uint64_t)h->scratch_bytes
