@@ -60,6 +60,9 @@ namespace f2 {
 #ifndef LUSYM_TAM  // test_and_mark with one shared bit mask (0: visited() then mark())
 #define LUSYM_TAM 1
 #endif
+#ifndef LUSYM_THREADS_PER_SM_SMALL  // ... for CTAs of at most 128 threads
+#define LUSYM_THREADS_PER_SM_SMALL LUSYM_THREADS_PER_SM
+#endif
 #ifndef LUSYM_THREADS_PER_SM  // register budget: 65536 / this
 #define LUSYM_THREADS_PER_SM 2048
 #endif
@@ -1180,7 +1183,11 @@ __device__ void bfs(const Fill2Params &p, Hdr &h, const VisMap<VIS> &bm, uint32_
 // limits them to one CTA per SM (the planner picks it).
 template <int KEY>
 struct NtCfg {
-    static constexpr int NT = KEY, MINB = LUSYM_THREADS_PER_SM / KEY;
+    // (LUSYM_THREADS_PER_SM_SMALL: a separate budget for 64- and 128-thread CTAs; 1536, i.e.
+    // ~40 registers, measured in session 2 against 2048: cfg2 +10%, cfg3 +6%, cfg1 +70%,
+    // profiles/r02/ab_regs2.log, so both stay at 2048)
+    static constexpr int NT = KEY,
+                         MINB = (KEY <= 128 ? LUSYM_THREADS_PER_SM_SMALL : LUSYM_THREADS_PER_SM) / KEY;
 };
 template <>
 struct NtCfg<1025> {
