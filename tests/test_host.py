@@ -53,6 +53,7 @@ def test_argument_errors_without_device():
     st = lib.lu_levelize(None, 5, None, None, 3, None, None, None)
     assert st == lu.LU_ERR_ARG
     assert lib.lu_sym_get_stats(None, None) == lu.LU_ERR_ARG
+    assert lib.lu_sym_nnz_bound(None, None, None) == lu.LU_ERR_ARG
     lib.lu_sym_destroy(None)
 
 
