@@ -48,6 +48,9 @@ namespace f2 {
 #ifndef LUSYM_GB_DIRECT_ATOMIC  // HBM visited slots: test-and-set by the atomic alone
 #define LUSYM_GB_DIRECT_ATOMIC 0
 #endif
+#ifndef LUSYM_GB_L1  // test_and_mark: HBM-slot pre-check loads cached in L1 (A/B knob)
+#define LUSYM_GB_L1 0
+#endif
 #ifndef LUSYM_PREFETCH_NEXT  // prefetch a new frontier vertex's adjacency row into L1
 #define LUSYM_PREFETCH_NEXT 0  // A/B: +7..15% slower (profiles/r02/ab_prefetch.log)
 #endif
@@ -269,7 +272,11 @@ __device__ __forceinline__ bool test_and_mark(const VisMap<VIS> &m, uint32_t *sm
         return !(old & b);
     }
 #endif
-    const uint32_t word = sh ? lds_bm(phys<VIS>(m, w)) : __ldcg(m.g + w);
+    // (LUSYM_GB_L1: the HBM slot's pre-check through L1.  Only this CTA writes its slot and
+    // bits only get set during a row, so a stale L1 copy can only miss bits, which the atomic
+    // then decides; the per-row clears are this CTA's own stores.)
+    const uint32_t word = sh ? lds_bm(phys<VIS>(m, w))
+                             : (LUSYM_GB_L1 ? __ldca(m.g + w) : __ldcg(m.g + w));
     if (word & b) return false;
     const uint32_t old = sh ? atom_or_bm(phys<VIS>(m, w), b) : atomicOr(m.g + w, b);
     if (old == 0)
