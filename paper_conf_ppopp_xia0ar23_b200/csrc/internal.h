@@ -107,6 +107,7 @@ struct MergeParams {
     unsigned long long *fail_cnt;
     unsigned long long *stats;         // [0] U entries read, [1] rounds, [2] waits
     int32_t q;                         // shared frontier capacity per buffer
+    int32_t cl_filter = 0;             // cluster mode: words of the per-CTA filter (0: none)
     // grid-wide mode (k_merge_grid): the whole GPU finishes the deferred rows one at a time in
     // increasing order when there are at most grid_max of them (0: never)
     int32_t grid_max = 0;
@@ -123,7 +124,7 @@ struct MergeParams {
 };
 // mode 0: one CTA per row, bitmap in shared memory; 1: one CTA, bitmap in an HBM slot;
 // 2: a cluster of g CTAs per row, bitmap sliced over their shared memories (DSMEM)
-size_t merge_smem_bytes(int n, int mode, int g, int q);
+size_t merge_smem_bytes(int n, int mode, int g, int q, bool filter = false);
 cudaError_t merge_configure(size_t smem);
 cudaError_t merge_max_clusters(int g, size_t smem, int *clusters);
 // sort list[0..min(*cnt, max)) ascending (one CTA; max <= 4096)

@@ -164,7 +164,7 @@ struct lu_sym {
     int32_t *defer_list = nullptr, *fail_list = nullptr;  // [defer_max] each
     int32_t *mspill = nullptr, *mwait = nullptr;
     uint32_t *mgbitmap = nullptr;
-    int merge_grid = 0, merge_q = 2048, merge_mode = 0, merge_g = 1;
+    int merge_grid = 0, merge_q = 2048, merge_mode = 0, merge_g = 1, merge_filter = 0;
     bool merge_smem_bm = true;
     size_t merge_smem = 0;
     bool tail_ran = false;
@@ -1005,16 +1005,20 @@ lu_status ensure_merge(lu_sym *h)
     h->merge_mode = -1;
     int max_rows = std::min(sms, h->defer_max);
     if (g > 1 && !getenv("LUSYM_MERGE_HBM_BITMAP")) {
-        const size_t sm = merge_smem_bytes(n, 2, g, h->merge_q);
-        int clusters = 0;
-        if (sm <= (size_t)smem_optin && merge_configure(sm) == cudaSuccess &&
-            merge_max_clusters(g, sm, &clusters) == cudaSuccess && clusters > 0) {
-            h->merge_mode = 2;
-            h->merge_g = g;
-            h->merge_smem = sm;
-            max_rows = std::min(clusters, h->defer_max);
+        // with the per-CTA filter of other ranks' bits when it fits (LUSYM_MERGE_NOFILTER: A/B)
+        for (int f = getenv("LUSYM_MERGE_NOFILTER") ? 0 : 1; f >= 0 && h->merge_mode < 0; --f) {
+            const size_t sm = merge_smem_bytes(n, 2, g, h->merge_q, f != 0);
+            int clusters = 0;
+            if (sm <= (size_t)smem_optin && merge_configure(sm) == cudaSuccess &&
+                merge_max_clusters(g, sm, &clusters) == cudaSuccess && clusters > 0) {
+                h->merge_mode = 2;
+                h->merge_g = g;
+                h->merge_smem = sm;
+                h->merge_filter = f ? (int)(((int64_t)n + 31) / 32) : 0;
+                max_rows = std::min(clusters, h->defer_max);
+            }
+            cudaGetLastError();
         }
-        cudaGetLastError();
     }
     if (h->merge_mode < 0) {
         h->merge_g = 1;
@@ -1136,6 +1140,7 @@ lu_status run_tail_list(lu_sym *h, int32_t *fill_count, const int32_t *list,
     mp.fail_cnt = slots + 2;
     mp.stats = slots + 3;
     mp.q = h->merge_q;
+    mp.cl_filter = h->merge_mode == 2 ? h->merge_filter : 0;
     if (h->mg_max > 0 || h->mg_head > 0) {
         // a short list: the whole grid, one row at a time (k_merge_grid); a longer one is left
         // to the clusters (the kernel checks the device-side count)

@@ -202,11 +202,32 @@ struct Bits {
         uint32_t *base = w + (gw & ((1 << sh) - 1));
         return r == rank ? base : cg::this_cluster().map_shared_rank(base, r);
     }
-    // test-and-set of bit v; true iff this call set it
+    uint32_t *filt = nullptr;  // cluster mode: bits this CTA has seen set in other ranks' words
+
+    // test-and-set of bit v; true iff this call set it.  A remote word's test first looks at
+    // the CTA's filter: bits are only ever set during a row, so a bit seen set (in a word this
+    // CTA read or set earlier) is set, and the DSMEM round trip is skipped; every remote word
+    // read or atomically modified is OR-ed into the filter.
     __device__ __forceinline__ bool tas(int v) const
     {
         const uint32_t b = 1u << (v & 31);
-        uint32_t *p = word(v >> 5);
+        const int gw = v >> 5;
+        if constexpr (CL) {
+            const int r = gw >> sh;
+            if (r != rank && filt) {
+                if (filt[gw] & b) return false;
+                uint32_t *p = cg::this_cluster().map_shared_rank(w + (gw & ((1 << sh) - 1)), r);
+                const uint32_t cur = *p;
+                if (cur & b) {
+                    atomicOr(filt + gw, cur);
+                    return false;
+                }
+                const uint32_t old = atomicOr(p, b);
+                atomicOr(filt + gw, old | b);
+                return !(old & b);
+            }
+        }
+        uint32_t *p = word(gw);
         if (*p & b) return false;
         return !(atomicOr(p, b) & b);
     }
@@ -250,6 +271,10 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
     int32_t *gq0 = p.spill + (size_t)blockIdx.x * 2 * p.spill_cap;
     int32_t *wait = p.wait + (size_t)blockIdx.x * p.list_max;
     const int tid = threadIdx.x;
+    if constexpr (CL) {
+        bm.filt = p.cl_filter ? bm.w + (1 << sh) : nullptr;
+        for (int w = tid; w < p.cl_filter; w += NT) bm.filt[w] = 0;
+    }
     const int nlist = (int)min(*p.list_cnt, (unsigned long long)p.list_max);
     if (MODE != 1)
         for (int w = bm.lo + tid; w < bm.hi; w += NT) lw[w] = 0;
@@ -553,6 +578,8 @@ __global__ void __launch_bounds__(NT, 1) k_merge_rows(const MergeParams p, int s
         // ---- fill(:) = 0 for the next row (L115)
         __syncthreads();
         for (int w = bm.lo + tid; w < bm.hi; w += NT) lw[w] = 0;
+        if constexpr (CL)
+            for (int w = tid; w < p.cl_filter; w += NT) bm.filt[w] = 0;
         // (the next claim's cluster barrier orders this before any rank's next seed)
     }
     if (tid == 0 && p.stats) {
@@ -1068,12 +1095,13 @@ cudaError_t merge_grid_launch(const MergeParams &p, int grid, cudaStream_t s)
 cudaError_t merge_configure_impl(size_t smem);
 cudaError_t merge_max_clusters_impl(int g, size_t smem, int *clusters);
 
-size_t merge_smem_bytes(int n, int mode, int g, int q)
+size_t merge_smem_bytes(int n, int mode, int g, int q, bool filter)
 {
     size_t b = kHdrBytes + (2 * (size_t)NT + kSent) * sizeof(long long) +
                2 * (size_t)q * sizeof(int32_t);
     if (mode == 0) b += (size_t)((n + 31) / 32) * sizeof(uint32_t);
     if (mode == 2) b += ((size_t)1 << cluster_shift(n, g)) * sizeof(uint32_t);
+    if (mode == 2 && filter) b += (size_t)((n + 31) / 32) * sizeof(uint32_t);
     return (b + 15) & ~(size_t)15;
 }
 
