@@ -409,6 +409,29 @@ const char *lu_status_str(lu_status s);
 /* Message of the last failing call on the calling host thread ("" if none). */
 const char *lu_last_error(void);
 
+/*
+ * Environment knobs of the symbolic phase (A/B experiments and diagnostics; none changes a
+ * result, DESIGN.md §5.1 has the measurements).  Read at lu_sym_create unless noted.
+ *   LUSYM_TIGHT_CLASSES=0     row classes by halving the shared visited map (default: the largest
+ *                             map that adds rows per SM, G5)
+ *   LUSYM_ASYNC_OCC=<k>       barrier-free BFS (bfs_async) in classes of at most k rows per SM
+ *                             (default 0: off; LU_F_ASYNC_BFS forces it); LUSYM_ASYNC_KEEP,
+ *                             LUSYM_ASYNC_SLEEP its donation threshold and idle poll (ns)
+ *                             (read once per process)
+ *   LUSYM_MERGE_GRID_HEAD=<k> the whole grid finishes the first k deferred rows (default 2),
+ *                             the clusters the rest; LUSYM_MERGE_GRID_MAX=<k> the whole list
+ *                             when it has at most k rows (default 0)
+ *   LUSYM_MERGE_CLUSTER=<g>   CTAs per deferred row in the tail (default 4; 1 = no cluster);
+ *                             LUSYM_MERGE_HBM_BITMAP, LUSYM_MERGE_NOFILTER variants
+ *   LUSYM_HEAVY_TOP=<k>       the last k rows in the shared-map class next to the sparse class
+ *                             (default 0; LUSYM_HEAVY_GRID its rows in flight) (read once)
+ *   LUSYM_DEFER_WINDOWS, LUSYM_SPARSE_DEFER_WINDOWS, LUSYM_FORCE_SPARSE, LUSYM_TOP_LBW
+ *                             deferral thresholds and planner test knobs
+ *   LUSYM_DEBUG_PLAN=1        print the row classes; LUSYM_DEBUG_CREATE=1 host time per create
+ *                             step (read once)
+ *   LUSYM_LIB=<path>          (Python binding) load another build of this library
+ */
+
 #ifdef __cplusplus
 }
 #endif
