@@ -125,12 +125,15 @@ class ClockSampler:
         self.proc = None
         self.stop = threading.Event()
         self.thread = None
+        self._nv = None
 
     def __enter__(self):
         try:
             import pynvml
             pynvml.nvmlInit()
             hd = pynvml.nvmlDeviceGetHandleByIndex(self._nvml_index())
+            self._nv = (pynvml, hd)
+            self._sample_nvml(pynvml, hd, pynvml.nvmlDeviceGetMaxClockInfo(hd, pynvml.NVML_CLOCK_SM))
             self.thread = threading.Thread(target=self._nvml, args=(pynvml, hd), daemon=True)
             self.thread.start()
             return self
@@ -156,15 +159,18 @@ class ClockSampler:
             return int(ids[self.index])
         return self.index
 
+    def _sample_nvml(self, pynvml, hd, mx):
+        try:
+            c = pynvml.nvmlDeviceGetClockInfo(hd, pynvml.NVML_CLOCK_SM)
+            r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(hd)
+            self.samples.append((float(c), float(mx), int(r), not (r & 1)))
+        except Exception:
+            pass
+
     def _nvml(self, pynvml, hd):
         mx = pynvml.nvmlDeviceGetMaxClockInfo(hd, pynvml.NVML_CLOCK_SM)
         while not self.stop.is_set():
-            try:
-                c = pynvml.nvmlDeviceGetClockInfo(hd, pynvml.NVML_CLOCK_SM)
-                r = pynvml.nvmlDeviceGetCurrentClocksEventReasons(hd)
-                self.samples.append((float(c), float(mx), int(r), not (r & 1)))
-            except Exception:
-                pass
+            self._sample_nvml(pynvml, hd, mx)
             self.stop.wait(self.PERIOD_S)
 
     def _read(self):
@@ -178,6 +184,9 @@ class ClockSampler:
                 continue
 
     def __exit__(self, *a):
+        if getattr(self, "_nv", None):  # one reading at the end of the region too (sub-ms regions)
+            pynvml, hd = self._nv
+            self._sample_nvml(pynvml, hd, pynvml.nvmlDeviceGetMaxClockInfo(hd, pynvml.NVML_CLOCK_SM))
         self.stop.set()
         if self.proc is not None:
             self.proc.terminate()
