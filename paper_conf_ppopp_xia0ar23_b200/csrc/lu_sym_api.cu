@@ -384,7 +384,7 @@ lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out,
     // register budget (chosen on a tie, i.e. when shared memory allows one CTA per SM anyway)
     // (64: only on request — a sparse class or threads_per_row = 64)
     const int nts[6] = {64, 128, 256, 512, 1024, 1025};
-    const int qs[5] = {256, 512, 1024, 2048, 4096};
+    const int qs[6] = {128, 256, 512, 1024, 2048, 4096};
     Cfg best = {0, 0, 0, 0, -1};
     for (int a = 0; a < 6; ++a) {
         const int nt = nts[a];
@@ -392,7 +392,7 @@ lu_status best_cfg(lu_sym *h, int smem_words, int vis, int smem_optin, Cfg *out,
         if (tpr > 0 && nt != tpr && !(tpr == 1024 && nt == 1025)) continue;
         if (tpr <= 0 && nt == 64) continue;
         const int threads = nt > 1024 ? 1024 : nt;
-        for (int b = 0; b < 5; ++b) {
+        for (int b = 0; b < 6; ++b) {
             if (qs[b] < min_q && h->opts.queue_capacity <= 0) continue;
             int q = h->opts.queue_capacity > 0 ? h->opts.queue_capacity : qs[b];
             if (h->opts.queue_capacity > 0 && b > 0) break;
@@ -624,7 +624,12 @@ lu_status plan(lu_sym *h)
         // measured slower on cfg3 than no shared visited words: 148/153/185 ms against 146 —
         // the window costs rows per SM, profiles/r02/ab_window.log)
         Cfg g;
-        if ((st = best_cfg(h, 0, kVisGlobal, smem_optin, &g, 64, 256)) != LU_OK) return st;
+        // 128-entry queues: the shared header, summary and queues of a 64-thread CTA then take
+        // 6 KB and 32 rows fit an SM (28 with 256 entries): cfg3 count 130 -> 124 ms
+        // (profiles/r02/sparse_minq.log; LUSYM_SPARSE_MINQ: A/B knob)
+        const char *mq = getenv("LUSYM_SPARSE_MINQ");
+        if ((st = best_cfg(h, 0, kVisGlobal, smem_optin, &g, 64, mq ? atoi(mq) : 128)) != LU_OK)
+            return st;
         size_t kc = 0;
         // candidates: the classes (from the top) with fewer rows per SM than the sparse class,
         // considered only when the top class's shared map holds it below 8 rows per SM
