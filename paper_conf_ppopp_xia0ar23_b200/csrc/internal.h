@@ -241,7 +241,8 @@ struct LevelizeScratch {
     int64_t *lt_fill = nullptr; // [n] scatter cursors
     int64_t *scan_blk = nullptr;
     int32_t *ctrl = nullptr;    // device control block
-    int32_t *chain = nullptr;   // [8n] J0 D0 J1 D1 nxt tail len best
+    int32_t *chain = nullptr;   // [12n] J0 D0 J1 D1 nxt tail len best, then 16n bytes of
+                                // per-head successor ranges
     int32_t n_cap = 0;
     int64_t lt_cap = 0;
 };

@@ -209,9 +209,11 @@ __global__ void __launch_bounds__(256) k_rank(int32_t n, int32_t *J0, int32_t *D
     if (t0 == 0) *rounds_out = r + 1;
 }
 
-// per chain: tail and length (stored at the head)
+// per chain: tail and length (stored at the head), and the tail's successor range, so that
+// relaxing a head is one 16-byte load away from its successor list (no tail -> range chain)
 __global__ void k_chain_info(int32_t n, const int32_t *J, const int32_t *D, const int32_t *nxt,
-                             int32_t *tail, int32_t *len)
+                             const int64_t *us, const int64_t *ue, int32_t *tail, int32_t *len,
+                             longlong2 *hu)
 {
     const int v = blockIdx.x * blockDim.x + threadIdx.x;
     if (v >= n) return;
@@ -219,6 +221,7 @@ __global__ void k_chain_info(int32_t n, const int32_t *J, const int32_t *D, cons
         const int h = J[v];
         tail[h] = v;
         len[h] = D[v] + 1;
+        hu[h] = make_longlong2(us[v], ue[v]);
     }
 }
 
@@ -248,6 +251,7 @@ struct KahnArgs {
     const int64_t *ltp;
     const int32_t *lti;
     const int32_t *tail, *len;
+    const longlong2 *hu;  // [n] per head: successor range of its chain's tail
     int32_t *indeg, *best, *queue;  // queue: 2 x n
     int32_t *ctrl;
     int32_t narrow_max;
@@ -261,9 +265,9 @@ template <class Push>
 __device__ __forceinline__ void relax(const KahnArgs &A, int h, Push &&push)
 {
     const int lane = threadIdx.x & 31;
-    const int t = A.tail[h];
+    const longlong2 r = A.hu[h];                    // the tail's successor range
     const int lvl = __ldcg(A.best + h) + A.len[h];  // level of every successor via this chain
-    const int64_t a = A.us[t], b = A.ue[t];
+    const int64_t a = r.x, b = r.y;
     for (int64_t eb = a; eb < b; eb += 32) {
         const int64_t e = eb + lane;
         bool z = false;
@@ -276,6 +280,7 @@ __device__ __forceinline__ void relax(const KahnArgs &A, int h, Push &&push)
         push(z, v);
     }
     if (A.ltp) {
+        const int t = A.tail[h];
         const int64_t c = A.ltp[t], d = A.ltp[t + 1];
         for (int64_t eb = c; eb < d; eb += 32) {
             const int64_t e = eb + lane;
@@ -442,11 +447,12 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
         LV_CK(dev_alloc((void **)&s.lt_fill, sizeof(int64_t) * n, st));
         LV_CK(dev_alloc((void **)&s.scan_blk, sizeof(int64_t) * scan_scratch_elems(n), st));
         LV_CK(dev_alloc((void **)&s.ctrl, sizeof(int32_t) * kCtrlInts, st));
-        LV_CK(dev_alloc((void **)&s.chain, sizeof(int32_t) * 8 * (size_t)n, st));
+        LV_CK(dev_alloc((void **)&s.chain, sizeof(int32_t) * 12 * (size_t)n, st));
         s.n_cap = n;
     }
     int32_t *J0 = s.chain, *D0 = J0 + n, *J1 = D0 + n, *D1 = J1 + n, *nxt = D1 + n;
     int32_t *tail = nxt + n, *len = tail + n, *best = len + n;
+    longlong2 *hu = reinterpret_cast<longlong2 *>(best + n);  // 16 n bytes, 16-B aligned
     const bool glu3 = rule == 1;
     const int g = aux_grid(n);
     const int gt = (n + 255) / 256;
@@ -508,7 +514,7 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
         LV_CK(cudaLaunchCooperativeKernel((const void *)k_rank, grid, 256, args, 0, st));
         info->launches += 1;
     }
-    k_chain_info<<<gt, 256, 0, st>>>(n, J0, D0, nxt, tail, len);
+    k_chain_info<<<gt, 256, 0, st>>>(n, J0, D0, nxt, s.ustart, s.uend, tail, len, hu);
     LV_CK(cudaGetLastError());
     // cons_queue (round 0)
     k_init_queue<<<gt, 256, 0, st>>>(n, s.indeg, J0, best, s.queue, s.ctrl);
@@ -531,6 +537,7 @@ cudaError_t levelize_run(int32_t n, const int64_t *rp_lu, const int32_t *ci_lu, 
     A.lti = lti;
     A.tail = tail;
     A.len = len;
+    A.hu = hu;
     A.indeg = s.indeg;
     A.best = best;
     A.queue = s.queue;
