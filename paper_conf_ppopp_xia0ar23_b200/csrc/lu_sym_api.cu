@@ -1005,7 +1005,10 @@ lu_status ensure_merge(lu_sym *h)
     const int n = h->n;
     // a cluster of G CTAs per deferred row (bitmap sliced over their shared memories), else
     // one CTA with the bitmap in shared memory, else in an HBM slot
-    int g = 4;
+    // 8 CTAs: with the first two rows on the whole grid, the tail's critical path is one
+    // hub's closure on its cluster (cfg3 tail 14.7 ms with 4, 12.4 with 8, 15.0 with 16;
+    // profiles/r02/merge_cluster_size.log)
+    int g = 8;
     if (const char *e = getenv("LUSYM_MERGE_CLUSTER")) g = atoi(e);  // A/B knob; 1 = no cluster
     h->merge_mode = -1;
     int max_rows = std::min(sms, h->defer_max);

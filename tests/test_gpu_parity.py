@@ -512,7 +512,7 @@ def test_deferred_rows_row_merge_tail(knob):
 
 
 @pytest.mark.parametrize("variant", [("LUSYM_MERGE_HBM_BITMAP", "1"), ("LUSYM_MERGE_CLUSTER", "1"),
-                                     ("LUSYM_MERGE_CLUSTER", "2"), ("LUSYM_MERGE_CLUSTER", "8"),
+                                     ("LUSYM_MERGE_CLUSTER", "2"), ("LUSYM_MERGE_CLUSTER", "4"),
                                      ("LUSYM_MERGE_CLUSTER", "16"),
                                      ("LUSYM_MERGE_GRID_MAX", "100000"),
                                      ("LUSYM_MERGE_GRID_HEAD", "0"),
@@ -520,7 +520,7 @@ def test_deferred_rows_row_merge_tail(knob):
 def test_deferred_rows_tail_variants(monkeypatch, variant):
     """The tail's bitmap placements: one CTA per row with an HBM slot or a shared-memory
     bitmap, and clusters of 2/8/16 CTAs with the bitmap sliced over distributed shared memory
-    (the default is 4); and the grid-wide mode (k_merge_grid) for every list however long, for
+    (the default is 8); and the grid-wide mode (k_merge_grid) for every list however long, for
     none of the rows, or for the first 7 (the default gives it the first 2)."""
     monkeypatch.setenv(*variant)
     for rp, ci in (_hub_matrix(), gen.circuit(40, 2), gen.lap2d(24)):
