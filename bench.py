@@ -60,7 +60,7 @@ def parse():
                     help="configs measured after the headline one (N=1 line's per_config block); "
                          "'' = none")
     ap.add_argument("--per-config-steps", type=int, default=3)
-    ap.add_argument("--per-config-warmup", type=int, default=3)
+    ap.add_argument("--per-config-warmup", type=int, default=5)
     ap.add_argument("--no-verify", action="store_true",
                     help="skip the parity check of every timed output (never for reported runs)")
     ap.add_argument("--apriori-partition", action="store_true",
