@@ -1164,8 +1164,14 @@ lu_status run_tail_list(lu_sym *h, int32_t *fill_count, const int32_t *list,
         mp.gpart = h->mg_ll + 4 * n + 64;
         mp.gctrl = h->mg_ctrl;
         mp.grid_filter = h->mg_filter;
-        CK(merge_grid_launch(mp, h->mg_grid, s));
-        h->launches += 1;
+        if (merge_grid_launch(mp, h->mg_grid, s) == cudaSuccess) {
+            h->launches += 1;
+        } else {
+            // a cooperative launch that cannot be made (e.g. a shared GPU): the clusters, whose
+            // claims then start at the first row, take the whole list
+            cudaGetLastError();
+            h->mg_max = h->mg_head = 0;
+        }
     }
     CK(merge_launch(mp, h->merge_mode, h->merge_g, h->merge_grid, h->merge_smem, s));
     h->launches += 2;
